@@ -1,0 +1,197 @@
+"""MAGIS schedule-evaluation ORACLE -- TEST INFRASTRUCTURE ONLY.
+
+A plain, slow, single-threaded CPU implementation of what the B200 path
+computes (§2.1, §5.2, §6.2, Alg. 3
+BetterThan P:1689-1692).  It shares no code with the CUDA path and must only
+be imported by ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
+``cpu_baseline`` / ``--impl reference`` legs.
+
+Pins (tests/test_oracle_*.py): Fig. 2(a) = 1056, Fig. 2(b) = 96
+(P:469-476), hand-computed toys T1/T2, closed forms, brute-force
+enumeration of all topological orders against an independently written
+interval formula, invariants, Eq. (1) = 98/56/52.
+
+Parity status per function:
+  * peak / status / argmax ....... pinned (paper numbers + brute force)
+  * swap-free latency ............ pinned (closed form P:406-408)
+  * swap latency (queues) ........ parity unpinned by the paper (reading P7);
+                                   pinned only by hand-computed toys T1
+  * pareto / best ................ pinned (definition, brute-force dominance)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "magis_oracle.c")
+_LIB = os.path.join(_HERE, "libmagis_oracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile the C oracle with gcc (plain -O2, no vectorisation tricks)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-std=c99", "-shared", "-fPIC", "-o", _LIB, _SRC, "-lm"])
+    return _LIB
+
+
+def _load():
+    global _lib
+    if _lib is not None:
+        return _lib
+    build()
+    lib = ctypes.CDLL(_LIB)
+    P = ctypes.c_void_p
+    lib.orc_graph_new.restype = P
+    lib.orc_graph_new.argtypes = [ctypes.c_int32, P, P, P, ctypes.c_int64, P, P, ctypes.c_int32,
+                                  P, P, P, ctypes.c_double, ctypes.c_double]
+    lib.orc_graph_free.argtypes = [P]
+    lib.orc_graph_n_total.restype = ctypes.c_int32
+    lib.orc_graph_n_total.argtypes = [P]
+    lib.orc_graph_n_edges.restype = ctypes.c_int64
+    lib.orc_graph_n_edges.argtypes = [P]
+    lib.orc_eval.argtypes = [P, P, P, P, P, P, P]
+    lib.orc_eval_batch.argtypes = [P, ctypes.c_int64, P, P, P, P, P]
+    lib.orc_pareto.restype = ctypes.c_int64
+    lib.orc_pareto.argtypes = [ctypes.c_int64, P, P, P, P, P]
+    lib.orc_best_mem.restype = ctypes.c_int64
+    lib.orc_best_mem.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_int64]
+    lib.orc_best_lat.restype = ctypes.c_int64
+    lib.orc_best_lat.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_double]
+    _lib = lib
+    return lib
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+class OracleGraph:
+    """Graph G = (V, E) with size(v), cost(v), outs(G) (Table 1),
+    plus the eligible tensors t_r with their late-user sets U_r (reading P6)
+    and the swap link model (bytes/s, latency; reading P7)."""
+
+    def __init__(self, size, cost, is_output, src, dst, elig=(), U=(),
+                 swap_Bps: float = 25e9, swap_lat: float = 1e-5):
+        self._lib = _load()
+        self.size = np.ascontiguousarray(size, dtype=np.int64)
+        self.cost = np.ascontiguousarray(cost, dtype=np.float64)
+        self.n = int(self.size.shape[0])
+        self.is_output = np.ascontiguousarray(is_output, dtype=np.uint8)
+        self.src = np.ascontiguousarray(src, dtype=np.int32)
+        self.dst = np.ascontiguousarray(dst, dtype=np.int32)
+        self.elig = np.ascontiguousarray(elig, dtype=np.int32).reshape(-1)
+        self.R = int(self.elig.shape[0])
+        U = list(U)
+        assert len(U) == self.R
+        ptr = np.zeros(self.R + 1, dtype=np.int64)
+        for r, u in enumerate(U):
+            ptr[r + 1] = ptr[r] + len(u)
+        self.U_ptr = ptr
+        self.U_idx = np.ascontiguousarray(np.concatenate([np.asarray(u, dtype=np.int32) for u in U])
+                                          if self.R else np.zeros(0, np.int32), dtype=np.int32)
+        self.swap_Bps = float(swap_Bps)
+        self.swap_lat = float(swap_lat)
+        h = self._lib.orc_graph_new(self.n, _ptr(self.size), _ptr(self.cost), _ptr(self.is_output),
+                                    int(self.src.shape[0]), _ptr(self.src), _ptr(self.dst), self.R,
+                                    _ptr(self.elig), _ptr(self.U_ptr), _ptr(self.U_idx),
+                                    self.swap_Bps, self.swap_lat)
+        if not h:
+            raise ValueError("oracle: malformed graph")
+        self._h = h
+        self.n_total = int(self._lib.orc_graph_n_total(h))
+        self.n_edges = int(self._lib.orc_graph_n_edges(h))
+
+    @classmethod
+    def from_workload(cls, wl):
+        """Build from a magis_inputs.Workload (input generator output)."""
+        return cls(wl.size, wl.cost, wl.is_output, wl.src, wl.dst, wl.elig, wl.U,
+                   wl.swap_Bps, wl.swap_lat)
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h:
+            self._lib.orc_graph_free(h)
+            self._h = None
+
+    def eval(self, perm, dec=None):
+        """-> (status, peak, latency, argmax_step) for one candidate."""
+        perm = np.ascontiguousarray(perm, dtype=np.int32)
+        assert perm.shape == (self.n_total,)
+        if dec is None:
+            dec = np.zeros(max(self.R, 1), dtype=np.uint8)
+        dec = np.ascontiguousarray(dec, dtype=np.uint8)
+        st = np.zeros(1, np.uint8)
+        pk = np.zeros(1, np.int64)
+        lt = np.zeros(1, np.float64)
+        am = np.zeros(1, np.int64)
+        self._lib.orc_eval(self._h, _ptr(perm), _ptr(dec), _ptr(st), _ptr(pk), _ptr(lt), _ptr(am))
+        return int(st[0]), int(pk[0]), float(lt[0]), int(am[0])
+
+    def eval_batch(self, perms, decs=None):
+        """perms: (K, n_total) int32; decs: (K, R) uint8 -> (status, peak, lat) arrays."""
+        perms = np.ascontiguousarray(perms, dtype=np.int32)
+        K = perms.shape[0]
+        assert perms.shape[1] == self.n_total
+        if decs is None or self.R == 0:
+            decs = np.zeros((K, max(self.R, 1)), dtype=np.uint8)
+        decs = np.ascontiguousarray(decs, dtype=np.uint8)
+        st = np.zeros(K, np.uint8)
+        pk = np.zeros(K, np.int64)
+        lt = np.zeros(K, np.float64)
+        self._lib.orc_eval_batch(self._h, K, _ptr(perms), _ptr(decs), _ptr(st), _ptr(pk), _ptr(lt))
+        return st, pk, lt
+
+
+def pareto(peak, lat, status, ids=None):
+    """Indices of the Pareto front (ascending peak), by brute-force dominance."""
+    lib = _load()
+    peak = np.ascontiguousarray(peak, dtype=np.int64)
+    lat = np.ascontiguousarray(lat, dtype=np.float64)
+    status = np.ascontiguousarray(status, dtype=np.uint8)
+    n = peak.shape[0]
+    ids = np.arange(n, dtype=np.int64) if ids is None else np.ascontiguousarray(ids, dtype=np.int64)
+    out = np.zeros(max(n, 1), np.int64)
+    nf = lib.orc_pareto(n, _ptr(peak), _ptr(lat), _ptr(status), _ptr(ids), _ptr(out))
+    return out[:nf].copy()
+
+
+def best_under_memory(peak, lat, status, M, ids=None):
+    """Alg. 3 BetterThan-best under memory limit M -> index or -1."""
+    lib = _load()
+    peak = np.ascontiguousarray(peak, dtype=np.int64)
+    lat = np.ascontiguousarray(lat, dtype=np.float64)
+    status = np.ascontiguousarray(status, dtype=np.uint8)
+    n = peak.shape[0]
+    ids = np.arange(n, dtype=np.int64) if ids is None else np.ascontiguousarray(ids, dtype=np.int64)
+    return int(lib.orc_best_mem(n, _ptr(peak), _ptr(lat), _ptr(status), _ptr(ids), int(M)))
+
+
+def best_under_latency(peak, lat, status, L, ids=None):
+    """Second optimisation mode: best under latency limit L."""
+    lib = _load()
+    peak = np.ascontiguousarray(peak, dtype=np.int64)
+    lat = np.ascontiguousarray(lat, dtype=np.float64)
+    status = np.ascontiguousarray(status, dtype=np.uint8)
+    n = peak.shape[0]
+    ids = np.arange(n, dtype=np.int64) if ids is None else np.ascontiguousarray(ids, dtype=np.int64)
+    return int(lib.orc_best_lat(n, _ptr(peak), _ptr(lat), _ptr(status), _ptr(ids), float(L)))
+
+
+def eq1_estimate(H, S, I, size, n):
+    """Eq. (1): M_f ~= sum_{(H\\S) u I} |v| + sum_{H n S} |v| / n.
+
+    H, S, I are collections of node ids; size maps id -> bytes.  Returns a
+    float (the paper's estimate; it is an approximation, reading P16)."""
+    H, S, I = set(H), set(S), set(I)
+    outside = (H - S) | I
+    return float(sum(size[v] for v in outside)) + sum(size[v] for v in (H & S)) / float(n)
+
+
+def eq1_m0(H, size):
+    """M_0 = sum_{v in H} |v| (Eq. (1))."""
+    return float(sum(size[v] for v in set(H)))

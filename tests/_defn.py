@@ -1,0 +1,143 @@
+"""Independent definitional evaluators used to PIN the oracle (tests only).
+
+These are written from the paper's formulas directly, in a different style
+from the C oracle (sets and interval sums instead of event/free lists), so a
+plausible slip in either shows up as a mismatch:
+
+* ``interval_peak``: M_i = sum_{u : S_u < i <= F_u} |u| (P:409-424 with the
+  1-based S_j = j-1 and the corrected strict inequality, reading P1), written
+  as an O(n^2) double loop over steps and tensors.
+* ``literal_peak``: the same with the literal, garbled S_j <= i <= F_j
+   -- used to show that the text's 1056 needs reading P1.
+* ``all_topo_orders``: brute-force enumeration of every topological order.
+"""
+from __future__ import annotations
+
+import itertools
+
+
+def succ_map(n, edges):
+    s = {v: set() for v in range(n)}
+    for u, v in edges:
+        s[u].add(v)
+    return s
+
+
+def intervals(order, edges, outputs):
+    """1-based S/F per paper: S_j = j-1, F_j = max_{v_k in suc(v_j)} k;
+    outputs live to n; no successors -> F_j = j (own step)."""
+    n = len(order)
+    step = {v: i + 1 for i, v in enumerate(order)}  # 1-based timestamps
+    suc = {}
+    for u, v in edges:
+        suc.setdefault(u, set()).add(v)
+    S, F = {}, {}
+    for v in order:
+        S[v] = step[v] - 1
+        if v in outputs:
+            F[v] = n
+        elif suc.get(v):
+            F[v] = max(step[w] for w in suc[v])
+        else:
+            F[v] = step[v]
+    return S, F
+
+
+def interval_peak(order, edges, size, outputs):
+    """max_i sum |u| over u with S_u < i <= F_u  (reading P1)."""
+    S, F = intervals(order, edges, outputs)
+    n = len(order)
+    best, arg = None, None
+    for i in range(1, n + 1):
+        m = sum(size[u] for u in order if S[u] < i <= F[u])
+        if best is None or m > best:
+            best, arg = m, i - 1
+    return best, arg
+
+
+def literal_peak(order, edges, size, outputs):
+    """Literal P:416 form S_j <= i <= F_j (garbled by one step)."""
+    S, F = intervals(order, edges, outputs)
+    n = len(order)
+    return max(sum(size[u] for u in order if S[u] <= i <= F[u]) for i in range(1, n + 1))
+
+
+def all_topo_orders(n, edges):
+    pre = {v: set() for v in range(n)}
+    for u, v in edges:
+        pre[v].add(u)
+    out = []
+
+    def rec(done, order):
+        if len(order) == n:
+            out.append(list(order))
+            return
+        for v in range(n):
+            if v not in done and pre[v] <= done:
+                done.add(v)
+                order.append(v)
+                rec(done, order)
+                order.pop()
+                done.remove(v)
+
+    rec(set(), [])
+    return out
+
+
+def is_topo(order, edges):
+    p = {v: i for i, v in enumerate(order)}
+    return all(p[u] < p[v] for u, v in edges)
+
+
+def transformed(n, edges, elig, U, dec):
+    """Fig. 8 rule semantics on an explicit edge set (reading P6); returns
+    (active node list, edge set, bytes map builder info)."""
+    edges = set(map(tuple, edges))
+    R = len(elig)
+    out = set()
+    moved = {}
+    for r in range(R):
+        for b in U[r]:
+            moved[(elig[r], b)] = r
+    for (u, v) in edges:
+        r = moved.get((u, v))
+        if r is not None and dec[r] == 1:
+            out.add((n + 3 * r, v))
+        elif r is not None and dec[r] == 2:
+            out.add((n + 3 * r + 2, v))
+        else:
+            out.add((u, v))
+    for r in range(R):
+        t = elig[r]
+        if dec[r] == 1:
+            for (u, v) in edges:
+                if v == t:
+                    out.add((u, n + 3 * r))
+        elif dec[r] == 2:
+            out.add((t, n + 3 * r + 1))
+            out.add((n + 3 * r + 1, n + 3 * r + 2))
+    active = set(range(n))
+    for r in range(R):
+        if dec[r] == 1:
+            active.add(n + 3 * r)
+        if dec[r] == 2:
+            active |= {n + 3 * r + 1, n + 3 * r + 2}
+    return active, out
+
+
+def defn_eval(n, edges, size, outputs, elig, U, dec, perm):
+    """Interval-sum peak on the transformed graph (no latency)."""
+    active, te = transformed(n, edges, elig, U, dec)
+    pos = {v: i for i, v in enumerate(perm)}
+    if any(pos[u] >= pos[v] for u, v in te):
+        return 2, -1
+    order = [v for v in perm if v in active]
+    sz = {}
+    for v in order:
+        if v < n:
+            sz[v] = size[v]
+        else:
+            r, k = divmod(v - n, 3)
+            sz[v] = 0 if k == 1 else size[elig[r]]
+    pk, _ = interval_peak(order, te, sz, set(outputs))
+    return 0, pk
