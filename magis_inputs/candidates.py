@@ -1,0 +1,101 @@
+"""Seeded candidate schedules (perm + decisions) -- INPUT GENERATION ONLY.
+
+Python front end of csrc/candgen.c (recipe in its header and DESIGN.md
+§Inputs).  Candidates depend only on (seed, global id), never on sharding.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from dataclasses import dataclass
+
+import numpy as np
+
+from .graph import Workload
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "csrc", "candgen.c")
+_LIB = os.path.join(_HERE, "csrc", "libcandgen.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-std=gnu99", "-shared", "-fPIC", "-o", _LIB, _SRC,
+                               "-lpthread"])
+    return _LIB
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        build()
+        lib = ctypes.CDLL(_LIB)
+        P = ctypes.c_void_p
+        i32, i64, u64 = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64
+        lib.candgen.argtypes = [i32, i32, P, P, P, P, P, P, P, u64, i32, i32, i32, i32, i32, i32,
+                                u64, i64, P, P, i32]
+        lib.candgen.restype = None
+        _lib = lib
+    return _lib
+
+
+@dataclass
+class CandidateSpec:
+    """Candidate mix: 75% random topo orders, 24% local moves,
+    1% random transposition; P(remat) = P(swap) = 5% per eligible tensor;
+    windows <= 64; Load/clone slack 0-8 steps."""
+    seed: int = 1
+    pct_random: int = 75
+    pct_local: int = 24
+    p_remat: int = 500      # per 10000
+    p_swap: int = 500       # per 10000
+    wmax: int = 64
+    slack: int = 8
+
+
+def csr(n: int, src: np.ndarray, dst: np.ndarray):
+    """Deduplicated successor / predecessor CSR (both sorted)."""
+    if src.size:
+        key = np.unique(src.astype(np.int64) * n + dst.astype(np.int64))
+        s = (key // n).astype(np.int32)
+        d = (key % n).astype(np.int32)
+    else:
+        s = d = np.zeros(0, np.int32)
+    sp = np.zeros(n + 1, np.int64)
+    np.add.at(sp, s.astype(np.int64) + 1, 1)
+    sp = np.cumsum(sp)
+    order = np.lexsort((s, d))
+    pp = np.zeros(n + 1, np.int64)
+    np.add.at(pp, d.astype(np.int64) + 1, 1)
+    pp = np.cumsum(pp)
+    return sp, d.copy(), pp, s[order].copy()
+
+
+class CandidateGenerator:
+    def __init__(self, wl: Workload, spec: CandidateSpec | None = None):
+        self.wl = wl
+        self.spec = spec or CandidateSpec()
+        self.succ_ptr, self.succ_idx, self.pred_ptr, self.pred_idx = csr(wl.n, wl.src, wl.dst)
+        self.U_ptr, self.U_idx = wl.U_arrays()
+        self.elig = np.ascontiguousarray(wl.elig, np.int32)
+
+    def generate(self, id0: int, K: int, nthreads: int | None = None, out=None):
+        """-> (perms int32 [K, n_total], decs uint8 [K, max(R,1)])."""
+        lib = _load()
+        wl, sp = self.wl, self.spec
+        NT = wl.n_total
+        if out is None:
+            perms = np.empty((K, NT), np.int32)
+            decs = np.zeros((K, max(wl.R, 1)), np.uint8)
+        else:
+            perms, decs = out
+        if nthreads is None:
+            nthreads = max(1, min(os.cpu_count() or 1, 64))
+        p = lambda a: a.ctypes.data_as(ctypes.c_void_p)
+        lib.candgen(wl.n, wl.R, p(self.succ_ptr), p(self.succ_idx), p(self.pred_ptr), p(self.pred_idx),
+                    p(self.elig), p(self.U_ptr), p(self.U_idx), ctypes.c_uint64(sp.seed),
+                    sp.pct_random, sp.pct_local, sp.p_remat, sp.p_swap, sp.wmax, sp.slack,
+                    ctypes.c_uint64(id0), K, p(perms), p(decs), int(nthreads))
+        return perms, decs
