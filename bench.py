@@ -1,0 +1,362 @@
+#!/usr/bin/env python
+"""Benchmark: batched MAGIS schedule evaluation on B200 (BASELINE.json metric).
+
+One step = one pass of the whole hot path over one batch of K synthetic
+candidates resident in HBM: magis_eval_schedules (inverse permutation ->
+validity -> last use -> alloc/free events -> scan/max -> latency) + the local
+Pareto front (magis_pareto_merge) + at N > 1 the all-gather of the fronts and
+the global merge.  Weak scaling: every rank scores its own K candidates
+(global ids [rank*K, (rank+1)*K)).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl magis|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "candidate schedules evaluated/sec (op-steps/s) at 1/2/4/8 B200; % HBM roofline"
+UNIT = "candidates/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c2", help="c2 (default, BASELINE configs[1]), c3, c4, c5")
+    ap.add_argument("--K", type=int, default=0, help="candidates per rank (default: the config's K)")
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--cap", type=int, default=4096)
+    ap.add_argument("--impl", default="magis", choices=["magis", "reference"])
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU-baseline wall time")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------- oracle pool --
+_WL = None
+
+
+def _pool_init(arrays):
+    global _WL
+    _WL = arrays
+
+
+def _oracle_chunk(args):
+    perms, decs = args
+    import oracle
+    size, cost, iso, src, dst, elig, U, B, lam = _WL
+    g = oracle.OracleGraph(size, cost, iso, src, dst, elig, U, B, lam)
+    t = time.perf_counter()
+    st, pk, lt = g.eval_batch(perms, decs)
+    return st, pk, lt, time.perf_counter() - t
+
+
+def oracle_pool_eval(pool, perms, decs, ncores):
+    parts = np.array_split(np.arange(len(perms)), ncores * 4)
+    jobs = [(perms[p], decs[p]) for p in parts if len(p)]
+    t = time.perf_counter()
+    res = pool.map(_oracle_chunk, jobs)
+    wall = time.perf_counter() - t
+    st = np.concatenate([r[0] for r in res])
+    pk = np.concatenate([r[1] for r in res])
+    lt = np.concatenate([r[2] for r in res])
+    return st, pk, lt, wall
+
+
+# ------------------------------------------------------------------- clocks --
+REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+           0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+           0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+
+class ClockSampler:
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active",
+                 "--format=csv,noheader,nounits", "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL,
+                text=True)
+            self.thr = threading.Thread(target=self._read, daemon=True)
+            self.thr.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 3:
+                try:
+                    self.rows.append((float(parts[0]), float(parts[1]), int(parts[2], 16)))
+                except ValueError:
+                    pass
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm = statistics.median(r[0] for r in self.rows)
+        mx = max(r[1] for r in self.rows)
+        mask = 0
+        for r in self.rows:
+            mask |= r[2]
+        reasons = [name for bit, name in REASONS.items() if mask & bit and name != "gpu_idle"]
+        return {"sm_mhz": sm, "sm_max_mhz": mx, "reasons": reasons, "samples": len(self.rows)}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json copy bandwidth)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic(config: str):
+    """dram read+write bytes per eval launch from the committed ncu capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            return json.load(f).get(config)
+    except Exception:
+        return None
+
+
+# -------------------------------------------------------------------- main --
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus != world and world > 1:
+        print(f"warning: --gpus {args.gpus} != WORLD_SIZE {world}", file=sys.stderr)
+
+    from magis_inputs import CONFIGS, CandidateGenerator, CandidateSpec, build_workload
+    cfg = args.config.lower()
+    K = args.K or CONFIGS[cfg]["K"]
+    if cfg == "c5" and not args.K:
+        K = 65536          # C5's 1M local moves are evaluated in 16 chunks of 64k; one chunk per step
+
+    ncores = os.cpu_count() or 1
+    pool = None
+    need_pool = (args.impl == "reference" and rank == 0) or (
+        args.impl == "magis" and rank == 0 and world == 1 and not args.no_cpu_baseline)
+    wl = build_workload(cfg)
+    if need_pool:
+        import multiprocessing as mp
+        arrays = (wl.size, wl.cost, wl.is_output, wl.src, wl.dst, wl.elig, wl.U, wl.swap_Bps, wl.swap_lat)
+        pool = mp.get_context("fork").Pool(ncores, initializer=_pool_init, initargs=(arrays,))
+
+    workload = {"workload": f"{cfg}: {CONFIGS[cfg]['desc']}", "graph": wl.name, "n_nodes": wl.n,
+                "n_edges": wl.n_edges, "R": wl.R, "n_total": wl.n_total, "K_per_rank": K,
+                "candidates": "75% random topo orders, 24% local moves (w<=64), 1% transposition; "
+                              "P(remat)=P(swap)=5%", "seed": args.seed}
+
+    if args.impl == "reference":
+        return run_reference(args, wl, K, workload, pool, ncores, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_asplos_chend0zll024_b200 import Graph, pareto_merge
+    from paper_conf_asplos_chend0zll024_b200.distributed import global_front
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    # --- inputs: generated (seeded, shard-independent) and made resident in HBM
+    t0 = time.perf_counter()
+    gen = CandidateGenerator(wl, CandidateSpec(seed=args.seed))
+    Ph, Dh = gen.generate(rank * K, K)
+    gen_s = time.perf_counter() - t0
+    Ph_t = torch.from_numpy(Ph).pin_memory()
+    Dh_t = torch.from_numpy(Dh).pin_memory()
+    P = Ph_t.to(dev)
+    D = Dh_t.to(dev)
+    t0 = time.perf_counter()
+    g = Graph.from_workload(wl, device=local)
+    load_s = time.perf_counter() - t0
+    R, NT = g.R, g.n_total
+    stream = torch.cuda.current_stream()
+    st = torch.empty(K, dtype=torch.uint8, device=dev)
+    pk = torch.empty(K, dtype=torch.int64, device=dev)
+    lt = torch.empty(K, dtype=torch.float64, device=dev)
+    ws = torch.empty(max(1, __import__("paper_conf_asplos_chend0zll024_b200").pareto_workspace_size(max(K, world * args.cap))),
+                     dtype=torch.uint8, device=dev)
+    mem_limit = int(wl.size.sum() // 8)
+
+    def step(ev_pair=None):
+        if ev_pair:
+            ev_pair[0].record(stream)
+        g.eval_schedules(P, D if R else None, st, pk, lt, stream=stream)
+        if ev_pair:
+            ev_pair[1].record(stream)
+        fr = pareto_merge(pk, lt, st, id_base=rank * K, cap=args.cap, mem_limit=mem_limit,
+                          lat_limit=float(wl.cost.sum() * 1.05), workspace=ws, stream=stream)
+        if world > 1:
+            fr = global_front(fr, args.cap, mem_limit, float(wl.cost.sum() * 1.05))
+        return fr
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        start.record(stream)
+        for i in range(args.steps):
+            fr = step(evs[i])
+        end.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    ms = start.elapsed_time(end)
+    kern_ms = [a.elapsed_time(b) for a, b in evs]
+    front_n = int(fr["front_n"].item())
+    t = torch.tensor([ms, max(kern_ms), statistics.mean(kern_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max, _, kern_avg = t.tolist()
+    ms_per_step = ms_max / args.steps
+    value = world * K / (ms_per_step / 1e3)
+
+    # --- roofline of the dominant kernel (eval): algorithmic bytes per launch
+    bytes_per_cand = 4 * NT + R + 17
+    alg_bytes = K * bytes_per_cand
+    achieved = alg_bytes / (kern_avg / 1e3) / 1e9
+    peak_gbs, peak_src = peaks()
+    tr = ncu_traffic(cfg)
+    roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak_gbs, "unit": "GB/s",
+            "frac": round(achieved / peak_gbs, 4), "traffic": tr, "peak_source": peak_src,
+            "kernel": "magis::eval_kernel", "alg_bytes_per_launch": alg_bytes,
+            "bytes_per_candidate": bytes_per_cand, "kernel_ms_avg": round(kern_avg, 4),
+            "kernel_share_of_step": round(kern_avg / ms_per_step, 4)}
+
+    # --- end to end: the C-ABI host-buffer call (H2D perms+dec, eval, D2H results)
+    e2e = None
+    if not args.no_e2e:
+        hst = np.empty(K, np.uint8)
+        hpk = np.empty(K, np.int64)
+        hlt = np.empty(K, np.float64)
+        out_pinned = (torch.empty(K, dtype=torch.uint8).pin_memory(), torch.empty(K, dtype=torch.int64).pin_memory(),
+                      torch.empty(K, dtype=torch.float64).pin_memory())
+        g.eval_schedules_host(Ph_t, Dh_t, out=out_pinned)     # warm (allocates staging once)
+        if world > 1:
+            dist.barrier()
+        n_e2e = max(1, min(args.steps, 5))
+        t0 = time.perf_counter()
+        for _ in range(n_e2e):
+            g.eval_schedules_host(Ph_t, Dh_t, out=out_pinned)
+        e2e_s = (time.perf_counter() - t0) / n_e2e
+        te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e = {"value": round(world * K / te.item(), 1), "unit": UNIT,
+               "h2d_bytes_per_step": int(K * NT * 4 + K * R), "d2h_bytes_per_step": int(K * 17),
+               "api": "magis_eval_schedules_host (pinned host buffers, chunked double-buffered copies)",
+               "s_per_step": round(te.item(), 5)}
+        ok_same = bool((out_pinned[1].numpy() == pk.cpu().numpy()).all())
+        e2e["matches_device_path"] = ok_same
+
+    # --- CPU baseline: the oracle, as it stands, on the host cores (rank 0, N=1)
+    cpu = None
+    if pool is not None:
+        st_h, pk_h, lt_h = st.cpu().numpy(), pk.cpu().numpy(), lt.cpu().numpy()
+        probe = 256
+        _, _, _, w = oracle_pool_eval(pool, Ph[:probe], Dh[:probe], ncores)
+        rate = probe / max(w, 1e-6)
+        S = int(min(K, max(probe, rate * args.cpu_seconds)))
+        rs, rp, rl, wall = oracle_pool_eval(pool, Ph[:S], Dh[:S], ncores)
+        okm = rs == 0
+        parity = bool((rs == st_h[:S]).all() and (rp == pk_h[:S]).all() and
+                      np.all(np.abs(rl[okm] - lt_h[:S][okm]) <= 1e-9 * np.abs(rl[okm])))
+        cpu = {"value": round(S / wall, 1), "unit": UNIT, "cores": ncores, "kind": "oracle",
+               "sample": f"first {S} of the {K} candidates (single-thread C oracle per process, "
+                         f"{ncores} processes), {wall:.1f} s",
+               "op_steps_per_s": round(S / wall * NT, 1), "parity_on_sample": parity}
+        pool.close()
+
+    if rank == 0:
+        gpu_launches = args.steps * (1 + 6 + (6 if world > 1 else 0))
+        line = {"metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+                "op_steps_per_s": round(value * NT, 1),
+                "config": {**workload, "parallelism": f"candidate-dp{world}",
+                           "l2": f"inputs larger than L2 ({K * NT * 4 / 1e9:.2f} GB of perms per rank)",
+                           "front_cap": args.cap, "front_n": front_n},
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk.summary(),
+                "gpu_launches": gpu_launches,
+                "setup": {"candidate_gen_s": round(gen_s, 3), "graph_load_s": round(load_s, 3),
+                          "eval_variant": g.info["variant"], "grid": g.info["grid"], "block": g.info["block"],
+                          "smem_bytes": g.info["smem_bytes"]}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_reference(args, wl, K, workload, pool, ncores, rank, world):
+    """--impl reference: the oracle (plain single-thread C per process) timed
+    as it stands on the host cores, rank 0 only, on bounded samples."""
+    if rank != 0:
+        return
+    from magis_inputs import CandidateGenerator, CandidateSpec
+    import oracle
+    gen = CandidateGenerator(wl, CandidateSpec(seed=args.seed))
+    S = 2048
+    Ph, Dh = gen.generate(0, S)
+    for _ in range(args.warmup):
+        oracle_pool_eval(pool, Ph[:256], Dh[:256], ncores)
+    walls = []
+    for _ in range(args.steps):
+        st, pk, lt, w = oracle_pool_eval(pool, Ph, Dh, ncores)
+        t0 = time.perf_counter()
+        oracle.pareto(pk, lt, st)
+        walls.append(w + time.perf_counter() - t0)
+    pool.close()
+    s = statistics.mean(walls)
+    value = S / s
+    line = {"metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(s * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "int64", "data": "synthetic", "impl": "reference",
+            "op_steps_per_s": round(value * wl.n_total, 1),
+            "config": {**workload, "parallelism": "cpu"},
+            "cpu_baseline": {"value": round(value, 1), "unit": UNIT, "cores": ncores, "kind": "oracle",
+                             "sample": f"{S} candidates per step (first {S} of the workload), {ncores} processes"},
+            "e2e": {"value": round(value, 1), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,222 @@
+/*
+ * magis.h -- C ABI of the B200-native batched schedule evaluator for MAGIS
+ * (Chen et al., "MAGIS: Memory Optimization via Coordinated Graph
+ * Transformation and Scheduling for DNN", ASPLOS '24).
+ *
+ * Citations "P:a-b" are line ranges of the paper text; readings
+ * "Pn" are listed in DESIGN.md §Readings.
+ *
+ * The library scores K candidate schedules of one computation graph at once.
+ * A candidate is a topological order of the super-graph (original ops plus,
+ * per eligible tensor, an optional re-materialised clone, Store and Load,
+ * §5.2) and one decision per eligible tensor (0 keep,
+ * 1 re-materialise, 2 swap).  Its score is the exact peak memory M_peak
+ * and the modelled latency.
+ *
+ * All calls are thread-safe with respect to distinct graphs; a graph is
+ * immutable after load and may be used from several streams (each call uses
+ * graph-owned workspace, so concurrent calls on ONE graph must be serialised
+ * by the caller on one stream).  Every entry point returns MAGIS_SUCCESS or a
+ * negative error code; magis_last_error() gives a thread-local message.
+ * There is no CPU fallback: without an sm_100 device every call that needs
+ * one returns MAGIS_E_UNSUPPORTED.
+ */
+#ifndef MAGIS_H
+#define MAGIS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#pragma GCC visibility push(default)   /* the library builds with -fvisibility=hidden */
+#endif
+
+#define MAGIS_ABI_VERSION 1
+
+enum {
+    MAGIS_SUCCESS = 0,
+    MAGIS_E_INVAL = -1,        /* bad argument or malformed graph            */
+    MAGIS_E_CYCLE = -2,        /* the graph is not a DAG          */
+    MAGIS_E_NOMEM = -3,        /* host or device allocation failed            */
+    MAGIS_E_CUDA = -4,         /* a CUDA runtime call failed                  */
+    MAGIS_E_UNSUPPORTED = -5,  /* no sm_100 device / graph too large          */
+    MAGIS_E_CAPACITY = -6      /* output capacity too small (see pareto)      */
+};
+
+/* Candidate status bits (per-candidate problems are data, not errors;
+ * reading P12).  Any nonzero status => peak = -1, latency = +inf. */
+enum {
+    MAGIS_ST_NOT_PERM = 1,     /* perm is not a permutation of [0, n_total)  */
+    MAGIS_ST_EDGE = 2,         /* a dependency of the transformed graph is violated
+                                  (only reported when bits 0 and 2 are clear) */
+    MAGIS_ST_BAD_DEC = 4       /* a decision is not 0/1/2, or 1 on a tensor
+                                  without inputs (re-mat needs A's inputs) */
+};
+
+/*
+ * Graph description (host memory; copied by magis_graph_load, the caller
+ * keeps ownership).  Table 1 / §2.1:
+ *   n_nodes       |V|; node ids 0..n_nodes-1.  Every op has one output tensor
+ *                 (reading P4); inputs/labels/weights are ordinary zero-cost
+ *                 nodes (reading P3).
+ *   out_bytes     [n_nodes] size(v) = |v| in bytes, >= 0 (int64: sums exceed 2^31).
+ *   cost          [n_nodes] cost(v) in seconds, finite, >= 0 (the operator
+ *                 performance cache of P:1780-1783).
+ *   is_output     [n_nodes] nonzero for outs(G) (live to the end, reading P2).
+ *   n_edges, edge_src, edge_dst
+ *                 E subset of V x V; (u, v) means v reads u's output.  E is a
+ *                 set: duplicates are merged (reading P17); self-loops rejected.
+ *   n_eligible    R, tensors the re-mat / swap rules may touch (the hot-spot
+ *                 filter of P:1619-1625).
+ *   eligible_tensor [R] t_r: not a graph output, no duplicates.
+ *   late_user_ptr [R+1], late_user_idx: U_r, non-empty, U_r subset of
+ *                 cons(t_r), no duplicates: the users served by the clone /
+ *                 the Load (reading P6; Fig. 8 "one user B" generalised).
+ *   swap_bytes_per_s > 0, swap_latency_s >= 0: a Store / Load of t takes
+ *                 swap_latency_s + |t| / swap_bytes_per_s on its copy queue
+ *                 (reading P7).  Ignored when R == 0.
+ *
+ * Super-graph ids: original v -> v; for eligible r: clone_r = n+3r,
+ * store_r = n+3r+1, load_r = n+3r+2; n_total = n + 3R.
+ */
+typedef struct magis_graph_desc {
+    int32_t n_nodes;
+    const int64_t* out_bytes;
+    const double* cost;
+    const uint8_t* is_output;
+    int64_t n_edges;
+    const int32_t* edge_src;
+    const int32_t* edge_dst;
+    int32_t n_eligible;
+    const int32_t* eligible_tensor;
+    const int64_t* late_user_ptr;
+    const int32_t* late_user_idx;
+    double swap_bytes_per_s;
+    double swap_latency_s;
+} magis_graph_desc;
+
+typedef struct magis_graph magis_graph;   /* opaque, library-owned */
+
+typedef struct magis_graph_info {
+    int32_t n_nodes;           /* n */
+    int32_t n_eligible;        /* R */
+    int32_t n_total;           /* n + 3R: length of one candidate perm */
+    int64_t n_edges;           /* deduplicated |E| */
+    int64_t n_super_edges;     /* edges of the super-graph (all gates) */
+    int32_t device;            /* CUDA device ordinal */
+    int32_t variant;           /* eval kernel variant: 0 = state in shared memory, 1 = global */
+    int32_t grid;              /* persistent CTAs per eval launch */
+    int32_t block;             /* threads per CTA */
+    int64_t smem_bytes;        /* dynamic shared memory per CTA */
+    int64_t table_bytes;       /* device bytes of the graph tables */
+    double base_cost;          /* sum of cost(v) over original nodes */
+} magis_graph_info;
+
+/*
+ * Validate and upload a graph.  Builds, on `device`, the consumer and input
+ * CSRs of the super-graph with per-edge activation gates, the node tables and
+ * the swap-event tables, plus the eval workspace.
+ * Errors: MAGIS_E_INVAL (null pointer, n_nodes < 1, id out of range, self
+ * loop, negative size or cost, non-finite cost, output marked eligible,
+ * duplicate eligible tensor, empty U_r, U_r not a subset of cons(t_r),
+ * duplicate in U_r, swap_bytes_per_s <= 0 with R > 0), MAGIS_E_CYCLE,
+ * MAGIS_E_NOMEM, MAGIS_E_CUDA, MAGIS_E_UNSUPPORTED (device is not sm_100,
+ * or n_total > 2^30).  On error *out is set to NULL.
+ */
+int magis_graph_load(const magis_graph_desc* desc, int device, magis_graph** out);
+
+/* Release a graph (NULL is a no-op).  Synchronises the graph's device. */
+int magis_graph_free(magis_graph* g);
+
+int magis_graph_info_get(const magis_graph* g, magis_graph_info* info);
+
+/*
+ * Score K candidates (the hot path):
+ *   perm -> inverse permutation -> validity of every active super-graph edge
+ *   -> last-use step per tensor -> alloc/free events -> prefix scan -> max,
+ *   plus the latency model (sum of compute costs; with swaps, the three
+ *   in-order queues compute / D2H / H2D of reading P7).
+ * d_perm     [K x n_total] int32, row-major, device memory: step -> super id.
+ * d_dec      [K x R] uint8 device memory, or NULL (all zero) when R == 0.
+ * d_status   [K] uint8  out: MAGIS_ST_* bits.
+ * d_peak     [K] int64  out: M_peak in bytes (-1 if status != 0).
+ * d_latency  [K] double out: seconds (+inf if status != 0).
+ * cuda_stream: cudaStream_t (NULL = legacy default stream).
+ * Asynchronous on the stream, no allocation, no host synchronisation.
+ * Errors: MAGIS_E_INVAL (K < 0, null pointer, dec NULL with R > 0),
+ * MAGIS_E_CUDA (launch failure).
+ */
+int magis_eval_schedules(const magis_graph* g, int64_t K, const int32_t* d_perm,
+                         const uint8_t* d_dec, uint8_t* d_status, int64_t* d_peak,
+                         double* d_latency, void* cuda_stream);
+
+/*
+ * The same evaluation with HOST buffers (end-to-end path): the candidates are
+ * copied host->device in chunks on `cuda_stream` and a second graph-owned
+ * stream, overlapped with evaluation, and the results copied back.  Pinned
+ * host memory gives overlap; pageable memory works but serialises.  Blocks
+ * until the results are in h_status / h_peak / h_latency.
+ * Errors as magis_eval_schedules.
+ */
+int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_t* h_perm,
+                              const uint8_t* h_dec, uint8_t* h_status, int64_t* h_peak,
+                              double* h_latency, void* cuda_stream);
+
+/*
+ * Pareto front of (peak, latency) over valid points,
+ * plus the BetterThan-best point of Alg. 3 in both optimisation
+ * modes.  a dominates b iff a.peak <= b.peak, a.lat <= b.lat and
+ * one is strict; among exact duplicates the smallest id survives (reading P10).
+ * Used for the per-rank front and again on the all-gathered fronts; it is
+ * collective-agnostic (the caller all-gathers, e.g. via NCCL).
+ * n           number of input points (>= 0).
+ * d_peak, d_lat [n] device memory.
+ * d_status    [n] device memory (status != 0 => ignored), or NULL (all valid).
+ * d_id        [n] int64 candidate ids, or NULL => id = id_base + index.
+ *             Points with a negative id are ignored (padding of gathered fronts).
+ * cap         capacity of the front outputs (>= 0).
+ * d_front_id, d_front_peak, d_front_lat [cap] out, ascending peak
+ *             (strictly decreasing latency); the first min(front, cap)
+ *             entries are the front, entries [front, cap) are padding
+ *             (id -1, peak -1, latency +inf), so a padded front can be
+ *             all-gathered and fed back into this call as is.
+ * d_front_n   [1] out: the true front size (may exceed cap: the caller
+ *             checks; the call itself stays asynchronous).
+ * mem_limit   >= 0: d_best[0] = argmin over valid points of
+ *             (max(peak, M), lat, peak, id) (Alg. 3 mode 1, reading P10b); -1 if
+ *             mem_limit < 0 or no valid point.
+ * lat_limit   >= 0: d_best[1] = argmin of (max(lat, L), peak, lat, id) (mode 2);
+ *             -1 if lat_limit < 0 or no valid point.  d_best may be NULL.
+ * d_workspace / workspace_bytes: caller-owned device scratch of at least
+ *             magis_pareto_workspace_size(n) bytes.
+ * Asynchronous on the stream; no allocation; no host synchronisation.
+ * Errors: MAGIS_E_INVAL, MAGIS_E_CAPACITY (workspace too small), MAGIS_E_CUDA.
+ */
+int64_t magis_pareto_workspace_size(int64_t n);
+
+int magis_pareto_merge(int64_t n, const int64_t* d_peak, const double* d_lat,
+                       const uint8_t* d_status, const int64_t* d_id, int64_t id_base,
+                       int64_t cap, int64_t* d_front_id, int64_t* d_front_peak,
+                       double* d_front_lat, int64_t* d_front_n, int64_t mem_limit,
+                       double lat_limit, int64_t* d_best, void* d_workspace,
+                       int64_t workspace_bytes, void* cuda_stream);
+
+/* Thread-local message for the last nonzero return on this thread. */
+const char* magis_last_error(void);
+
+/* ABI version (MAGIS_ABI_VERSION) and whether an sm_100 device is visible. */
+int magis_abi_version(void);
+int magis_device_supported(int device);
+
+#if defined(__GNUC__)
+#pragma GCC visibility pop
+#endif
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* MAGIS_H */

@@ -1,0 +1,473 @@
+// magis_graph.cu -- graph loader and ABI glue.
+//
+// Validates the graph of Table 1 / §2.1, deduplicates E (a set,
+// reading P17), checks acyclicity (a schedule must satisfy every dependency,
+// P:402-405), and builds the super-graph the re-materialisation and swapping
+// rules can produce (§5.2, Fig. 8): per eligible tensor t_r an
+// optional clone (reads pre(t_r), serves U_r), Store (reads t_r) and Load
+// (reads the Store, serves U_r).  Every super-graph edge carries an
+// activation gate so that one static CSR serves every decision vector.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <numeric>
+#include <vector>
+
+#include "magis_internal.h"
+
+namespace magis {
+
+static thread_local std::string g_err;
+
+int set_error(int code, const std::string& msg) {
+    g_err = msg;
+    return code;
+}
+void clear_error() { g_err.clear(); }
+
+}  // namespace magis
+
+using namespace magis;
+
+extern "C" const char* magis_last_error(void) { return g_err.c_str(); }
+extern "C" int magis_abi_version(void) { return MAGIS_ABI_VERSION; }
+
+extern "C" int magis_device_supported(int device) {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    if (device < 0 || device >= n) return 0;
+    cudaDeviceProp p;
+    if (cudaGetDeviceProperties(&p, device) != cudaSuccess) return 0;
+    return p.major == 10 ? 1 : 0;
+}
+
+namespace {
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int d) {
+        cudaGetDevice(&prev);
+        cudaSetDevice(d);
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+#define CK(call)                                                                   \
+    do {                                                                           \
+        cudaError_t _e = (call);                                                   \
+        if (_e != cudaSuccess) {                                                   \
+            cudaGetLastError();                                                    \
+            return set_error(MAGIS_E_CUDA, std::string(#call ": ") + cudaGetErrorString(_e)); \
+        }                                                                          \
+    } while (0)
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+}  // namespace
+
+extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_graph** out) {
+    clear_error();
+    if (!out) return set_error(MAGIS_E_INVAL, "out is NULL");
+    *out = nullptr;
+    if (!d) return set_error(MAGIS_E_INVAL, "desc is NULL");
+    const int32_t n = d->n_nodes;
+    const int32_t R = d->n_eligible;
+    if (n < 1) return set_error(MAGIS_E_INVAL, "n_nodes < 1");
+    if (R < 0) return set_error(MAGIS_E_INVAL, "n_eligible < 0");
+    if (d->n_edges < 0) return set_error(MAGIS_E_INVAL, "n_edges < 0");
+    if (!d->out_bytes || !d->cost || !d->is_output)
+        return set_error(MAGIS_E_INVAL, "null node array");
+    if (d->n_edges > 0 && (!d->edge_src || !d->edge_dst))
+        return set_error(MAGIS_E_INVAL, "null edge array");
+    if (R > 0 && (!d->eligible_tensor || !d->late_user_ptr || !d->late_user_idx))
+        return set_error(MAGIS_E_INVAL, "null eligible array");
+    if ((int64_t)n + 3 * (int64_t)R > (1 << 30))
+        return set_error(MAGIS_E_UNSUPPORTED, "n_total > 2^30");
+    if (R > (1 << 23)) return set_error(MAGIS_E_UNSUPPORTED, "n_eligible > 2^23");
+    for (int32_t v = 0; v < n; v++) {
+        if (d->out_bytes[v] < 0) return set_error(MAGIS_E_INVAL, "negative out_bytes at node " + std::to_string(v));
+        if (!(d->cost[v] >= 0.0) || !std::isfinite(d->cost[v]))
+            return set_error(MAGIS_E_INVAL, "negative or non-finite cost at node " + std::to_string(v));
+    }
+    if (R > 0 && !(d->swap_bytes_per_s > 0.0 && std::isfinite(d->swap_bytes_per_s)))
+        return set_error(MAGIS_E_INVAL, "swap_bytes_per_s must be > 0");
+    if (R > 0 && !(d->swap_latency_s >= 0.0 && std::isfinite(d->swap_latency_s)))
+        return set_error(MAGIS_E_INVAL, "swap_latency_s must be >= 0");
+
+    // --- E as a set (reading P17) ------------------------------------------
+    std::vector<uint64_t> keys;
+    keys.reserve((size_t)d->n_edges);
+    for (int64_t e = 0; e < d->n_edges; e++) {
+        int32_t u = d->edge_src[e], v = d->edge_dst[e];
+        if (u < 0 || u >= n || v < 0 || v >= n)
+            return set_error(MAGIS_E_INVAL, "edge id out of range at edge " + std::to_string(e));
+        if (u == v) return set_error(MAGIS_E_INVAL, "self-loop at node " + std::to_string(u));
+        keys.push_back(((uint64_t)(uint32_t)u << 32) | (uint32_t)v);
+    }
+    std::sort(keys.begin(), keys.end());
+    keys.erase(std::unique(keys.begin(), keys.end()), keys.end());
+    const int64_t E = (int64_t)keys.size();
+    std::vector<int32_t> succ_ptr(n + 1, 0), succ(E), pred_ptr(n + 1, 0), pred(E);
+    for (auto k : keys) { succ_ptr[(k >> 32) + 1]++; pred_ptr[(uint32_t)k + 1]++; }
+    for (int32_t v = 0; v < n; v++) { succ_ptr[v + 1] += succ_ptr[v]; pred_ptr[v + 1] += pred_ptr[v]; }
+    {
+        std::vector<int32_t> fs(succ_ptr.begin(), succ_ptr.end() - 1), fp(pred_ptr.begin(), pred_ptr.end() - 1);
+        for (auto k : keys) {
+            int32_t u = (int32_t)(k >> 32), v = (int32_t)(uint32_t)k;
+            succ[fs[u]++] = v;
+            pred[fp[v]++] = u;
+        }
+    }
+    // --- acyclicity --------------------------------------------
+    {
+        std::vector<int32_t> indeg(n), stack;
+        for (int32_t v = 0; v < n; v++) {
+            indeg[v] = pred_ptr[v + 1] - pred_ptr[v];
+            if (!indeg[v]) stack.push_back(v);
+        }
+        int32_t seen = 0;
+        while (!stack.empty()) {
+            int32_t u = stack.back();
+            stack.pop_back();
+            seen++;
+            for (int32_t e = succ_ptr[u]; e < succ_ptr[u + 1]; e++)
+                if (--indeg[succ[e]] == 0) stack.push_back(succ[e]);
+        }
+        if (seen != n) return set_error(MAGIS_E_CYCLE, "the graph has a cycle");
+    }
+    // --- eligible tensors (reading P6) -------------------------------------
+    std::vector<int32_t> r_of(n, -1);
+    int64_t nU = R > 0 ? d->late_user_ptr[R] : 0;
+    if (R > 0 && d->late_user_ptr[0] != 0) return set_error(MAGIS_E_INVAL, "late_user_ptr[0] != 0");
+    for (int32_t r = 0; r < R; r++) {
+        int32_t t = d->eligible_tensor[r];
+        if (t < 0 || t >= n) return set_error(MAGIS_E_INVAL, "eligible id out of range");
+        if (d->is_output[t]) return set_error(MAGIS_E_INVAL, "graph output marked eligible: " + std::to_string(t));
+        if (r_of[t] >= 0) return set_error(MAGIS_E_INVAL, "duplicate eligible tensor " + std::to_string(t));
+        r_of[t] = r;
+        int64_t a = d->late_user_ptr[r], b = d->late_user_ptr[r + 1];
+        if (b <= a) return set_error(MAGIS_E_INVAL, "empty U_r for r=" + std::to_string(r));
+        std::vector<int32_t> us(d->late_user_idx + a, d->late_user_idx + b);
+        std::sort(us.begin(), us.end());
+        if (std::unique(us.begin(), us.end()) != us.end())
+            return set_error(MAGIS_E_INVAL, "duplicate late user for r=" + std::to_string(r));
+        for (int32_t bb : us) {
+            if (bb < 0 || bb >= n || !std::binary_search(succ.begin() + succ_ptr[t], succ.begin() + succ_ptr[t + 1], bb))
+                return set_error(MAGIS_E_INVAL, "U_r not a subset of cons(t_r) for r=" + std::to_string(r));
+        }
+    }
+    const int32_t NT = n + 3 * R;
+
+    // --- super-graph edges with gates (Fig. 8) ------------------------------
+    struct SE { int32_t u, v, gate; };
+    std::vector<SE> se;
+    se.reserve((size_t)E + 2 * (size_t)nU + 2 * (size_t)R + 16);
+    std::vector<std::vector<int32_t>> Uset(R);
+    for (int32_t r = 0; r < R; r++) {
+        Uset[r].assign(d->late_user_idx + d->late_user_ptr[r], d->late_user_idx + d->late_user_ptr[r + 1]);
+        std::sort(Uset[r].begin(), Uset[r].end());
+    }
+    for (auto k : keys) {
+        int32_t u = (int32_t)(k >> 32), v = (int32_t)(uint32_t)k;
+        int32_t r = r_of[u];
+        if (r >= 0 && std::binary_search(Uset[r].begin(), Uset[r].end(), v)) {
+            se.push_back({u, v, (r << 2) | 0});              // t_r -> b kept (dec 0)
+            se.push_back({n + 3 * r, v, (r << 2) | 1});      // clone_r -> b (dec 1)
+            se.push_back({n + 3 * r + 2, v, (r << 2) | 2});  // load_r -> b (dec 2)
+        } else {
+            se.push_back({u, v, kAlways});
+        }
+    }
+    for (int32_t r = 0; r < R; r++) {
+        int32_t t = d->eligible_tensor[r];
+        for (int32_t e = pred_ptr[t]; e < pred_ptr[t + 1]; e++)
+            se.push_back({pred[e], n + 3 * r, (r << 2) | 1});   // A' reads A's inputs
+        se.push_back({t, n + 3 * r + 1, (r << 2) | 2});          // A -> Store
+        se.push_back({n + 3 * r + 1, n + 3 * r + 2, (r << 2) | 2});  // Store -> Load
+    }
+    const int64_t SEn = (int64_t)se.size();
+    if (SEn > INT32_MAX) return set_error(MAGIS_E_UNSUPPORTED, "too many super-graph edges");
+
+    std::vector<int32_t> cons_ptr(NT + 1, 0), in_ptr(NT + 1, 0);
+    for (auto& x : se) { cons_ptr[x.u + 1]++; in_ptr[x.v + 1]++; }
+    for (int32_t v = 0; v < NT; v++) { cons_ptr[v + 1] += cons_ptr[v]; in_ptr[v + 1] += in_ptr[v]; }
+    std::vector<int2> cons_ent(SEn), in_ent(SEn);
+    {
+        std::sort(se.begin(), se.end(), [](const SE& a, const SE& b) { return a.u != b.u ? a.u < b.u : a.v < b.v; });
+        for (int64_t i = 0; i < SEn; i++) cons_ent[i] = make_int2(se[i].v, se[i].gate);
+        std::sort(se.begin(), se.end(), [](const SE& a, const SE& b) { return a.v != b.v ? a.v < b.v : a.u < b.u; });
+        for (int64_t i = 0; i < SEn; i++) in_ent[i] = make_int2(se[i].u, se[i].gate);
+    }
+    // --- node tables (reading P5, P9) ----------------------------------------
+    std::vector<int64_t> size(NT);
+    std::vector<double> cost(NT, 0.0);
+    std::vector<int32_t> ngate(NT, kAlways);
+    std::vector<uint8_t> nflag(NT, 0);
+    double base_cost = 0.0;
+    for (int32_t v = 0; v < n; v++) {
+        size[v] = d->out_bytes[v];
+        cost[v] = d->cost[v];
+        nflag[v] = (uint8_t)((d->is_output[v] ? kFlagOutput : 0) | kFlagCompute);
+        base_cost += d->cost[v];
+    }
+    std::vector<int32_t> elig(R), U_ptr(R + 1, 0), U_idx((size_t)nU);
+    std::vector<double> xfer(R), tcost(R);
+    std::vector<uint8_t> rflag(R);
+    for (int32_t r = 0; r < R; r++) {
+        int32_t t = d->eligible_tensor[r];
+        elig[r] = t;
+        size[n + 3 * r] = d->out_bytes[t];        // clone A' = |A|
+        size[n + 3 * r + 1] = 0;                   // Store: data in external storage
+        size[n + 3 * r + 2] = d->out_bytes[t];    // Load = |A|
+        cost[n + 3 * r] = d->cost[t];              // cost(A') = cost(A)
+        ngate[n + 3 * r] = (r << 2) | 1;
+        ngate[n + 3 * r + 1] = (r << 2) | 2;
+        ngate[n + 3 * r + 2] = (r << 2) | 2;
+        nflag[n + 3 * r] = kFlagCompute;
+        xfer[r] = d->swap_latency_s + (double)d->out_bytes[t] / d->swap_bytes_per_s;
+        tcost[r] = d->cost[t];
+        rflag[r] = (uint8_t)(pred_ptr[t + 1] > pred_ptr[t] ? kRHasInput : 0);
+        U_ptr[r + 1] = U_ptr[r] + (int32_t)Uset[r].size();
+        std::copy(Uset[r].begin(), Uset[r].end(), U_idx.begin() + U_ptr[r]);
+    }
+
+    // --- upload ----------------------------------------------------------------
+    if (!magis_device_supported(device))
+        return set_error(MAGIS_E_UNSUPPORTED, "device " + std::to_string(device) +
+                         " is not an sm_100 (B200) GPU; there is no CPU fallback");
+    DeviceGuard guard(device);
+    magis_graph* g = new (std::nothrow) magis_graph();
+    if (!g) return set_error(MAGIS_E_NOMEM, "host allocation failed");
+    g->device = device;
+    g->n_edges = E;
+    g->n_super_edges = SEn;
+    struct Part { const void* src; size_t bytes; size_t off; };
+    std::vector<Part> parts;
+    size_t off = 0;
+    auto add = [&](const void* p, size_t b) { parts.push_back({p, b, off}); size_t o = off; off = align_up(off + std::max<size_t>(b, 1), 256); return o; };
+    size_t o_cons_ptr = add(cons_ptr.data(), cons_ptr.size() * 4);
+    size_t o_cons_ent = add(cons_ent.data(), cons_ent.size() * 8);
+    size_t o_in_ptr = add(in_ptr.data(), in_ptr.size() * 4);
+    size_t o_in_ent = add(in_ent.data(), in_ent.size() * 8);
+    size_t o_size = add(size.data(), size.size() * 8);
+    size_t o_cost = add(cost.data(), cost.size() * 8);
+    size_t o_ngate = add(ngate.data(), ngate.size() * 4);
+    size_t o_nflag = add(nflag.data(), nflag.size());
+    size_t o_elig = add(elig.data(), elig.size() * 4);
+    size_t o_Uptr = add(U_ptr.data(), U_ptr.size() * 4);
+    size_t o_Uidx = add(U_idx.data(), U_idx.size() * 4);
+    size_t o_xfer = add(xfer.data(), xfer.size() * 8);
+    size_t o_tcost = add(tcost.data(), tcost.size() * 8);
+    size_t o_rflag = add(rflag.data(), rflag.size());
+    g->blob_bytes = off;
+    cudaError_t e = cudaMalloc(&g->blob, off);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        delete g;
+        return set_error(MAGIS_E_NOMEM, "cudaMalloc graph tables failed");
+    }
+    std::vector<char> host(off, 0);
+    for (auto& p : parts)
+        if (p.bytes) std::memcpy(host.data() + p.off, p.src, p.bytes);
+    e = cudaMemcpy(g->blob, host.data(), off, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(g->blob);
+        delete g;
+        return set_error(MAGIS_E_CUDA, "upload of graph tables failed");
+    }
+    char* b = (char*)g->blob;
+    DevGraph& dg = g->dev;
+    dg.n = n;
+    dg.R = R;
+    dg.NT = NT;
+    dg.max_events = 3 * R + (int32_t)nU;
+    dg.cons_ptr = (const int32_t*)(b + o_cons_ptr);
+    dg.cons_ent = (const int2*)(b + o_cons_ent);
+    dg.in_ptr = (const int32_t*)(b + o_in_ptr);
+    dg.in_ent = (const int2*)(b + o_in_ent);
+    dg.size = (const int64_t*)(b + o_size);
+    dg.cost = (const double*)(b + o_cost);
+    dg.ngate = (const int32_t*)(b + o_ngate);
+    dg.nflag = (const uint8_t*)(b + o_nflag);
+    dg.elig = (const int32_t*)(b + o_elig);
+    dg.U_ptr = (const int32_t*)(b + o_Uptr);
+    dg.U_idx = (const int32_t*)(b + o_Uidx);
+    dg.xfer = (const double*)(b + o_xfer);
+    dg.tcost = (const double*)(b + o_tcost);
+    dg.rflag = (const uint8_t*)(b + o_rflag);
+    dg.base_cost = base_cost;
+
+    e = eval_configure(dg, device, &g->cfg);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(g->blob);
+        delete g;
+        return set_error(MAGIS_E_CUDA, std::string("eval_configure: ") + cudaGetErrorString(e));
+    }
+    if (g->cfg.variant == 1) {
+        g->gws_bytes = g->cfg.state_bytes * (size_t)g->cfg.grid;
+        e = cudaMalloc(&g->gws, g->gws_bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            cudaFree(g->blob);
+            delete g;
+            return set_error(MAGIS_E_NOMEM, "cudaMalloc eval workspace failed");
+        }
+    }
+    *out = g;
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int magis_graph_free(magis_graph* g) {
+    clear_error();
+    if (!g) return MAGIS_SUCCESS;
+    DeviceGuard guard(g->device);
+    cudaDeviceSynchronize();
+    if (g->blob) cudaFree(g->blob);
+    if (g->gws) cudaFree(g->gws);
+    for (int i = 0; i < 2; i++) {
+        if (g->stage[i]) cudaFree(g->stage[i]);
+        if (g->ev_h2d[i]) cudaEventDestroy(g->ev_h2d[i]);
+        if (g->ev_done[i]) cudaEventDestroy(g->ev_done[i]);
+    }
+    if (g->aux) cudaStreamDestroy(g->aux);
+    cudaGetLastError();
+    delete g;
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int magis_graph_info_get(const magis_graph* g, magis_graph_info* info) {
+    clear_error();
+    if (!g || !info) return set_error(MAGIS_E_INVAL, "null argument");
+    info->n_nodes = g->dev.n;
+    info->n_eligible = g->dev.R;
+    info->n_total = g->dev.NT;
+    info->n_edges = g->n_edges;
+    info->n_super_edges = g->n_super_edges;
+    info->device = g->device;
+    info->variant = g->cfg.variant;
+    info->grid = g->cfg.grid;
+    info->block = g->cfg.block;
+    info->smem_bytes = (int64_t)g->cfg.smem;
+    info->table_bytes = (int64_t)g->blob_bytes;
+    info->base_cost = g->dev.base_cost;
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int magis_eval_schedules(const magis_graph* g, int64_t K, const int32_t* d_perm,
+                                    const uint8_t* d_dec, uint8_t* d_status, int64_t* d_peak,
+                                    double* d_latency, void* cuda_stream) {
+    clear_error();
+    if (!g) return set_error(MAGIS_E_INVAL, "graph is NULL");
+    if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
+    if (K == 0) return MAGIS_SUCCESS;
+    if (!d_perm || !d_status || !d_peak || !d_latency)
+        return set_error(MAGIS_E_INVAL, "null device pointer");
+    if (g->dev.R > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R > 0");
+    DeviceGuard guard(g->device);
+    cudaError_t e = eval_launch(g->dev, g->cfg, g->gws, K, d_perm, d_dec, d_status, d_peak,
+                                d_latency, (cudaStream_t)cuda_stream);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return set_error(MAGIS_E_CUDA, std::string("eval launch: ") + cudaGetErrorString(e));
+    }
+    return MAGIS_SUCCESS;
+}
+
+// End-to-end host path: chunked, double-buffered H2D -> eval -> D2H.
+extern "C" int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_t* h_perm,
+                                         const uint8_t* h_dec, uint8_t* h_status,
+                                         int64_t* h_peak, double* h_latency,
+                                         void* cuda_stream) {
+    clear_error();
+    if (!g) return set_error(MAGIS_E_INVAL, "graph is NULL");
+    if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
+    if (K == 0) return MAGIS_SUCCESS;
+    if (!h_perm || !h_status || !h_peak || !h_latency)
+        return set_error(MAGIS_E_INVAL, "null host pointer");
+    const int32_t R = g->dev.R, NT = g->dev.NT;
+    if (R > 0 && !h_dec) return set_error(MAGIS_E_INVAL, "h_dec is NULL but R > 0");
+    DeviceGuard guard(g->device);
+    cudaStream_t s0 = (cudaStream_t)cuda_stream;
+    // chunk of ~64 MiB of perms
+    int64_t chunk = std::max<int64_t>(1, (64ll << 20) / ((int64_t)NT * 4));
+    chunk = std::min<int64_t>(chunk, K);
+    const size_t perm_b = align_up((size_t)chunk * NT * 4, 256);
+    const size_t dec_b = align_up((size_t)chunk * std::max(R, 1), 256);
+    const size_t out_b = align_up((size_t)chunk * 17, 256);
+    if (g->stage_K < chunk) {
+        for (int i = 0; i < 2; i++) {
+            if (g->stage[i]) cudaFree(g->stage[i]);
+            g->stage[i] = nullptr;
+            CK(cudaMalloc(&g->stage[i], perm_b + dec_b + out_b + 256));
+            if (!g->ev_h2d[i]) CK(cudaEventCreateWithFlags(&g->ev_h2d[i], cudaEventDisableTiming));
+            if (!g->ev_done[i]) CK(cudaEventCreateWithFlags(&g->ev_done[i], cudaEventDisableTiming));
+        }
+        if (!g->aux) CK(cudaStreamCreateWithFlags(&g->aux, cudaStreamNonBlocking));
+        g->stage_K = chunk;
+    }
+    // copies on aux, compute on s0; two buffers alternate.
+    int64_t nchunks = (K + chunk - 1) / chunk;
+    for (int64_t c = 0; c < nchunks; c++) {
+        int b = (int)(c & 1);
+        int64_t k0 = c * chunk, kc = std::min(chunk, K - k0);
+        char* base = (char*)g->stage[b];
+        int32_t* dp = (int32_t*)base;
+        uint8_t* dd = (uint8_t*)(base + perm_b);
+        int64_t* dpk = (int64_t*)(base + perm_b + dec_b);
+        double* dlt = (double*)(base + perm_b + dec_b + align_up((size_t)chunk * 8, 64));
+        uint8_t* dst = (uint8_t*)(base + perm_b + dec_b + 2 * align_up((size_t)chunk * 8, 64));
+        // buffer b is free once the D2H of chunk c-2 finished
+        if (c >= 2) CK(cudaStreamWaitEvent(g->aux, g->ev_done[b], 0));
+        CK(cudaMemcpyAsync(dp, h_perm + k0 * NT, (size_t)kc * NT * 4, cudaMemcpyHostToDevice, g->aux));
+        if (R > 0) CK(cudaMemcpyAsync(dd, h_dec + k0 * R, (size_t)kc * R, cudaMemcpyHostToDevice, g->aux));
+        CK(cudaEventRecord(g->ev_h2d[b], g->aux));
+        CK(cudaStreamWaitEvent(s0, g->ev_h2d[b], 0));
+        cudaError_t e = eval_launch(g->dev, g->cfg, g->gws, kc, dp, R > 0 ? dd : nullptr, dst, dpk, dlt, s0);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return set_error(MAGIS_E_CUDA, std::string("eval launch: ") + cudaGetErrorString(e));
+        }
+        CK(cudaMemcpyAsync(h_status + k0, dst, (size_t)kc, cudaMemcpyDeviceToHost, s0));
+        CK(cudaMemcpyAsync(h_peak + k0, dpk, (size_t)kc * 8, cudaMemcpyDeviceToHost, s0));
+        CK(cudaMemcpyAsync(h_latency + k0, dlt, (size_t)kc * 8, cudaMemcpyDeviceToHost, s0));
+        CK(cudaEventRecord(g->ev_done[b], s0));
+    }
+    CK(cudaStreamSynchronize(s0));
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int64_t magis_pareto_workspace_size(int64_t n) {
+    return n < 0 ? 0 : pareto_workspace_size(n);
+}
+
+extern "C" int magis_pareto_merge(int64_t n, const int64_t* d_peak, const double* d_lat,
+                                  const uint8_t* d_status, const int64_t* d_id, int64_t id_base,
+                                  int64_t cap, int64_t* d_front_id, int64_t* d_front_peak,
+                                  double* d_front_lat, int64_t* d_front_n, int64_t mem_limit,
+                                  double lat_limit, int64_t* d_best, void* d_workspace,
+                                  int64_t workspace_bytes, void* cuda_stream) {
+    clear_error();
+    if (n < 0 || cap < 0) return set_error(MAGIS_E_INVAL, "n < 0 or cap < 0");
+    if (!d_front_n) return set_error(MAGIS_E_INVAL, "d_front_n is NULL");
+    if (n > 0 && (!d_peak || !d_lat))
+        return set_error(MAGIS_E_INVAL, "null input pointer");
+    if (cap > 0 && (!d_front_id || !d_front_peak || !d_front_lat))
+        return set_error(MAGIS_E_INVAL, "null front pointer");
+    if (workspace_bytes < pareto_workspace_size(n) || (n > 0 && !d_workspace))
+        return set_error(MAGIS_E_CAPACITY, "workspace smaller than magis_pareto_workspace_size(n)");
+    cudaError_t e = pareto_launch(n, d_peak, d_lat, d_status, d_id, id_base, cap, d_front_id,
+                                  d_front_peak, d_front_lat, d_front_n, mem_limit, lat_limit,
+                                  d_best, d_workspace, (cudaStream_t)cuda_stream);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return set_error(MAGIS_E_CUDA, std::string("pareto launch: ") + cudaGetErrorString(e));
+    }
+    return MAGIS_SUCCESS;
+}

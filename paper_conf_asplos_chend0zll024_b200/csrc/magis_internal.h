@@ -1,0 +1,104 @@
+// magis_internal.h -- shared declarations of the B200 evaluation library.
+// Not part of the ABI (see include/magis.h).
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+#include <string>
+
+#include <cuda_runtime.h>
+
+#include "magis.h"
+
+namespace magis {
+
+// Activation gate of a super-graph node or edge (reading P6, Fig. 8):
+// -1 = always active, otherwise (r << 2) | d = active iff dec[r] == d.
+constexpr int32_t kAlways = -1;
+
+// Per-node flags.
+constexpr uint8_t kFlagOutput = 1;    // outs(G): live to the end (reading P2)
+constexpr uint8_t kFlagCompute = 2;   // runs on the compute queue (original op or clone)
+
+// Per-eligible flags.
+constexpr uint8_t kRHasInput = 1;     // t_r has inputs: re-mat allowed
+
+// Swap-latency event types, in the order events at one step are applied.
+constexpr uint32_t kEvStall = 0;      // compute op waits for a Load it reads
+constexpr uint32_t kEvProduce = 1;    // producer t_r of a swapped tensor finishes
+constexpr uint32_t kEvStore = 2;      // Store on the D2H queue
+constexpr uint32_t kEvLoad = 3;       // Load on the H2D queue
+
+// Device view of one loaded graph (all pointers are device memory).
+struct DevGraph {
+    int32_t n;           // original nodes
+    int32_t R;           // eligible tensors
+    int32_t NT;          // n + 3R
+    int32_t max_events;  // 3R + |U| (swap events of one candidate, upper bound)
+    const int32_t* cons_ptr;   // [NT+1]
+    const int2* cons_ent;      // (consumer id, gate)
+    const int32_t* in_ptr;     // [NT+1]
+    const int2* in_ent;        // (input id, gate)
+    const int64_t* size;       // [NT] device bytes of the node's output when active (P5, P9)
+    const double* cost;        // [NT] compute cost (0 for Store / Load)
+    const int32_t* ngate;      // [NT]
+    const uint8_t* nflag;      // [NT]
+    const int32_t* elig;       // [R] t_r
+    const int32_t* U_ptr;      // [R+1]
+    const int32_t* U_idx;      // U_r
+    const double* xfer;        // [R] swap_latency + |t_r| / bytes_per_s
+    const double* tcost;       // [R] cost(t_r)
+    const uint8_t* rflag;      // [R]
+    double base_cost;          // sum of cost over original nodes
+};
+
+struct EvalConfig {
+    int variant;          // 0: per-candidate state in shared memory, 1: in global workspace
+    int grid;
+    int block;
+    size_t smem;          // dynamic shared memory per CTA
+    size_t state_bytes;   // per-CTA candidate state
+};
+
+// Per-CTA candidate state layout (same in shared or global memory).
+struct StateLayout {
+    size_t pos, last, A, Fr, C, evkey_in, evkey_out, evcb, endT, endS, endL, dec, total;
+};
+StateLayout state_layout(int32_t NT, int32_t R, int32_t max_events);
+
+cudaError_t eval_configure(const DevGraph& g, int device, EvalConfig* cfg);
+cudaError_t eval_launch(const DevGraph& g, const EvalConfig& cfg, void* gws, int64_t K,
+                        const int32_t* perm, const uint8_t* dec, uint8_t* status,
+                        int64_t* peak, double* lat, cudaStream_t stream);
+
+int64_t pareto_workspace_size(int64_t n);
+cudaError_t pareto_launch(int64_t n, const int64_t* peak, const double* lat,
+                          const uint8_t* status, const int64_t* id, int64_t id_base,
+                          int64_t cap, int64_t* front_id, int64_t* front_peak,
+                          double* front_lat, int64_t* front_n, int64_t mem_limit,
+                          double lat_limit, int64_t* best, void* ws, cudaStream_t stream);
+
+// thread-local error reporting
+int set_error(int code, const std::string& msg);
+void clear_error();
+
+}  // namespace magis
+
+// The opaque graph handle.
+struct magis_graph {
+    int device = 0;
+    magis::DevGraph dev{};
+    magis::EvalConfig cfg{};
+    void* blob = nullptr;          // device tables
+    size_t blob_bytes = 0;
+    void* gws = nullptr;           // global per-CTA workspace (variant 1)
+    size_t gws_bytes = 0;
+    int64_t n_edges = 0;
+    int64_t n_super_edges = 0;
+    // host-buffer (end-to-end) path: lazily allocated staging
+    cudaStream_t aux = nullptr;
+    int64_t stage_K = 0;
+    void* stage[2] = {nullptr, nullptr};
+    cudaEvent_t ev_h2d[2] = {nullptr, nullptr};
+    cudaEvent_t ev_done[2] = {nullptr, nullptr};
+};

@@ -1,0 +1,48 @@
+"""Cross-rank Pareto merge.
+
+Candidates shard over ranks by contiguous global-id ranges; each rank scores
+its shard and computes its local front with magis_pareto_merge; the padded
+fronts (cap points of (id, peak, latency)) are all-gathered over the process
+group (NCCL over NVLink on B200, gloo in the CPU tests) and every rank re-runs
+the same deterministic merge, so all ranks hold the identical global front
+and BetterThan-best ids (Alg. 3).  This is the path's only
+exchange step.
+"""
+from __future__ import annotations
+
+from typing import Callable, Dict, Optional
+
+import torch
+import torch.distributed as dist
+
+from . import magis
+
+
+def shard_range(K: int, rank: int, world: int):
+    """Contiguous global-id range [lo, hi) of this rank."""
+    return K * rank // world, K * (rank + 1) // world
+
+
+def gather_fronts(front: Dict[str, torch.Tensor], group=None) -> Dict[str, torch.Tensor]:
+    """All-gather the padded local fronts (id, peak, lat; each [cap])."""
+    world = dist.get_world_size(group)
+    out = {}
+    for key in ("front_id", "front_peak", "front_lat"):
+        t = front[key].contiguous()
+        buf = torch.empty(world * t.numel(), dtype=t.dtype, device=t.device)
+        dist.all_gather_into_tensor(buf, t, group=group)
+        out[key] = buf
+    return out
+
+
+def global_front(front: Dict[str, torch.Tensor], cap: int, mem_limit: int = -1,
+                 lat_limit: float = -1.0, group=None,
+                 merge: Optional[Callable] = None) -> Dict[str, torch.Tensor]:
+    """Merge this rank's padded front with every other rank's.
+
+    ``merge`` defaults to the device merge (magis_pareto_merge); the CPU gloo
+    tests pass a host implementation with the same contract."""
+    g = gather_fronts(front, group)
+    merge = merge or (lambda peak, lat, ids, cap, M, L: magis.pareto_merge(
+        peak, lat, None, ids=ids, cap=cap, mem_limit=M, lat_limit=L))
+    return merge(g["front_peak"], g["front_lat"], g["front_id"], cap, mem_limit, lat_limit)

@@ -1,0 +1,229 @@
+"""Thin ctypes binding of libmagis.so (include/magis.h) -- argument marshalling only.
+
+Every step of the evaluation runs in the library's sm_100a kernels; PyTorch
+supplies device memory and streams.  There is no fallback: if libmagis.so is
+missing or no B200 is visible, the calls raise MagisError.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional, Sequence
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libmagis.so")
+
+MAGIS_SUCCESS = 0
+ERRORS = {-1: "MAGIS_E_INVAL", -2: "MAGIS_E_CYCLE", -3: "MAGIS_E_NOMEM", -4: "MAGIS_E_CUDA",
+          -5: "MAGIS_E_UNSUPPORTED", -6: "MAGIS_E_CAPACITY"}
+ST_NOT_PERM, ST_EDGE, ST_BAD_DEC = 1, 2, 4
+
+# names declared in include/magis.h (checked by tests/test_abi.py)
+EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magis_eval_schedules",
+           "magis_eval_schedules_host", "magis_pareto_workspace_size", "magis_pareto_merge",
+           "magis_last_error", "magis_abi_version", "magis_device_supported"]
+
+
+class MagisError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{ERRORS.get(code, code)}: {msg}")
+        self.code = code
+
+
+class GraphDesc(ctypes.Structure):
+    _fields_ = [("n_nodes", ctypes.c_int32), ("out_bytes", ctypes.c_void_p), ("cost", ctypes.c_void_p),
+                ("is_output", ctypes.c_void_p), ("n_edges", ctypes.c_int64), ("edge_src", ctypes.c_void_p),
+                ("edge_dst", ctypes.c_void_p), ("n_eligible", ctypes.c_int32),
+                ("eligible_tensor", ctypes.c_void_p), ("late_user_ptr", ctypes.c_void_p),
+                ("late_user_idx", ctypes.c_void_p), ("swap_bytes_per_s", ctypes.c_double),
+                ("swap_latency_s", ctypes.c_double)]
+
+
+class GraphInfo(ctypes.Structure):
+    _fields_ = [("n_nodes", ctypes.c_int32), ("n_eligible", ctypes.c_int32), ("n_total", ctypes.c_int32),
+                ("n_edges", ctypes.c_int64), ("n_super_edges", ctypes.c_int64), ("device", ctypes.c_int32),
+                ("variant", ctypes.c_int32), ("grid", ctypes.c_int32), ("block", ctypes.c_int32),
+                ("smem_bytes", ctypes.c_int64), ("table_bytes", ctypes.c_int64), ("base_cost", ctypes.c_double)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libmagis.so (raises if it is not built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise MagisError(-5, f"{LIB_PATH} not built (run __graft_entry__.build()); there is no fallback")
+    L = ctypes.CDLL(LIB_PATH)
+    P, i32, i64, d = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_double
+    L.magis_graph_load.argtypes = [ctypes.POINTER(GraphDesc), ctypes.c_int, ctypes.POINTER(P)]
+    L.magis_graph_load.restype = ctypes.c_int
+    L.magis_graph_free.argtypes = [P]
+    L.magis_graph_free.restype = ctypes.c_int
+    L.magis_graph_info_get.argtypes = [P, ctypes.POINTER(GraphInfo)]
+    L.magis_graph_info_get.restype = ctypes.c_int
+    L.magis_eval_schedules.argtypes = [P, i64, P, P, P, P, P, P]
+    L.magis_eval_schedules.restype = ctypes.c_int
+    L.magis_eval_schedules_host.argtypes = [P, i64, P, P, P, P, P, P]
+    L.magis_eval_schedules_host.restype = ctypes.c_int
+    L.magis_pareto_workspace_size.argtypes = [i64]
+    L.magis_pareto_workspace_size.restype = i64
+    L.magis_pareto_merge.argtypes = [i64, P, P, P, P, i64, i64, P, P, P, P, i64, d, P, P, i64, P]
+    L.magis_pareto_merge.restype = ctypes.c_int
+    L.magis_last_error.argtypes = []
+    L.magis_last_error.restype = ctypes.c_char_p
+    L.magis_abi_version.restype = ctypes.c_int
+    L.magis_device_supported.argtypes = [ctypes.c_int]
+    L.magis_device_supported.restype = ctypes.c_int
+    _lib = L
+    return L
+
+
+def _check(code: int):
+    if code != MAGIS_SUCCESS:
+        msg = lib().magis_last_error()
+        raise MagisError(code, msg.decode() if msg else "")
+
+
+def _np_ptr(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.c_void_p) if a is not None and a.size else None
+
+
+def _tptr(t) -> Optional[int]:
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream_ptr(stream) -> Optional[ctypes.c_void_p]:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+class Graph:
+    """A loaded graph (magis_graph_load).  Arguments follow Table 1:
+    out_bytes = size(v), cost = cost(v), is_output = outs(G), edges E, plus the
+    eligible tensors t_r with late users U_r and the swap link model."""
+
+    def __init__(self, out_bytes, cost, is_output, edge_src, edge_dst, eligible: Sequence[int] = (),
+                 late_users: Sequence[Sequence[int]] = (), swap_bytes_per_s: float = 25e9,
+                 swap_latency_s: float = 1e-5, device: int = 0):
+        L = lib()
+        self._L = L
+        self._h = None
+        ob = np.ascontiguousarray(out_bytes, np.int64)
+        co = np.ascontiguousarray(cost, np.float64)
+        io = np.ascontiguousarray(is_output, np.uint8)
+        es = np.ascontiguousarray(edge_src, np.int32)
+        ed = np.ascontiguousarray(edge_dst, np.int32)
+        el = np.ascontiguousarray(eligible, np.int32).reshape(-1)
+        lu = [np.asarray(u, np.int32) for u in late_users]
+        ptr = np.zeros(len(lu) + 1, np.int64)
+        for i, u in enumerate(lu):
+            ptr[i + 1] = ptr[i] + u.size
+        idx = np.ascontiguousarray(np.concatenate(lu) if lu else np.zeros(0, np.int32), np.int32)
+        self._keep = (ob, co, io, es, ed, el, ptr, idx)
+        d = GraphDesc(int(ob.size), _np_ptr(ob), _np_ptr(co), _np_ptr(io), int(es.size), _np_ptr(es),
+                      _np_ptr(ed), int(el.size), _np_ptr(el), ptr.ctypes.data_as(ctypes.c_void_p),
+                      _np_ptr(idx), float(swap_bytes_per_s), float(swap_latency_s))
+        h = ctypes.c_void_p()
+        _check(L.magis_graph_load(ctypes.byref(d), int(device), ctypes.byref(h)))
+        self._h = h
+        self.device = device
+        info = GraphInfo()
+        _check(L.magis_graph_info_get(h, ctypes.byref(info)))
+        self.info = {f: getattr(info, f) for f, _ in GraphInfo._fields_}
+        self.n_total = info.n_total
+        self.R = info.n_eligible
+        self.n = info.n_nodes
+
+    @classmethod
+    def from_workload(cls, wl, device: int = 0) -> "Graph":
+        return cls(wl.size, wl.cost, wl.is_output, wl.src, wl.dst, wl.elig, wl.U, wl.swap_Bps,
+                   wl.swap_lat, device)
+
+    def close(self):
+        if self._h:
+            self._L.magis_graph_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def eval_schedules(self, perm, dec=None, status=None, peak=None, latency=None, stream=None):
+        """perm: cuda int32 [K, n_total]; dec: cuda uint8 [K, R] (or None if R == 0).
+        Returns (status uint8 [K], peak int64 [K], latency float64 [K]) device tensors."""
+        import torch
+        K = int(perm.shape[0])
+        assert perm.dtype == torch.int32 and perm.is_cuda and perm.is_contiguous()
+        assert perm.shape[1] == self.n_total, (perm.shape, self.n_total)
+        if self.R:
+            assert dec is not None and dec.dtype == torch.uint8 and dec.is_contiguous()
+            assert dec.shape[0] == K and dec.shape[1] == self.R
+        dev = perm.device
+        status = torch.empty(K, dtype=torch.uint8, device=dev) if status is None else status
+        peak = torch.empty(K, dtype=torch.int64, device=dev) if peak is None else peak
+        latency = torch.empty(K, dtype=torch.float64, device=dev) if latency is None else latency
+        _check(self._L.magis_eval_schedules(self._h, K, _tptr(perm), _tptr(dec) if self.R else None,
+                                            _tptr(status), _tptr(peak), _tptr(latency),
+                                            _stream_ptr(stream)))
+        return status, peak, latency
+
+    def eval_schedules_host(self, perm: np.ndarray, dec: Optional[np.ndarray] = None, out=None,
+                            stream=None):
+        """End-to-end call with host buffers (pinned numpy views or torch CPU tensors)."""
+        import torch
+
+        def as_np(x, dt):
+            if isinstance(x, torch.Tensor):
+                return x.numpy()
+            return np.ascontiguousarray(x, dt)
+        p = as_np(perm, np.int32)
+        K = p.shape[0]
+        assert p.shape[1] == self.n_total
+        dd = as_np(dec, np.uint8) if (self.R and dec is not None) else None
+        if out is None:
+            st = np.empty(K, np.uint8)
+            pk = np.empty(K, np.int64)
+            lt = np.empty(K, np.float64)
+        else:
+            st, pk, lt = (as_np(o, None) for o in out)
+        _check(self._L.magis_eval_schedules_host(self._h, K, _np_ptr(p), _np_ptr(dd), _np_ptr(st),
+                                                 _np_ptr(pk), _np_ptr(lt), _stream_ptr(stream)))
+        return st, pk, lt
+
+
+def pareto_workspace_size(n: int) -> int:
+    return int(lib().magis_pareto_workspace_size(int(n)))
+
+
+def pareto_merge(peak, lat, status, ids=None, id_base: int = 0, cap: int = 4096,
+                 mem_limit: int = -1, lat_limit: float = -1.0, workspace=None, out=None, stream=None):
+    """Pareto front (ascending peak) + BetterThan-best ids, all on the device.
+    Returns dict of device tensors: front_id, front_peak, front_lat [cap],
+    front_n [1], best [2] (mem-limit mode, latency-limit mode)."""
+    import torch
+    n = int(peak.shape[0])
+    dev = peak.device
+    if out is None:
+        out = {"front_id": torch.empty(cap, dtype=torch.int64, device=dev),
+               "front_peak": torch.empty(cap, dtype=torch.int64, device=dev),
+               "front_lat": torch.empty(cap, dtype=torch.float64, device=dev),
+               "front_n": torch.empty(1, dtype=torch.int64, device=dev),
+               "best": torch.empty(2, dtype=torch.int64, device=dev)}
+    wsb = pareto_workspace_size(n)
+    if workspace is None or workspace.numel() < wsb:
+        workspace = torch.empty(max(wsb, 1), dtype=torch.uint8, device=dev)
+    _check(lib().magis_pareto_merge(n, _tptr(peak), _tptr(lat), _tptr(status), _tptr(ids), int(id_base),
+                                    int(cap), _tptr(out["front_id"]), _tptr(out["front_peak"]),
+                                    _tptr(out["front_lat"]), _tptr(out["front_n"]), int(mem_limit),
+                                    float(lat_limit), _tptr(out["best"]), _tptr(workspace),
+                                    int(workspace.numel()), _stream_ptr(stream)))
+    return out
