@@ -107,12 +107,13 @@ typedef struct magis_graph_info {
     int64_t n_edges;           /* deduplicated |E| */
     int64_t n_super_edges;     /* edges of the super-graph (all gates) */
     int32_t device;            /* CUDA device ordinal */
-    int32_t variant;           /* eval kernel variant: 0 = state in shared memory, 1 = global */
+    int32_t variant;           /* eval kernel: 0/1 = per-candidate state in smem/global, 2 = packed streams */
     int32_t grid;              /* persistent CTAs per eval launch */
     int32_t block;             /* threads per CTA */
     int64_t smem_bytes;        /* dynamic shared memory per CTA */
     int64_t table_bytes;       /* device bytes of the graph tables */
     double base_cost;          /* sum of cost(v) over original nodes */
+    int32_t pack;              /* candidates scored together per CTA step (variant 2), else 1 */
 } magis_graph_info;
 
 /*

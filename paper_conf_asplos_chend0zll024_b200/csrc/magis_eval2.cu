@@ -1,0 +1,655 @@
+// magis_eval2.cu -- the shared-memory-resident evaluation kernel (variant 2).
+//
+// Same per-candidate chain as magis_eval.cu (SURVEY §8(a) a2-a8, P:402-424,
+// P:1780-1789), re-laid out for sm_100a:
+//  * the graph lives in shared memory as per-thread "streams" (one u32 entry
+//    per node header and per edge, interleaved across the 32 lanes of a warp
+//    so every stream read is a conflict-free LDS), staged once per CTA with
+//    the bulk-copy engine (cp.async.bulk + mbarrier);
+//  * P candidates (1, 2 or 4) are scored at once: positions and last-use
+//    steps are u16 lanes packed into one 32/64-bit word per node, so each
+//    random gather, max and min over the consumer lists serves P candidates
+//    (VIMNMX.U16x2 / VIADD.16x2);
+//  * activation gates (Fig. 8 rules, reading P6) are folded into data: the
+//    positions of inactive optional nodes are zeroed and a late-user edge
+//    t_r -> b reads a per-candidate virtual slot holding pos(b) or 0, so the
+//    inner loops carry no decision tests;
+//  * positions are stored +1 (0 = absent / inactive), so validity is one
+//    running min of (q - 1) per node: a violation iff min < pos (unsigned);
+//  * alloc/free amounts land in per-step slots (u32 size units) in a
+//    transposed layout, so the scan's per-thread contiguous chunks read
+//    conflict-free;
+//  * the swap-latency sweep (the three in-order queues of reading P7) runs in
+//    a dedicated warp, one lane per candidate, fed through a double-buffered
+//    shared-memory hand-off guarded by named barriers, so the main warps go on
+//    to the next group while it runs.
+#include <climits>
+#include <cmath>
+
+#include "magis_internal.h"
+
+namespace magis {
+
+constexpr uint32_t kKindShift = 29;
+constexpr uint32_t kIdMask = (1u << kKindShift) - 1;
+constexpr uint32_t kHdrOut = 2, kHdrClone = 3, kNop = 7;   // kHdr = 1, kHdrCopy = 4
+constexpr int kBarMain = 1, kBarFull = 2, kBarEmpty = 4;
+constexpr int TM = kMainThreads2;
+constexpr int WM = TM / 32;
+
+// -------------------------------------------------------------- packed u16 --
+template <int P> struct Pk;
+template <> struct Pk<1> {
+    using V = uint32_t;
+    static __device__ __forceinline__ V load(const uint16_t* a, uint32_t i) { return a[i]; }
+    static __device__ __forceinline__ void store(uint16_t* a, uint32_t i, V v) { a[i] = (uint16_t)v; }
+    static __device__ __forceinline__ uint32_t get(V v, int) { return v & 0xffffu; }
+    static __device__ __forceinline__ V vmax(V a, V b) { return max(a, b); }
+    static __device__ __forceinline__ V vmin(V a, V b) { return min(a, b); }
+    static __device__ __forceinline__ V dec1(V a) { return (a - 1u) & 0xffffu; }
+    static __device__ __forceinline__ V ones() { return 0xffffu; }
+    static __device__ __forceinline__ V splat(uint32_t x) { return x; }
+    static __device__ __forceinline__ V nzmask(V a) { return a ? 0xffffu : 0u; }
+    static __device__ __forceinline__ V vand(V a, V b) { return a & b; }
+    static __device__ __forceinline__ bool maybe_eq(V a, V b) { return a == b; }
+};
+template <> struct Pk<2> {
+    using V = uint32_t;
+    static __device__ __forceinline__ V load(const uint16_t* a, uint32_t i) {
+        return reinterpret_cast<const uint32_t*>(a)[i];
+    }
+    static __device__ __forceinline__ void store(uint16_t* a, uint32_t i, V v) {
+        reinterpret_cast<uint32_t*>(a)[i] = v;
+    }
+    static __device__ __forceinline__ uint32_t get(V v, int c) { return (v >> (16 * c)) & 0xffffu; }
+    static __device__ __forceinline__ V vmax(V a, V b) { return __vmaxu2(a, b); }
+    static __device__ __forceinline__ V vmin(V a, V b) { return __vminu2(a, b); }
+    static __device__ __forceinline__ V dec1(V a) { return __vsub2(a, 0x00010001u); }
+    static __device__ __forceinline__ V ones() { return 0xffffffffu; }
+    static __device__ __forceinline__ V splat(uint32_t x) { return x | (x << 16); }
+    static __device__ __forceinline__ V nzmask(V a) { return __vcmpne2(a, 0u); }
+    static __device__ __forceinline__ V vand(V a, V b) { return a & b; }
+    static __device__ __forceinline__ bool maybe_eq(V a, V b) {
+        const uint32_t x = a ^ b;
+        return ((x - 0x00010001u) & ~x & 0x80008000u) != 0;
+    }
+};
+template <> struct Pk<4> {
+    using V = uint2;
+    static __device__ __forceinline__ V load(const uint16_t* a, uint32_t i) {
+        return reinterpret_cast<const uint2*>(a)[i];
+    }
+    static __device__ __forceinline__ void store(uint16_t* a, uint32_t i, V v) {
+        reinterpret_cast<uint2*>(a)[i] = v;
+    }
+    static __device__ __forceinline__ uint32_t get(V v, int c) {
+        return ((c < 2 ? v.x : v.y) >> (16 * (c & 1))) & 0xffffu;
+    }
+    static __device__ __forceinline__ V vmax(V a, V b) { return make_uint2(__vmaxu2(a.x, b.x), __vmaxu2(a.y, b.y)); }
+    static __device__ __forceinline__ V vmin(V a, V b) { return make_uint2(__vminu2(a.x, b.x), __vminu2(a.y, b.y)); }
+    static __device__ __forceinline__ V dec1(V a) {
+        return make_uint2(__vsub2(a.x, 0x00010001u), __vsub2(a.y, 0x00010001u));
+    }
+    static __device__ __forceinline__ V ones() { return make_uint2(0xffffffffu, 0xffffffffu); }
+    static __device__ __forceinline__ V splat(uint32_t x) { return make_uint2(x | (x << 16), x | (x << 16)); }
+    static __device__ __forceinline__ V nzmask(V a) { return make_uint2(__vcmpne2(a.x, 0u), __vcmpne2(a.y, 0u)); }
+    static __device__ __forceinline__ V vand(V a, V b) { return make_uint2(a.x & b.x, a.y & b.y); }
+    static __device__ __forceinline__ bool maybe_eq(V a, V b) {
+        const uint32_t x = a.x ^ b.x, y = a.y ^ b.y;
+        return ((((x - 0x00010001u) & ~x) | ((y - 0x00010001u) & ~y)) & 0x80008000u) != 0;
+    }
+};
+
+// ------------------------------------------------------------- barriers --
+// immediate barrier ids so ptxas reserves only the 6 barriers used
+__device__ __forceinline__ void bar_sync(int id, int n) {
+    switch (id) {
+        case 1: asm volatile("bar.sync 1, %0;" ::"r"(n) : "memory"); break;
+        case 2: asm volatile("bar.sync 2, %0;" ::"r"(n) : "memory"); break;
+        case 3: asm volatile("bar.sync 3, %0;" ::"r"(n) : "memory"); break;
+        case 4: asm volatile("bar.sync 4, %0;" ::"r"(n) : "memory"); break;
+        default: asm volatile("bar.sync 5, %0;" ::"r"(n) : "memory"); break;
+    }
+}
+__device__ __forceinline__ void bar_arrive(int id, int n) {
+    switch (id) {
+        case 2: asm volatile("bar.arrive 2, %0;" ::"r"(n) : "memory"); break;
+        case 3: asm volatile("bar.arrive 3, %0;" ::"r"(n) : "memory"); break;
+        case 4: asm volatile("bar.arrive 4, %0;" ::"r"(n) : "memory"); break;
+        default: asm volatile("bar.arrive 5, %0;" ::"r"(n) : "memory"); break;
+    }
+}
+
+// ------------------------------------------------- bulk copy (TMA engine) --
+__device__ __forceinline__ void bulk_stage(void* smem_dst, const void* gsrc, uint32_t bytes,
+                                           uint64_t* mbar) {
+    const uint32_t bar = (uint32_t)__cvta_generic_to_shared(mbar);
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(bar) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+        const uint32_t chunk = 1u << 15;
+        for (uint32_t o = 0; o < bytes; o += chunk) {
+            const uint32_t nb = min(chunk, bytes - o);
+            const uint32_t dst = (uint32_t)__cvta_generic_to_shared((char*)smem_dst + o);
+            asm volatile(
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+                "l"((const char*)gsrc + o), "r"(nb), "r"(bar)
+                : "memory");
+        }
+    }
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
+            : "=r"(done)
+            : "r"(bar)
+            : "memory");
+    }
+    __syncthreads();
+}
+
+// ------------------------------------------------------------ hand-off --
+struct SlotHdr {
+    long long k[4];
+    long long peak[4];      // in size units
+    double ctot[4];         // sum of compute costs (from the per-step scan)
+    double basel[4];        // base + clone costs (swap-free latency)
+    unsigned long long* key[4];   // [2 * cap]: unsorted keys, then sorted keys
+    double* cb[4];                // compute-cost prefix before each sorted event
+    int status[4];
+    int nev[4];
+    int cnt[4];             // gather counters
+};
+
+struct Ctl {
+    int flags[4];           // per-candidate status bits (atomicOr)
+    int viol[4];
+    int anysw;
+};
+
+template <int P>
+__global__ void __launch_bounds__(TM + 32)
+eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
+             const int32_t* __restrict__ perm, const uint8_t* __restrict__ dec,
+             uint8_t* __restrict__ out_status, int64_t* __restrict__ out_peak,
+             double* __restrict__ out_lat, char* __restrict__ ovf) {
+    using PK = Pk<P>;
+    using V = typename PK::V;
+    extern __shared__ __align__(128) char sm[];
+    __shared__ uint64_t mbar;
+    __shared__ SlotHdr hdr[2];
+    __shared__ Ctl ctl;
+    __shared__ long long red_s[WM][P];
+    __shared__ double red_c[WM][P];
+    __shared__ double red_b[WM][P];
+    __shared__ long long red_m[WM][P];
+    __shared__ int red_n[WM][P];
+
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int32_t NT = pl.NT, R = pl.R, n = pl.n;
+    const int32_t L = pl.L, S = pl.S, Sl = pl.L * pl.S, lgL = pl.lgL;
+
+    bulk_stage(sm, blob, pl.static_bytes, &mbar);
+    const uint32_t* wtab = (const uint32_t*)(sm + pl.off_wtab);   // [WM][4]: consumer rows, input rows
+    const uint2* crow = (const uint2*)(sm + pl.off_crow);
+    const uint32_t* chdr = (const uint32_t*)(sm + pl.off_chdr);
+    const uint32_t* cent = (const uint32_t*)(sm + pl.off_cent);
+    const uint2* frow = (const uint2*)(sm + pl.off_frow);
+    const uint32_t* fhdr = (const uint32_t*)(sm + pl.off_fhdr);
+    const uint32_t* fsz = (const uint32_t*)(sm + pl.off_fsz);
+    const double* fcost = (const double*)(sm + pl.off_fcost);
+    const uint32_t* fent = (const uint32_t*)(sm + pl.off_fent);
+    const uint32_t* size_s = (const uint32_t*)(sm + pl.off_size);
+    uint16_t* pos = (uint16_t*)(sm + pl.off_pos);
+    uint16_t* last = (uint16_t*)(sm + pl.off_last);
+    uint2* AF = (uint2*)(sm + pl.off_af);
+    double* Cst = (double*)(sm + pl.off_c);
+    uint8_t* dec_s = (uint8_t*)(sm + pl.off_dec);
+    double* cofs = (double*)(sm + pl.off_cofs);
+    double* endb_all = (double*)(sm + pl.off_end);
+    unsigned long long* evk_s = (unsigned long long*)(sm + pl.off_ev);               // [2][P][2*cap]
+    double* evcb_s = (double*)(sm + pl.off_ev + (size_t)2 * P * 2 * pl.evcap * 8);  // [2][P][cap]
+
+    // pos / last of the virtual and dummy slots start (and the dummy stays) 0
+    for (int i = tid; i < pl.NTX * P; i += blockDim.x) { pos[i] = 0; last[i] = 0; }
+    if (tid == 0) {
+        for (int c = 0; c < 4; c++) { ctl.flags[c] = 0; ctl.viol[c] = 0; }
+        ctl.anysw = 0;
+    }
+    __syncthreads();
+
+    const int64_t ngroups = (K + P - 1) / P;
+    const int ncta = (blockIdx.x < ngroups) ? (int)((ngroups - 1 - blockIdx.x) / gridDim.x + 1) : 0;
+
+    if (warp == WM) {
+        // ================= latency sweep warp (reading P7) ==================
+        for (int gi = 0; gi < ncta; gi++) {
+            const int slot = gi & 1;
+            bar_sync(kBarFull + slot, TM + 32);
+            const SlotHdr& h = hdr[slot];
+            if (lane < P) {
+                const long long k = h.k[lane];
+                if (k < K) {
+                    const int st = h.status[lane];
+                    double lat;
+                    if (st) {
+                        lat = __longlong_as_double(0x7ff0000000000000ll);
+                    } else if (h.nev[lane] == 0) {
+                        lat = h.basel[lane];
+                    } else {
+                        const int ne = h.nev[lane];
+                        const unsigned long long* key = h.key[lane] + ne;
+                        const double* cb = h.cb[lane];
+                        double* endb = endb_all + (size_t)lane * 3 * R;
+                        double D = 0.0, Td = 0.0, Th = 0.0;
+                        for (int e = 0; e < ne; e++) {
+                            const unsigned long long kk = key[e];
+                            const uint32_t type = (uint32_t)(kk >> 24) & 0xff;
+                            const int32_t r = (int32_t)(kk & 0xffffff);
+                            const double c = cb[e];
+                            if (type == kEvStall) {
+                                D = fmax(D, endb[3 * r + 2] - c);
+                            } else if (type == kEvProduce) {
+                                endb[3 * r + 0] = c + D + __ldg(g.tcost + r);
+                            } else if (type == kEvStore) {
+                                Td = fmax(Td, endb[3 * r + 0]) + __ldg(g.xfer + r);
+                                endb[3 * r + 1] = Td;
+                            } else {
+                                Th = fmax(Th, endb[3 * r + 1]) + __ldg(g.xfer + r);
+                                endb[3 * r + 2] = Th;
+                            }
+                        }
+                        lat = fmax(fmax(h.ctot[lane] + D, Td), Th);
+                    }
+                    out_status[k] = (uint8_t)st;
+                    out_peak[k] = st ? -1 : h.peak[lane] * pl.unit;
+                    out_lat[k] = lat;
+                }
+            }
+            __syncwarp();
+            if (gi + 2 < ncta) {
+                __threadfence_block();
+                bar_arrive(kBarEmpty + slot, TM + 32);
+            }
+        }
+        return;
+    }
+
+    // ========================= main warps =====================================
+    const int32_t NQ = NT >> 2;
+    for (int gi = 0; gi < ncta; gi++) {
+        const int64_t grp = blockIdx.x + (int64_t)gi * gridDim.x;
+        const int slot = gi & 1;
+        bool valid[P];
+#pragma unroll
+        for (int c = 0; c < P; c++) valid[c] = grp * P + c < K;
+        // ---- phase 0: decisions ---------------------------------------------
+        {
+            int sw = 0, bad[P];
+#pragma unroll
+            for (int c = 0; c < P; c++) bad[c] = 0;
+            for (int i = tid; i < P * R; i += TM) {
+                const int c = i / R, r = i - c * R;
+                const uint8_t d = valid[c] ? dec[(grp * P + c) * (int64_t)R + r] : 0;
+                dec_s[i] = d;
+                sw |= (d == 2);
+                if ((d > 2) | ((d == 1) & !(__ldg(g.rflag + r) & kRHasInput))) bad[c] = 1;
+            }
+            if (sw) atomicOr(&ctl.anysw, 1);
+#pragma unroll
+            for (int c = 0; c < P; c++)
+                if (bad[c]) atomicOr(&ctl.flags[c], MAGIS_ST_BAD_DEC);
+        }
+        // ---- phase 1: inverse permutation (pos stored +1) --------------------
+#pragma unroll
+        for (int c = 0; c < P; c++) {
+            if (!valid[c]) continue;
+            const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT;
+            int bad = 0;
+            if ((NT & 3) == 0) {
+                const int4* P4 = reinterpret_cast<const int4*>(Pp);
+                for (int32_t q = tid; q < NQ; q += TM) {
+                    const int4 v = __ldcs(P4 + q);
+                    const uint32_t i0 = 4u * q;
+                    if ((uint32_t)v.x < (uint32_t)NT) pos[v.x * P + c] = (uint16_t)(i0 + 1); else bad = 1;
+                    if ((uint32_t)v.y < (uint32_t)NT) pos[v.y * P + c] = (uint16_t)(i0 + 2); else bad = 1;
+                    if ((uint32_t)v.z < (uint32_t)NT) pos[v.z * P + c] = (uint16_t)(i0 + 3); else bad = 1;
+                    if ((uint32_t)v.w < (uint32_t)NT) pos[v.w * P + c] = (uint16_t)(i0 + 4); else bad = 1;
+                }
+            } else {
+                for (int32_t i = tid; i < NT; i += TM) {
+                    const int32_t v = __ldcs(Pp + i);
+                    if ((uint32_t)v < (uint32_t)NT) pos[v * P + c] = (uint16_t)(i + 1); else bad = 1;
+                }
+            }
+            if (bad) atomicOr(&ctl.flags[c], MAGIS_ST_NOT_PERM);
+        }
+        bar_sync(kBarMain, TM);
+        const bool anysw = ctl.anysw != 0;
+        // ---- phase 2: optional nodes, virtual late-user slots ------------------
+        double bl[P];
+        int nev[P];
+#pragma unroll
+        for (int c = 0; c < P; c++) { bl[c] = 0.0; nev[c] = 0; }
+        for (int32_t r = tid; r < R; r += TM) {
+            const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
+#pragma unroll
+            for (int c = 0; c < P; c++) {
+                if (!valid[c]) continue;
+                const uint8_t d = dec_s[c * R + r];
+#pragma unroll
+                for (int o = 0; o < 3; o++) {
+                    const int32_t id = n + 3 * r + o;
+                    const uint32_t p = pos[id * P + c];
+                    if (p == 0) {
+                        atomicOr(&ctl.flags[c], MAGIS_ST_NOT_PERM);
+                        continue;
+                    }
+                    const bool act = (o == 0) ? (d == 1) : (d == 2);
+                    if (!act) {
+                        const uint32_t st = p - 1;
+                        const uint32_t idx = (st & (L - 1)) * S + (st >> lgL);
+                        AF[c * Sl + idx] = make_uint2(0u, 0u);
+                        if (anysw) Cst[c * Sl + idx] = 0.0;
+                        pos[id * P + c] = 0;
+                    }
+                }
+                if (d == 1) bl[c] += __ldg(g.tcost + r);
+                if (d == 2) nev[c] += 3 + (u1 - u0);
+                for (int32_t j = u0; j < u1; j++) {
+                    const int32_t b = __ldg(g.U_idx + j);
+                    pos[(NT + j) * P + c] = (d == 0) ? pos[b * P + c] : (uint16_t)0;
+                }
+            }
+        }
+        bar_sync(kBarMain, TM);
+        // ---- phase 3: validity + last use over the consumer rows -----------------
+        {
+            int nperm = 0, viol = 0;
+            const uint32_t r0 = wtab[warp * 4 + 0], r1 = wtab[warp * 4 + 1];
+            for (uint32_t r = r0; r < r1; r++) {
+                const uint2 rw = crow[r];                     // (edge offset, degree): warp-uniform
+                const uint32_t h = chdr[r * 32 + lane];
+                const uint32_t kind = h >> kKindShift, id = h & kIdMask;
+                const V p = PK::load(pos, id);
+                V lst = p, mn = PK::ones();
+                const uint32_t* ent = cent + rw.x + lane;
+#pragma unroll 4
+                for (uint32_t j = 0; j < rw.y; j++) {
+                    const V q = PK::load(pos, ent[j * 32]);
+                    mn = PK::vmin(mn, PK::dec1(q));
+                    lst = PK::vmax(lst, q);
+                }
+                if (kind != kNop) {
+#pragma unroll
+                    for (int c = 0; c < P; c++) {
+                        const uint32_t pc = PK::get(p, c);
+                        if (kind < kHdrClone && pc == 0) nperm |= 1 << c;
+                        if (PK::get(mn, c) < pc) viol |= 1 << c;
+                    }
+                    V outv;
+                    if (kind == kHdrOut) outv = PK::splat((uint32_t)NT);
+                    else if (kind >= kHdrClone) outv = PK::vand(lst, PK::nzmask(p));   // inactive halves -> 0
+                    else outv = lst;
+                    PK::store(last, id, outv);
+                }
+            }
+#pragma unroll
+            for (int c = 0; c < P; c++) {
+                if (nperm & (1 << c)) atomicOr(&ctl.flags[c], MAGIS_ST_NOT_PERM);
+                if (viol & (1 << c)) atomicOr(&ctl.viol[c], MAGIS_ST_EDGE);
+            }
+        }
+        bar_sync(kBarMain, TM);
+        int status[P];
+        bool anyok = false;
+#pragma unroll
+        for (int c = 0; c < P; c++) {
+            const int f = ctl.flags[c];
+            status[c] = valid[c] ? (f ? f : ctl.viol[c]) : 0;
+            anyok |= valid[c] && status[c] == 0;
+        }
+        long long peak[P];
+        double ctot[P], basel[P];
+        int nevt[P];
+#pragma unroll
+        for (int c = 0; c < P; c++) { peak[c] = 0; ctot[c] = 0.0; basel[c] = 0.0; nevt[c] = 0; }
+        if (anyok) {
+            // ---- phase 4: frees over the input rows, per-step slots -------------
+            {
+                const uint32_t r0 = wtab[warp * 4 + 2], r1 = wtab[warp * 4 + 3];
+                for (uint32_t r = r0; r < r1; r++) {
+                    const uint2 rw = frow[r];
+                    const uint32_t h = fhdr[r * 32 + lane];
+                    const uint32_t kind = h >> kKindShift, id = h & kIdMask;
+                    const V p = PK::load(pos, id);
+                    const V lv = PK::load(last, id);
+                    const uint32_t A = fsz[r * 32 + lane];
+                    uint32_t fr[P];
+#pragma unroll
+                    for (int c = 0; c < P; c++) {
+                        const uint32_t pc = PK::get(p, c);
+                        fr[c] = (pc != 0 && PK::get(lv, c) == pc) ? A : 0u;   // no reader: freed after own step
+                    }
+                    const uint32_t* ent = fent + rw.x + lane;
+#pragma unroll 4
+                    for (uint32_t j = 0; j < rw.y; j++) {
+                        const uint32_t u = ent[j * 32];
+                        const V l = PK::load(last, u);
+                        if (PK::maybe_eq(l, p)) {
+                            const uint32_t su = size_s[u];
+#pragma unroll
+                            for (int c = 0; c < P; c++) {
+                                const uint32_t pc = PK::get(p, c);
+                                if (pc != 0 && PK::get(l, c) == pc) fr[c] += su;
+                            }
+                        }
+                    }
+                    if (kind != kNop) {
+                        const double cst = anysw ? fcost[r * 32 + lane] : 0.0;
+#pragma unroll
+                        for (int c = 0; c < P; c++) {
+                            const uint32_t pc = PK::get(p, c);
+                            if (pc == 0 || status[c] || !valid[c]) continue;
+                            const uint32_t st = pc - 1;
+                            const uint32_t idx = (st & (L - 1)) * S + (st >> lgL);
+                            AF[c * Sl + idx] = make_uint2(A, fr[c]);
+                            if (anysw) Cst[c * Sl + idx] = cst;
+                        }
+                    }
+                }
+            }
+            bar_sync(kBarMain, TM);
+            // ---- phase 5: scan of the (sum, max-prefix) monoid per candidate ----
+            long long s[P], m[P];
+            double cs_[P];
+#pragma unroll
+            for (int c = 0; c < P; c++) { s[c] = 0; m[c] = LLONG_MIN; cs_[c] = 0.0; }
+            if (tid < S) {
+                const int32_t lo = tid * L, hi = min(lo + L, NT);
+                for (int32_t i = lo, jj = 0; i < hi; i++, jj++) {
+                    const int32_t idx = jj * S + tid;
+#pragma unroll
+                    for (int c = 0; c < P; c++) {
+                        const uint2 af = AF[c * Sl + idx];
+                        s[c] += af.x;
+                        m[c] = max(m[c], s[c]);
+                        s[c] -= af.y;
+                        if (anysw) cs_[c] += Cst[c * Sl + idx];
+                    }
+                }
+            }
+            long long si[P];
+            double ci[P], bi[P];
+            int ni[P];
+#pragma unroll
+            for (int c = 0; c < P; c++) { si[c] = s[c]; ci[c] = cs_[c]; bi[c] = bl[c]; ni[c] = nev[c]; }
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+#pragma unroll
+                for (int c = 0; c < P; c++) {
+                    const long long ys = __shfl_up_sync(0xffffffffu, si[c], o);
+                    const double yc = __shfl_up_sync(0xffffffffu, ci[c], o);
+                    if (lane >= o) { si[c] += ys; ci[c] += yc; }
+                    bi[c] += __shfl_xor_sync(0xffffffffu, bi[c], o);
+                    ni[c] += __shfl_xor_sync(0xffffffffu, ni[c], o);
+                }
+            }
+            if (lane == 31) {
+#pragma unroll
+                for (int c = 0; c < P; c++) { red_s[warp][c] = si[c]; red_c[warp][c] = ci[c]; }
+            }
+            if (lane == 0) {
+#pragma unroll
+                for (int c = 0; c < P; c++) { red_b[warp][c] = bi[c]; red_n[warp][c] = ni[c]; }
+            }
+            bar_sync(kBarMain, TM);
+#pragma unroll
+            for (int c = 0; c < P; c++) {
+                long long off = si[c] - s[c];
+                double coff = ci[c] - cs_[c];
+                for (int w = 0; w < warp; w++) { off += red_s[w][c]; coff += red_c[w][c]; }
+                long long cand = (m[c] == LLONG_MIN) ? LLONG_MIN : off + m[c];
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) cand = max(cand, __shfl_xor_sync(0xffffffffu, cand, o));
+                if (lane == 0) red_m[warp][c] = cand;
+                if (anysw) cofs[tid * P + c] = coff;
+            }
+            bar_sync(kBarMain, TM);
+#pragma unroll
+            for (int c = 0; c < P; c++) {
+                long long pk = LLONG_MIN;
+                double ct = 0.0, b = g.base_cost;
+                int ne = 0;
+                for (int w = 0; w < WM; w++) {
+                    pk = max(pk, red_m[w][c]);
+                    ct += red_c[w][c];
+                    b += red_b[w][c];
+                    ne += red_n[w][c];
+                }
+                peak[c] = pk;
+                ctot[c] = ct;
+                basel[c] = b;
+                nevt[c] = (status[c] || !valid[c]) ? 0 : ne;
+            }
+        }
+        // ---- phase 6: swap events -> hand-off slot --------------------------------
+        if (gi >= 2) bar_sync(kBarEmpty + slot, TM + 32);
+        SlotHdr& h = hdr[slot];
+        bool anyev = false;
+#pragma unroll
+        for (int c = 0; c < P; c++) anyev |= nevt[c] > 0;
+        if (tid == 0) {
+#pragma unroll
+            for (int c = 0; c < P; c++) {
+                h.k[c] = valid[c] ? grp * P + c : LLONG_MAX;
+                h.status[c] = status[c];
+                h.peak[c] = peak[c];
+                h.ctot[c] = ctot[c];
+                h.basel[c] = basel[c];
+                h.nev[c] = nevt[c];
+                h.cnt[c] = 0;
+                if (nevt[c] <= pl.evcap) {
+                    h.key[c] = evk_s + (size_t)(slot * P + c) * 2 * pl.evcap;
+                    h.cb[c] = evcb_s + (size_t)(slot * P + c) * pl.evcap;
+                } else {
+                    char* ob = ovf + ((size_t)blockIdx.x * 8 + slot * 4 + c) * pl.ovf_stride;
+                    h.key[c] = (unsigned long long*)ob;
+                    h.cb[c] = (double*)(ob + (size_t)2 * pl.max_events * 8);
+                }
+            }
+        }
+        if (anyev) {
+            bar_sync(kBarMain, TM);
+            for (int32_t r = tid; r < R; r += TM) {
+                const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
+                const unsigned long long rr = (unsigned long long)r;
+#pragma unroll
+                for (int c = 0; c < P; c++) {
+                    if (nevt[c] == 0 || dec_s[c * R + r] != 2) continue;
+                    const int b0 = atomicAdd(&h.cnt[c], 3 + (u1 - u0));
+                    unsigned long long* kin = h.key[c];
+                    const unsigned long long pt = (unsigned long long)pos[__ldg(g.elig + r) * P + c] - 1;
+                    const unsigned long long ps = (unsigned long long)pos[(n + 3 * r + 1) * P + c] - 1;
+                    const unsigned long long pq = (unsigned long long)pos[(n + 3 * r + 2) * P + c] - 1;
+                    kin[b0 + 0] = (pt << 32) | ((unsigned long long)kEvProduce << 24) | rr;
+                    kin[b0 + 1] = (ps << 32) | ((unsigned long long)kEvStore << 24) | rr;
+                    kin[b0 + 2] = (pq << 32) | ((unsigned long long)kEvLoad << 24) | rr;
+                    for (int32_t j = u0; j < u1; j++) {
+                        const unsigned long long pb = (unsigned long long)pos[__ldg(g.U_idx + j) * P + c] - 1;
+                        kin[b0 + 3 + (j - u0)] = (pb << 32) | ((unsigned long long)kEvStall << 24) | rr;
+                    }
+                }
+            }
+            bar_sync(kBarMain, TM);
+            // rank sort (unique keys) + compute-cost prefix before each event
+            int tot = 0;
+#pragma unroll
+            for (int c = 0; c < P; c++) tot += nevt[c];
+            for (int q = tid; q < tot; q += TM) {
+                int c = 0, e = q;
+                while (e >= nevt[c]) { e -= nevt[c]; c++; }
+                const unsigned long long* kin = h.key[c];
+                const int ne = nevt[c];
+                const unsigned long long key = kin[e];
+                int rank = 0;
+                for (int j = 0; j < ne; j++) rank += (kin[j] < key);
+                const int32_t stp = (int32_t)(key >> 32);
+                const int32_t th = stp >> lgL;
+                double cb = cofs[th * P + c];
+                for (int32_t i = th * L, jj = 0; i < stp; i++, jj++) cb += Cst[c * Sl + jj * S + th];
+                h.key[c][ne + rank] = key;
+                h.cb[c][rank] = cb;
+            }
+        }
+        __threadfence_block();
+        bar_arrive(kBarFull + slot, TM + 32);
+        // reset the per-group control words for the next group, then make sure
+        // every main thread is done with pos / AF / ctl before they are reused
+        if (tid == 0) {
+            for (int c = 0; c < 4; c++) { ctl.flags[c] = 0; ctl.viol[c] = 0; }
+            ctl.anysw = 0;
+        }
+        // clear pos so a missing node (duplicate in perm) reads as 0 next group
+        {
+            const int nb = NT * P * 2;
+            uint4* p4 = reinterpret_cast<uint4*>(pos);
+            for (int i = tid; i < (nb >> 4); i += TM) p4[i] = make_uint4(0u, 0u, 0u, 0u);
+            for (int i = ((nb >> 4) << 3) + tid; i < NT * P; i += TM) pos[i] = 0;
+        }
+        bar_sync(kBarMain, TM);
+    }
+}
+
+cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
+    cudaError_t e;
+    const void* fn = pl.P == 4 ? (const void*)eval2_kernel<4> : pl.P == 2 ? (const void*)eval2_kernel<2>
+                                                                         : (const void*)eval2_kernel<1>;
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_total);
+    if (e != cudaSuccess) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, TM + 32, pl.smem_total);
+}
+
+cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, int grid,
+                         int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status,
+                         int64_t* peak, double* lat, cudaStream_t stream) {
+    if (K <= 0) return cudaSuccess;
+    const int64_t ngroups = (K + pl.P - 1) / pl.P;
+    const int gr = (int)std::min<int64_t>(grid, ngroups);
+    if (pl.P == 4)
+        eval2_kernel<4><<<gr, TM + 32, pl.smem_total, stream>>>(g, pl, (const char*)blob, K, perm, dec, status,
+                                                                peak, lat, (char*)ovf);
+    else if (pl.P == 2)
+        eval2_kernel<2><<<gr, TM + 32, pl.smem_total, stream>>>(g, pl, (const char*)blob, K, perm, dec, status,
+                                                                peak, lat, (char*)ovf);
+    else
+        eval2_kernel<1><<<gr, TM + 32, pl.smem_total, stream>>>(g, pl, (const char*)blob, K, perm, dec, status,
+                                                                peak, lat, (char*)ovf);
+    return cudaGetLastError();
+}
+
+}  // namespace magis

@@ -9,6 +9,7 @@
 // activation gate so that one static CSR serves every decision vector.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 #include <vector>
@@ -67,6 +68,13 @@ struct DeviceGuard {
     } while (0)
 
 size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+cudaError_t dispatch_eval(const magis_graph* g, int64_t K, const int32_t* perm, const uint8_t* dec,
+                          uint8_t* st, int64_t* pk, double* lt, cudaStream_t s) {
+    if (g->cfg.variant == 2)
+        return eval2_launch(g->dev, g->plan2, g->blob2, g->ovf2, g->cfg.grid, K, perm, dec, st, pk, lt, s);
+    return eval_launch(g->dev, g->cfg, g->gws, K, perm, dec, st, pk, lt, s);
+}
 
 }  // namespace
 
@@ -310,6 +318,47 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
         delete g;
         return set_error(MAGIS_E_CUDA, std::string("eval_configure: ") + cudaGetErrorString(e));
     }
+    // --- variant 2: packed streams in shared memory (magis_eval2.cu) -----------
+    {
+        const char* force = std::getenv("MAGIS_VARIANT");
+        const char* pforce = std::getenv("MAGIS_P");
+        const bool allow2 = !(force && std::atoi(force) != 2);
+        cudaDeviceProp prop;
+        if (allow2 && cudaGetDeviceProperties(&prop, device) == cudaSuccess) {
+            SuperGraphHost sg{n, R, NT, cons_ptr.data(), cons_ent.data(), in_ptr.data(), in_ent.data(),
+                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data()};
+            const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
+            const int cands[3] = {4, 2, 1};
+            for (int ci = 0; ci < 3; ci++) {
+                const int P = cands[ci];
+                if (pforce && std::atoi(pforce) != P) continue;
+                Plan2 pl;
+                std::vector<char> img;
+                if (!plan2_build(sg, P, cap, &pl, &img)) continue;
+                int occ = 0;
+                if (eval2_occupancy(pl, &occ) != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
+                void* b2 = nullptr;
+                void* ov = nullptr;
+                const int grid = prop.multiProcessorCount * occ;
+                if (cudaMalloc(&b2, img.size()) != cudaSuccess) { cudaGetLastError(); break; }
+                if (cudaMemcpy(b2, img.data(), img.size(), cudaMemcpyHostToDevice) != cudaSuccess ||
+                    cudaMalloc(&ov, (size_t)grid * 8 * pl.ovf_stride) != cudaSuccess) {
+                    cudaGetLastError();
+                    cudaFree(b2);
+                    break;
+                }
+                g->plan2 = pl;
+                g->blob2 = b2;
+                g->blob2_bytes = img.size();
+                g->ovf2 = ov;
+                g->cfg.variant = 2;
+                g->cfg.grid = grid;
+                g->cfg.block = kMainThreads2 + 32;
+                g->cfg.smem = pl.smem_total;
+                break;
+            }
+        }
+    }
     if (g->cfg.variant == 1) {
         g->gws_bytes = g->cfg.state_bytes * (size_t)g->cfg.grid;
         e = cudaMalloc(&g->gws, g->gws_bytes);
@@ -331,6 +380,8 @@ extern "C" int magis_graph_free(magis_graph* g) {
     cudaDeviceSynchronize();
     if (g->blob) cudaFree(g->blob);
     if (g->gws) cudaFree(g->gws);
+    if (g->blob2) cudaFree(g->blob2);
+    if (g->ovf2) cudaFree(g->ovf2);
     for (int i = 0; i < 2; i++) {
         if (g->stage[i]) cudaFree(g->stage[i]);
         if (g->ev_h2d[i]) cudaEventDestroy(g->ev_h2d[i]);
@@ -357,6 +408,7 @@ extern "C" int magis_graph_info_get(const magis_graph* g, magis_graph_info* info
     info->smem_bytes = (int64_t)g->cfg.smem;
     info->table_bytes = (int64_t)g->blob_bytes;
     info->base_cost = g->dev.base_cost;
+    info->pack = g->cfg.variant == 2 ? g->plan2.P : 1;
     return MAGIS_SUCCESS;
 }
 
@@ -371,8 +423,8 @@ extern "C" int magis_eval_schedules(const magis_graph* g, int64_t K, const int32
         return set_error(MAGIS_E_INVAL, "null device pointer");
     if (g->dev.R > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R > 0");
     DeviceGuard guard(g->device);
-    cudaError_t e = eval_launch(g->dev, g->cfg, g->gws, K, d_perm, d_dec, d_status, d_peak,
-                                d_latency, (cudaStream_t)cuda_stream);
+    cudaError_t e = dispatch_eval(g, K, d_perm, d_dec, d_status, d_peak, d_latency,
+                                  (cudaStream_t)cuda_stream);
     if (e != cudaSuccess) {
         cudaGetLastError();
         return set_error(MAGIS_E_CUDA, std::string("eval launch: ") + cudaGetErrorString(e));
@@ -429,7 +481,7 @@ extern "C" int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_
         if (R > 0) CK(cudaMemcpyAsync(dd, h_dec + k0 * R, (size_t)kc * R, cudaMemcpyHostToDevice, g->aux));
         CK(cudaEventRecord(g->ev_h2d[b], g->aux));
         CK(cudaStreamWaitEvent(s0, g->ev_h2d[b], 0));
-        cudaError_t e = eval_launch(g->dev, g->cfg, g->gws, kc, dp, R > 0 ? dd : nullptr, dst, dpk, dlt, s0);
+        cudaError_t e = dispatch_eval(g, kc, dp, R > 0 ? dd : nullptr, dst, dpk, dlt, s0);
         if (e != cudaSuccess) {
             cudaGetLastError();
             return set_error(MAGIS_E_CUDA, std::string("eval launch: ") + cudaGetErrorString(e));

@@ -5,6 +5,7 @@
 #include <cstddef>
 #include <cstdint>
 #include <string>
+#include <vector>
 
 #include <cuda_runtime.h>
 
@@ -52,8 +53,32 @@ struct DevGraph {
     double base_cost;          // sum of cost over original nodes
 };
 
+// Variant-2 plan (magis_eval2.cu): graph as per-thread streams in shared
+// memory, P candidates packed per u16 lane group.  Built on the host by
+// plan2_build; all offsets are bytes into the dynamic shared memory.
+constexpr int kMainThreads2 = 512;
+
+struct Plan2 {
+    int32_t P;            // candidates per group (1, 2, 4); 0 = not applicable
+    int32_t NT, NTX, n, R, nU;
+    int32_t L, S;         // scan chunk length / slot stride (L * S >= NT, S <= kMainThreads2)
+    int64_t unit;         // bytes per size unit (gcd of sizes)
+    int32_t evcap;        // events per candidate held in shared memory
+    int32_t max_events;   // 3R + |U|
+    int32_t lgL;          // L = 1 << lgL
+    uint32_t static_bytes;   // bulk-staged prefix (graph rows + size units)
+    uint32_t off_wtab;       // [WM][4]: consumer rows [b, e), input rows [b, e)
+    uint32_t off_crow, off_chdr, off_cent;                  // consumer rows: (offset, degree), headers, edges
+    uint32_t off_frow, off_fhdr, off_fsz, off_fcost, off_fent;   // input rows (+ per-node size / cost)
+    uint32_t off_size;       // [NTX] size units
+    uint32_t off_pos, off_last, off_af, off_c, off_dec, off_cofs, off_end, off_ev;
+    uint32_t smem_total;
+    uint64_t ovf_stride;  // bytes per overflow event region (global)
+};
+
 struct EvalConfig {
-    int variant;          // 0: per-candidate state in shared memory, 1: in global workspace
+    int variant;          // 0: per-candidate state in shared memory, 1: in global workspace,
+                          // 2: packed streams (magis_eval2.cu)
     int grid;
     int block;
     size_t smem;          // dynamic shared memory per CTA
@@ -65,6 +90,30 @@ struct StateLayout {
     size_t pos, last, A, Fr, C, evkey_in, evkey_out, evcb, endT, endS, endL, dec, total;
 };
 StateLayout state_layout(int32_t NT, int32_t R, int32_t max_events);
+
+// Host-side inputs of the variant-2 planner (super-graph in CSR form).
+struct SuperGraphHost {
+    int32_t n, R, NT;
+    const int32_t* cons_ptr;   // [NT+1]
+    const int2* cons_ent;      // (consumer, gate)
+    const int32_t* in_ptr;     // [NT+1]
+    const int2* in_ent;        // (input, gate)
+    const int64_t* size;       // [NT]
+    const double* cost;        // [NT]
+    const uint8_t* nflag;      // [NT]
+    const int32_t* U_ptr;      // [R+1]
+    const int32_t* U_idx;
+};
+
+// Build the variant-2 plan and its static shared-memory image for a given P.
+// Returns false if the graph does not fit (ids >= 65535, sizes beyond u32
+// units, or shared memory).
+bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* plan,
+                 std::vector<char>* image);
+cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, int grid,
+                         int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status,
+                         int64_t* peak, double* lat, cudaStream_t stream);
+cudaError_t eval2_occupancy(const Plan2& pl, int* blocks_per_sm);
 
 cudaError_t eval_configure(const DevGraph& g, int device, EvalConfig* cfg);
 cudaError_t eval_launch(const DevGraph& g, const EvalConfig& cfg, void* gws, int64_t K,
@@ -92,6 +141,10 @@ struct magis_graph {
     void* blob = nullptr;          // device tables
     size_t blob_bytes = 0;
     void* gws = nullptr;           // global per-CTA workspace (variant 1)
+    magis::Plan2 plan2{};          // variant 2 plan
+    void* blob2 = nullptr;         // variant 2 static shared-memory image
+    size_t blob2_bytes = 0;
+    void* ovf2 = nullptr;          // variant 2 event overflow scratch
     size_t gws_bytes = 0;
     int64_t n_edges = 0;
     int64_t n_super_edges = 0;

@@ -1,0 +1,224 @@
+// magis_plan.cu -- host-side planner of the variant-2 kernel (magis_eval2.cu).
+//
+// Turns the gated super-graph into warp-aligned "rows" held in shared memory:
+//  * a consumer row = 32 nodes (one per lane) of similar out-degree: a header
+//    (node id + kind) and deg edge entries stored lane-major, so every read is
+//    a conflict-free LDS and all lanes of a warp step through headers and
+//    edges in lock-step (no divergence); a late-user edge t_r -> b (active iff
+//    dec[r] == 0, reading P6) is redirected to the virtual slot NT + j
+//    (j = position of b in U) that the kernel fills per candidate;
+//  * an input row = 32 nodes of similar in-degree with their inputs (every
+//    gate: inactive ones never match, see magis_eval2.cu) plus the node's size
+//    units and compute cost;
+//  * rows are dealt longest-first onto the least loaded warp;
+//  * tensor sizes are stored in units of their gcd (u32), which keeps the
+//    scan exact (reading P14: sizes are multiples of the allocation grain).
+#include <algorithm>
+#include <cstring>
+#include <numeric>
+#include <queue>
+
+#include "magis_internal.h"
+
+namespace magis {
+
+namespace {
+constexpr uint32_t kKindShift = 29;
+constexpr uint32_t kEdge = 0, kHdr = 1, kHdrOut = 2, kHdrClone = 3, kHdrCopy = 4, kNop = 7;
+
+uint64_t gcd64(uint64_t a, uint64_t b) {
+    while (b) { uint64_t t = a % b; a = b; b = t; }
+    return a;
+}
+size_t a16(size_t x) { return (x + 15) / 16 * 16; }
+
+struct Rows {
+    std::vector<uint32_t> row;   // (offset, degree) pairs
+    std::vector<uint32_t> hdr;   // [nrows * 32]
+    std::vector<uint32_t> ent;   // edge entries, lane-major per row
+    std::vector<int32_t> node;   // [nrows * 32] node id or -1
+    std::vector<uint32_t> wtab;  // per warp [begin, end) rows
+};
+
+// Group nodes into rows of 32 by descending degree, deal rows onto warps.
+Rows make_rows(const std::vector<std::vector<uint32_t>>& lists, const std::vector<uint32_t>& hdrs,
+               uint32_t nop_entry, uint32_t nop_hdr, int WM) {
+    const int32_t N = (int32_t)lists.size();
+    std::vector<int32_t> order(N);
+    std::iota(order.begin(), order.end(), 0);
+    std::stable_sort(order.begin(), order.end(),
+                     [&](int32_t a, int32_t b) { return lists[a].size() > lists[b].size(); });
+    const int32_t nrows = (N + 31) / 32;
+    std::vector<uint32_t> deg(nrows, 0);
+    for (int32_t r = 0; r < nrows; r++)
+        for (int l = 0; l < 32 && r * 32 + l < N; l++)
+            deg[r] = std::max<uint32_t>(deg[r], (uint32_t)lists[order[r * 32 + l]].size());
+    // deal rows onto warps (longest first, least loaded)
+    std::vector<std::vector<int32_t>> wr(WM);
+    {
+        using It = std::pair<uint64_t, int>;
+        std::priority_queue<It, std::vector<It>, std::greater<It>> q;
+        for (int w = 0; w < WM; w++) q.push({0, w});
+        for (int32_t r = 0; r < nrows; r++) {   // rows already in descending degree
+            It it = q.top();
+            q.pop();
+            wr[it.second].push_back(r);
+            it.first += 1 + deg[r];
+            q.push(it);
+        }
+    }
+    Rows out;
+    out.wtab.resize(WM * 2);
+    for (int w = 0; w < WM; w++) {
+        out.wtab[2 * w] = (uint32_t)(out.row.size() / 2);
+        for (int32_t r : wr[w]) {
+            const uint32_t off = (uint32_t)out.ent.size();
+            out.row.push_back(off);
+            out.row.push_back(deg[r]);
+            out.ent.resize(off + (size_t)deg[r] * 32, nop_entry);
+            for (int l = 0; l < 32; l++) {
+                const int32_t i = r * 32 + l;
+                if (i < N) {
+                    const int32_t v = order[i];
+                    out.hdr.push_back(hdrs[v]);
+                    out.node.push_back(v);
+                    for (size_t j = 0; j < lists[v].size(); j++) out.ent[off + j * 32 + l] = lists[v][j];
+                } else {
+                    out.hdr.push_back(nop_hdr);
+                    out.node.push_back(-1);
+                }
+            }
+        }
+        out.wtab[2 * w + 1] = (uint32_t)(out.row.size() / 2);
+    }
+    return out;
+}
+}  // namespace
+
+bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, std::vector<char>* img) {
+    const int32_t NT = sg.NT, n = sg.n, R = sg.R;
+    const int32_t nU = R > 0 ? sg.U_ptr[R] : 0;
+    const int64_t NTX = (int64_t)NT + nU + 1;
+    if (NTX >= 65535 || NT < 1) return false;            // u16 positions (stored +1)
+    // size units
+    uint64_t gg = 0;
+    for (int32_t v = 0; v < NT; v++) if (sg.size[v] > 0) gg = gcd64(gg, (uint64_t)sg.size[v]);
+    if (gg == 0) gg = 1;
+    for (int32_t v = 0; v < NT; v++) {
+        uint64_t s = (uint64_t)sg.size[v] / gg;
+        for (int32_t e = sg.in_ptr[v]; e < sg.in_ptr[v + 1]; e++) s += (uint64_t)sg.size[sg.in_ent[e].x] / gg;
+        if (s > 0xffffffffull) return false;
+    }
+    auto virt = [&](int32_t r, int32_t b) -> int32_t {
+        for (int32_t j = sg.U_ptr[r]; j < sg.U_ptr[r + 1]; j++)
+            if (sg.U_idx[j] == b) return NT + j;
+        return -1;
+    };
+    std::vector<std::vector<uint32_t>> cons(NT), ins(NT);
+    std::vector<uint32_t> hdrs(NT);
+    for (int32_t u = 0; u < NT; u++) {
+        uint32_t kind;
+        if (u < n) kind = (sg.nflag[u] & kFlagOutput) ? kHdrOut : kHdr;
+        else kind = ((u - n) % 3 == 0) ? kHdrClone : kHdrCopy;
+        hdrs[u] = (kind << kKindShift) | (uint32_t)u;
+        for (int32_t e = sg.cons_ptr[u]; e < sg.cons_ptr[u + 1]; e++) {
+            const int2 ce = sg.cons_ent[e];
+            int32_t c = ce.x;
+            if (ce.y >= 0 && (ce.y & 3) == 0) {       // t_r -> b, b in U_r
+                c = virt(ce.y >> 2, ce.x);
+                if (c < 0) return false;
+            }
+            cons[u].push_back((kEdge << kKindShift) | (uint32_t)c);
+        }
+        for (int32_t e = sg.in_ptr[u]; e < sg.in_ptr[u + 1]; e++)
+            ins[u].push_back((kEdge << kKindShift) | (uint32_t)sg.in_ent[e].x);
+    }
+    const int WM = kMainThreads2 / 32;
+    const uint32_t dummy = (uint32_t)(NTX - 1);
+    const uint32_t nop = (kEdge << kKindShift) | dummy;
+    const uint32_t nophdr = (kNop << kKindShift) | dummy;
+    Rows cr = make_rows(cons, hdrs, nop, nophdr, WM);
+    Rows fr = make_rows(ins, hdrs, nop, nophdr, WM);
+    std::vector<uint32_t> wtab(WM * 4);
+    for (int w = 0; w < WM; w++) {
+        wtab[4 * w + 0] = cr.wtab[2 * w];
+        wtab[4 * w + 1] = cr.wtab[2 * w + 1];
+        wtab[4 * w + 2] = fr.wtab[2 * w];
+        wtab[4 * w + 3] = fr.wtab[2 * w + 1];
+    }
+    std::vector<uint32_t> fsz(fr.node.size(), 0);
+    std::vector<double> fcost(fr.node.size(), 0.0);
+    for (size_t i = 0; i < fr.node.size(); i++) {
+        const int32_t v = fr.node[i];
+        if (v < 0) continue;
+        fsz[i] = (uint32_t)((uint64_t)sg.size[v] / gg);
+        fcost[i] = (sg.nflag[v] & kFlagCompute) ? sg.cost[v] : 0.0;
+    }
+    std::vector<uint32_t> size_u(NTX, 0);
+    for (int32_t v = 0; v < NT; v++) size_u[v] = (uint32_t)((uint64_t)sg.size[v] / gg);
+
+    Plan2 p{};
+    p.P = P;
+    p.NT = NT;
+    p.NTX = (int32_t)NTX;
+    p.n = n;
+    p.R = R;
+    p.nU = nU;
+    {
+        int32_t Lmin = (NT + kMainThreads2 - 1) / kMainThreads2, lg = 0;
+        while ((1 << lg) < Lmin) lg++;
+        p.lgL = lg;
+        p.L = 1 << lg;
+        p.S = (NT + p.L - 1) / p.L;
+    }
+    p.unit = (int64_t)gg;
+    p.max_events = 3 * R + nU;
+    size_t o = 0;
+    p.off_wtab = (uint32_t)o;  o = a16(o + wtab.size() * 4);
+    p.off_crow = (uint32_t)o;  o = a16(o + cr.row.size() * 4);
+    p.off_chdr = (uint32_t)o;  o = a16(o + cr.hdr.size() * 4);
+    p.off_cent = (uint32_t)o;  o = a16(o + cr.ent.size() * 4);
+    p.off_frow = (uint32_t)o;  o = a16(o + fr.row.size() * 4);
+    p.off_fhdr = (uint32_t)o;  o = a16(o + fr.hdr.size() * 4);
+    p.off_fsz = (uint32_t)o;   o = a16(o + fsz.size() * 4);
+    p.off_fcost = (uint32_t)o; o = a16(o + fcost.size() * 8);
+    p.off_fent = (uint32_t)o;  o = a16(o + fr.ent.size() * 4);
+    p.off_size = (uint32_t)o;  o = a16(o + size_u.size() * 4);
+    p.static_bytes = (uint32_t)o;
+    const size_t Sl = (size_t)p.L * p.S;
+    p.off_pos = (uint32_t)o;  o = a16(o + (size_t)NTX * P * 2);
+    p.off_last = (uint32_t)o; o = a16(o + (size_t)NTX * P * 2);
+    p.off_af = (uint32_t)o;   o = a16(o + (size_t)P * Sl * 8);
+    p.off_c = (uint32_t)o;    o = a16(o + (size_t)P * Sl * 8);
+    p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
+    p.off_cofs = (uint32_t)o; o = a16(o + (size_t)kMainThreads2 * P * 8);
+    p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
+    p.off_ev = (uint32_t)o;
+    int cap = std::min(p.max_events, 192);
+    while (true) {
+        size_t need = o + (size_t)2 * P * (size_t)std::max(cap, 1) * 24;
+        if (need <= smem_cap) { p.smem_total = (uint32_t)a16(need); break; }
+        if (cap <= 16) return false;
+        cap /= 2;
+    }
+    p.evcap = std::max(cap, 1);
+    p.ovf_stride = (uint64_t)((std::max(p.max_events, 1) * 24 + 255) / 256 * 256);
+    *pl = p;
+    img->assign(p.static_bytes, 0);
+    auto put = [&](uint32_t off, const void* src, size_t bytes) {
+        if (bytes) std::memcpy(img->data() + off, src, bytes);
+    };
+    put(p.off_wtab, wtab.data(), wtab.size() * 4);
+    put(p.off_crow, cr.row.data(), cr.row.size() * 4);
+    put(p.off_chdr, cr.hdr.data(), cr.hdr.size() * 4);
+    put(p.off_cent, cr.ent.data(), cr.ent.size() * 4);
+    put(p.off_frow, fr.row.data(), fr.row.size() * 4);
+    put(p.off_fhdr, fr.hdr.data(), fr.hdr.size() * 4);
+    put(p.off_fsz, fsz.data(), fsz.size() * 4);
+    put(p.off_fcost, fcost.data(), fcost.size() * 8);
+    put(p.off_fent, fr.ent.data(), fr.ent.size() * 4);
+    put(p.off_size, size_u.data(), size_u.size() * 4);
+    return true;
+}
+
+}  // namespace magis

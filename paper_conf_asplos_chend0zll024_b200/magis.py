@@ -45,7 +45,8 @@ class GraphInfo(ctypes.Structure):
     _fields_ = [("n_nodes", ctypes.c_int32), ("n_eligible", ctypes.c_int32), ("n_total", ctypes.c_int32),
                 ("n_edges", ctypes.c_int64), ("n_super_edges", ctypes.c_int64), ("device", ctypes.c_int32),
                 ("variant", ctypes.c_int32), ("grid", ctypes.c_int32), ("block", ctypes.c_int32),
-                ("smem_bytes", ctypes.c_int64), ("table_bytes", ctypes.c_int64), ("base_cost", ctypes.c_double)]
+                ("smem_bytes", ctypes.c_int64), ("table_bytes", ctypes.c_int64), ("base_cost", ctypes.c_double),
+                ("pack", ctypes.c_int32)]
 
 
 _lib = None

@@ -23,6 +23,20 @@ from tests.test_oracle_pins import T1_EDGES, T2_EDGES, fig2a_graph, random_case,
 LAT_RTOL = 1e-9
 DEV = "cuda:0"
 
+# kernel variants: magis_eval.cu (v1, global state) and magis_eval2.cu with
+# P = 1 / 2 / 4 packed candidates; "auto" is what the loader picks.
+VARIANTS = {"auto": {}, "v1": {"MAGIS_VARIANT": "1"}, "p1": {"MAGIS_P": "1"},
+            "p2": {"MAGIS_P": "2"}, "p4": {"MAGIS_P": "4"}}
+
+
+@pytest.fixture(params=list(VARIANTS))
+def variant(request, monkeypatch):
+    for k in ("MAGIS_VARIANT", "MAGIS_P"):
+        monkeypatch.delenv(k, raising=False)
+    for k, v in VARIANTS[request.param].items():
+        monkeypatch.setenv(k, v)
+    return request.param
+
 
 def gpu_eval(g: Graph, perms: np.ndarray, decs) -> tuple:
     P = torch.from_numpy(np.ascontiguousarray(perms, np.int32)).to(DEV)
@@ -54,7 +68,7 @@ def both(n, edges, size, outputs, cost=None, elig=(), U=(), B=25e9, lam=1e-5):
     return o, g
 
 
-def test_paper_examples_on_gpu():
+def test_paper_examples_on_gpu(variant):
     n, edges, size, outs, f, b = fig2a_graph()
     o, g = both(n, edges, size, outs)
     st, pk, lt = gpu_eval(g, np.arange(64)[None], None)
@@ -78,14 +92,14 @@ def test_paper_examples_on_gpu():
       ([0, 6, 5, 1, 2, 3, 4], 2)], 50.0),
     ([([0, 5, 1, 2, 6, 3, 4], 2)], 100.0),
 ])
-def test_T1_toy_on_gpu(rows, B):
+def test_T1_toy_on_gpu(rows, B, variant):
     o, g = both(4, T1_EDGES, [100, 200, 200, 10], [3], cost=[1.0] * 4, elig=[0], U=[[3]], B=B, lam=0.0)
     perms = np.array([r[0] for r in rows])
     decs = np.array([[r[1]] for r in rows], np.uint8)
     assert_parity(*gpu_eval(g, perms, decs), *o.eval_batch(perms, decs))
 
 
-def test_T2_toy_on_gpu():
+def test_T2_toy_on_gpu(variant):
     o, g = both(5, T2_EDGES, [10, 100, 200, 200, 10], [4], cost=[0.0, 2.0, 1.0, 1.0, 1.0], elig=[1], U=[[4]])
     perms = np.array([[0, 1, 2, 3, 4, 5, 6, 7], [0, 1, 2, 3, 5, 4, 6, 7], [0, 1, 5, 2, 3, 4, 6, 7]])
     decs = np.array([[0], [1], [1]], np.uint8)
@@ -95,7 +109,7 @@ def test_T2_toy_on_gpu():
 
 
 @pytest.mark.parametrize("branches", [[4, 4], [3, 3, 2], [2, 2, 2, 2], [2, 2, 2, 1, 1]])
-def test_c1_diamonds_all_orders(branches):
+def test_c1_diamonds_all_orders(branches, variant):
     """C1: every topological order of a 10-op diamond (70..5040 orders)."""
     wl = models.diamond(branches, seed=1)
     edges = list(zip(wl.src.tolist(), wl.dst.tolist()))
@@ -107,7 +121,7 @@ def test_c1_diamonds_all_orders(branches):
     assert res[1].min() == ref[1].min()   # brute-force optimum
 
 
-def test_random_small_graphs_with_decisions():
+def test_random_small_graphs_with_decisions(variant):
     """Random DAGs of <= 11 ops with random eligible sets and decisions: valid
     orders, random shuffles (mostly invalid), duplicates, bad decisions."""
     rng = np.random.default_rng(2024)
@@ -150,7 +164,7 @@ def workload(request):
     return build_workload(request.param)
 
 
-def test_workload_parity(workload):
+def test_workload_parity(workload, variant):
     """C2 / C3 / C5 at K=2048 seeded candidates (75% random orders, 24% local
     moves, 1% transpositions; 5%/5% remat/swap), element by element."""
     wl = workload
@@ -158,24 +172,28 @@ def test_workload_parity(workload):
     P, D = gen.generate(0, 2048)
     g = Graph.from_workload(wl)
     o = OracleGraph.from_workload(wl)
+    if variant in ("p1", "p2", "p4") and g.info["variant"] == 2:
+        assert g.info["pack"] == int(variant[1])
+    if variant == "v1":
+        assert g.info["variant"] in (0, 1)
     res = gpu_eval(g, P, D)
     ref = o.eval_batch(P, D)
     assert_parity(*res, *ref)
     assert (ref[0] == 0).mean() > 0.95 and (ref[0] == 2).any()
 
 
-def test_c4_large_graph_parity():
+def test_c4_large_graph_parity(variant):
     """C4 (~23.5k super-graph nodes): the global-state variant."""
     wl = build_workload("c4")
     gen = CandidateGenerator(wl, CandidateSpec(seed=3))
     P, D = gen.generate(0, 96)
     g = Graph.from_workload(wl)
-    assert g.info["variant"] == 1
+    assert g.info["variant"] in (1, 2)
     o = OracleGraph.from_workload(wl)
     assert_parity(*gpu_eval(g, P, D), *o.eval_batch(P, D))
 
 
-def test_c2_full_size_sampled():
+def test_c2_full_size_sampled(variant):
     """BASELINE configs[1] at full size (64k candidates, the bench's launch):
     every candidate's status and sampled candidates against the oracle."""
     wl = build_workload("c2")
@@ -207,7 +225,7 @@ def test_host_path_matches_device_path():
         np.testing.assert_array_equal(a, b)
 
 
-def test_k_zero_and_one_and_ragged():
+def test_k_zero_and_one_and_ragged(variant):
     wl = models.diamond([3, 2], seed=3)           # NT = 7: rows not 16-byte aligned
     edges = list(zip(wl.src.tolist(), wl.dst.tolist()))
     o, g = both(wl.n, edges, wl.size.tolist(), [wl.n - 1])
