@@ -171,8 +171,19 @@ struct Ctl {
     int anysw;
 };
 
-template <int P>
-__global__ void __launch_bounds__(TM + 32)
+// per-group results of the cross-warp fold (written by warp 0)
+struct Fold {
+    long long peak[4];
+    double ctot[4];
+    double basel[4];
+    int nev[4];
+    double woff[4][WM];     // exclusive compute-cost prefix per warp
+};
+
+constexpr long long kNegInf = -(1ll << 62);
+
+template <int P, int LMAX>
+__global__ void __launch_bounds__(TM + 32, 1)
 eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
              const int32_t* __restrict__ perm, const uint8_t* __restrict__ dec,
              uint8_t* __restrict__ out_status, int64_t* __restrict__ out_peak,
@@ -183,11 +194,12 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     __shared__ uint64_t mbar;
     __shared__ SlotHdr hdr[2];
     __shared__ Ctl ctl;
-    __shared__ long long red_s[WM][P];
-    __shared__ double red_c[WM][P];
-    __shared__ double red_b[WM][P];
-    __shared__ long long red_m[WM][P];
-    __shared__ int red_n[WM][P];
+    __shared__ Fold fold;
+    __shared__ long long agg_s[WM][P];
+    __shared__ long long agg_m[WM][P];
+    __shared__ double agg_c[WM][P];
+    __shared__ double agg_b[WM][P];
+    __shared__ int agg_n[WM][P];
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int32_t NT = pl.NT, R = pl.R, n = pl.n;
@@ -200,16 +212,14 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const uint32_t* cent = (const uint32_t*)(sm + pl.off_cent);
     const uint2* frow = (const uint2*)(sm + pl.off_frow);
     const uint32_t* fhdr = (const uint32_t*)(sm + pl.off_fhdr);
-    const uint32_t* fsz = (const uint32_t*)(sm + pl.off_fsz);
-    const double* fcost = (const double*)(sm + pl.off_fcost);
     const uint32_t* fent = (const uint32_t*)(sm + pl.off_fent);
     const uint32_t* size_s = (const uint32_t*)(sm + pl.off_size);
+    const double* cost_s = (const double*)(sm + pl.off_cost);
     uint16_t* pos = (uint16_t*)(sm + pl.off_pos);
     uint16_t* last = (uint16_t*)(sm + pl.off_last);
-    uint2* AF = (uint2*)(sm + pl.off_af);
-    double* Cst = (double*)(sm + pl.off_c);
+    uint32_t* Fs = (uint32_t*)(sm + pl.off_af);           // [P][Sl] bytes freed after each step (units)
     uint8_t* dec_s = (uint8_t*)(sm + pl.off_dec);
-    double* cofs = (double*)(sm + pl.off_cofs);
+    double* cofs = (double*)(sm + pl.off_cofs);           // [TM][P] cost prefix within the warp
     double* endb_all = (double*)(sm + pl.off_end);
     unsigned long long* evk_s = (unsigned long long*)(sm + pl.off_ev);               // [2][P][2*cap]
     double* evcb_s = (double*)(sm + pl.off_ev + (size_t)2 * P * 2 * pl.evcap * 8);  // [2][P][cap]
@@ -280,7 +290,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     }
 
     // ========================= main warps =====================================
-    const int32_t NQ = NT >> 2;
+    const int32_t lo = tid * L;                 // this thread's step chunk [lo, lo + L)
+    const bool vec4 = (NT & 3) == 0;
     for (int gi = 0; gi < ncta; gi++) {
         const int64_t grp = blockIdx.x + (int64_t)gi * gridDim.x;
         const int slot = gi & 1;
@@ -304,27 +315,41 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             for (int c = 0; c < P; c++)
                 if (bad[c]) atomicOr(&ctl.flags[c], MAGIS_ST_BAD_DEC);
         }
-        // ---- phase 1: inverse permutation (pos stored +1) --------------------
+        // ---- phase 1: inverse permutation (pos stored +1); this thread's
+        //      chunk of every candidate's perm stays in registers for the scan
+        int32_t pr[P][LMAX];
 #pragma unroll
         for (int c = 0; c < P; c++) {
-            if (!valid[c]) continue;
-            const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT;
+            const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT + lo;
             int bad = 0;
-            if ((NT & 3) == 0) {
-                const int4* P4 = reinterpret_cast<const int4*>(Pp);
-                for (int32_t q = tid; q < NQ; q += TM) {
-                    const int4 v = __ldcs(P4 + q);
-                    const uint32_t i0 = 4u * q;
+#pragma unroll
+            for (int j = 0; j < LMAX; j += 4) {
+                int4 v = make_int4(-1, -1, -1, -1);
+                if (valid[c] && j < L && lo + j < NT) {
+                    if (vec4) {
+                        v = __ldcs(reinterpret_cast<const int4*>(Pp + j));
+                    } else {
+                        v.x = __ldcs(Pp + j);
+                        if (lo + j + 1 < NT) v.y = __ldcs(Pp + j + 1);
+                        if (lo + j + 2 < NT) v.z = __ldcs(Pp + j + 2);
+                        if (lo + j + 3 < NT) v.w = __ldcs(Pp + j + 3);
+                    }
+                    const uint32_t i0 = (uint32_t)(lo + j);
                     if ((uint32_t)v.x < (uint32_t)NT) pos[v.x * P + c] = (uint16_t)(i0 + 1); else bad = 1;
-                    if ((uint32_t)v.y < (uint32_t)NT) pos[v.y * P + c] = (uint16_t)(i0 + 2); else bad = 1;
-                    if ((uint32_t)v.z < (uint32_t)NT) pos[v.z * P + c] = (uint16_t)(i0 + 3); else bad = 1;
-                    if ((uint32_t)v.w < (uint32_t)NT) pos[v.w * P + c] = (uint16_t)(i0 + 4); else bad = 1;
+                    if (i0 + 1 < (uint32_t)NT) {
+                        if ((uint32_t)v.y < (uint32_t)NT) pos[v.y * P + c] = (uint16_t)(i0 + 2); else bad = 1;
+                    }
+                    if (i0 + 2 < (uint32_t)NT) {
+                        if ((uint32_t)v.z < (uint32_t)NT) pos[v.z * P + c] = (uint16_t)(i0 + 3); else bad = 1;
+                    }
+                    if (i0 + 3 < (uint32_t)NT) {
+                        if ((uint32_t)v.w < (uint32_t)NT) pos[v.w * P + c] = (uint16_t)(i0 + 4); else bad = 1;
+                    }
                 }
-            } else {
-                for (int32_t i = tid; i < NT; i += TM) {
-                    const int32_t v = __ldcs(Pp + i);
-                    if ((uint32_t)v < (uint32_t)NT) pos[v * P + c] = (uint16_t)(i + 1); else bad = 1;
-                }
+                pr[c][j] = v.x;
+                if (j + 1 < LMAX) pr[c][j + 1] = v.y;
+                if (j + 2 < LMAX) pr[c][j + 2] = v.z;
+                if (j + 3 < LMAX) pr[c][j + 3] = v.w;
             }
             if (bad) atomicOr(&ctl.flags[c], MAGIS_ST_NOT_PERM);
         }
@@ -352,9 +377,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     const bool act = (o == 0) ? (d == 1) : (d == 2);
                     if (!act) {
                         const uint32_t st = p - 1;
-                        const uint32_t idx = (st & (L - 1)) * S + (st >> lgL);
-                        AF[c * Sl + idx] = make_uint2(0u, 0u);
-                        if (anysw) Cst[c * Sl + idx] = 0.0;
+                        Fs[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = 0u;
                         pos[id * P + c] = 0;
                     }
                 }
@@ -413,13 +436,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             status[c] = valid[c] ? (f ? f : ctl.viol[c]) : 0;
             anyok |= valid[c] && status[c] == 0;
         }
-        long long peak[P];
-        double ctot[P], basel[P];
-        int nevt[P];
-#pragma unroll
-        for (int c = 0; c < P; c++) { peak[c] = 0; ctot[c] = 0.0; basel[c] = 0.0; nevt[c] = 0; }
         if (anyok) {
-            // ---- phase 4: frees over the input rows, per-step slots -------------
+            // ---- phase 4: frees over the input rows -> per-step slots ------------
             {
                 const uint32_t r0 = wtab[warp * 4 + 2], r1 = wtab[warp * 4 + 3];
                 for (uint32_t r = r0; r < r1; r++) {
@@ -428,12 +446,19 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     const uint32_t kind = h >> kKindShift, id = h & kIdMask;
                     const V p = PK::load(pos, id);
                     const V lv = PK::load(last, id);
-                    const uint32_t A = fsz[r * 32 + lane];
                     uint32_t fr[P];
+                    bool selff = false;
 #pragma unroll
                     for (int c = 0; c < P; c++) {
                         const uint32_t pc = PK::get(p, c);
-                        fr[c] = (pc != 0 && PK::get(lv, c) == pc) ? A : 0u;   // no reader: freed after own step
+                        const bool m = pc != 0 && PK::get(lv, c) == pc;    // no reader: freed after own step
+                        selff |= m;
+                        fr[c] = m ? 1u : 0u;
+                    }
+                    if (selff) {
+                        const uint32_t A = size_s[id];
+#pragma unroll
+                        for (int c = 0; c < P; c++) fr[c] *= A;
                     }
                     const uint32_t* ent = fent + rw.x + lane;
 #pragma unroll 4
@@ -450,107 +475,122 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         }
                     }
                     if (kind != kNop) {
-                        const double cst = anysw ? fcost[r * 32 + lane] : 0.0;
 #pragma unroll
                         for (int c = 0; c < P; c++) {
                             const uint32_t pc = PK::get(p, c);
                             if (pc == 0 || status[c] || !valid[c]) continue;
                             const uint32_t st = pc - 1;
-                            const uint32_t idx = (st & (L - 1)) * S + (st >> lgL);
-                            AF[c * Sl + idx] = make_uint2(A, fr[c]);
-                            if (anysw) Cst[c * Sl + idx] = cst;
+                            Fs[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = fr[c];
                         }
                     }
                 }
             }
             bar_sync(kBarMain, TM);
             // ---- phase 5: scan of the (sum, max-prefix) monoid per candidate ----
+            //      alloc = size of the op at each step (perm chunk in registers),
+            //      free = Fs slot; compute cost per step for the swap sweep
             long long s[P], m[P];
             double cs_[P];
 #pragma unroll
-            for (int c = 0; c < P; c++) { s[c] = 0; m[c] = LLONG_MIN; cs_[c] = 0.0; }
-            if (tid < S) {
-                const int32_t lo = tid * L, hi = min(lo + L, NT);
-                for (int32_t i = lo, jj = 0; i < hi; i++, jj++) {
-                    const int32_t idx = jj * S + tid;
+            for (int c = 0; c < P; c++) { s[c] = 0; m[c] = kNegInf; cs_[c] = 0.0; }
+#pragma unroll
+            for (int j = 0; j < LMAX; j++) {
+                if (j < L && lo + j < NT) {
 #pragma unroll
                     for (int c = 0; c < P; c++) {
-                        const uint2 af = AF[c * Sl + idx];
-                        s[c] += af.x;
+                        const int32_t v = pr[c][j];
+                        if ((uint32_t)v >= (uint32_t)NT) continue;     // invalid candidate: ignored later
+                        const bool act = v < n || pos[v * P + c] != 0;
+                        const uint32_t A = act ? size_s[v] : 0u;
+                        s[c] += A;
                         m[c] = max(m[c], s[c]);
-                        s[c] -= af.y;
-                        if (anysw) cs_[c] += Cst[c * Sl + idx];
+                        s[c] -= Fs[c * Sl + j * S + tid];
+                        if (anysw && act) cs_[c] += cost_s[v];
                     }
                 }
             }
-            long long si[P];
-            double ci[P], bi[P];
+            // warp-level monoid scan: (s1, m1) then (s2, m2) = (s1 + s2, max(m1, s1 + m2))
+            double bi[P];
             int ni[P];
 #pragma unroll
-            for (int c = 0; c < P; c++) { si[c] = s[c]; ci[c] = cs_[c]; bi[c] = bl[c]; ni[c] = nev[c]; }
+            for (int c = 0; c < P; c++) {
+                long long ss = s[c], mm = m[c];
+                double cc = cs_[c];
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-#pragma unroll
-                for (int c = 0; c < P; c++) {
-                    const long long ys = __shfl_up_sync(0xffffffffu, si[c], o);
-                    const double yc = __shfl_up_sync(0xffffffffu, ci[c], o);
-                    if (lane >= o) { si[c] += ys; ci[c] += yc; }
-                    bi[c] += __shfl_xor_sync(0xffffffffu, bi[c], o);
-                    ni[c] += __shfl_xor_sync(0xffffffffu, ni[c], o);
+                for (int o = 1; o < 32; o <<= 1) {
+                    const long long ps = __shfl_up_sync(0xffffffffu, ss, o);
+                    const long long pm = __shfl_up_sync(0xffffffffu, mm, o);
+                    const double pc = __shfl_up_sync(0xffffffffu, cc, o);
+                    if (lane >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
                 }
-            }
-            if (lane == 31) {
+                if (anysw) cofs[tid * P + c] = cc - cs_[c];
+                if (lane == 31) { agg_s[warp][c] = ss; agg_m[warp][c] = mm; agg_c[warp][c] = cc; }
+                double b = bl[c];
+                int nn = nev[c];
 #pragma unroll
-                for (int c = 0; c < P; c++) { red_s[warp][c] = si[c]; red_c[warp][c] = ci[c]; }
+                for (int o = 16; o > 0; o >>= 1) {
+                    b += __shfl_xor_sync(0xffffffffu, b, o);
+                    nn += __shfl_xor_sync(0xffffffffu, nn, o);
+                }
+                bi[c] = b;
+                ni[c] = nn;
             }
             if (lane == 0) {
 #pragma unroll
-                for (int c = 0; c < P; c++) { red_b[warp][c] = bi[c]; red_n[warp][c] = ni[c]; }
+                for (int c = 0; c < P; c++) { agg_b[warp][c] = bi[c]; agg_n[warp][c] = ni[c]; }
             }
             bar_sync(kBarMain, TM);
+            if (warp == 0) {
+                // fold the WM warp aggregates (lanes >= WM hold the identity)
 #pragma unroll
-            for (int c = 0; c < P; c++) {
-                long long off = si[c] - s[c];
-                double coff = ci[c] - cs_[c];
-                for (int w = 0; w < warp; w++) { off += red_s[w][c]; coff += red_c[w][c]; }
-                long long cand = (m[c] == LLONG_MIN) ? LLONG_MIN : off + m[c];
+                for (int c = 0; c < P; c++) {
+                    long long ss = lane < WM ? agg_s[lane][c] : 0;
+                    long long mm = lane < WM ? agg_m[lane][c] : kNegInf;
+                    double cc = lane < WM ? agg_c[lane][c] : 0.0;
+                    double b = lane < WM ? agg_b[lane][c] : 0.0;
+                    int nn = lane < WM ? agg_n[lane][c] : 0;
+                    const double c0 = cc;
 #pragma unroll
-                for (int o = 16; o > 0; o >>= 1) cand = max(cand, __shfl_xor_sync(0xffffffffu, cand, o));
-                if (lane == 0) red_m[warp][c] = cand;
-                if (anysw) cofs[tid * P + c] = coff;
-            }
-            bar_sync(kBarMain, TM);
-#pragma unroll
-            for (int c = 0; c < P; c++) {
-                long long pk = LLONG_MIN;
-                double ct = 0.0, b = g.base_cost;
-                int ne = 0;
-                for (int w = 0; w < WM; w++) {
-                    pk = max(pk, red_m[w][c]);
-                    ct += red_c[w][c];
-                    b += red_b[w][c];
-                    ne += red_n[w][c];
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const long long ps = __shfl_up_sync(0xffffffffu, ss, o);
+                        const long long pm = __shfl_up_sync(0xffffffffu, mm, o);
+                        const double pc = __shfl_up_sync(0xffffffffu, cc, o);
+                        if (lane >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
+                        b += __shfl_xor_sync(0xffffffffu, b, o == 1 ? 16 : o >> 1);
+                        nn += __shfl_xor_sync(0xffffffffu, nn, o == 1 ? 16 : o >> 1);
+                    }
+                    if (lane < WM) fold.woff[c][lane] = cc - c0;
+                    if (lane == 31) {
+                        fold.peak[c] = mm;
+                        fold.ctot[c] = cc;
+                        fold.basel[c] = g.base_cost + b;
+                        fold.nev[c] = (status[c] || !valid[c]) ? 0 : nn;
+                    }
                 }
-                peak[c] = pk;
-                ctot[c] = ct;
-                basel[c] = b;
-                nevt[c] = (status[c] || !valid[c]) ? 0 : ne;
             }
+            bar_sync(kBarMain, TM);
+        } else if (tid == 0) {
+#pragma unroll
+            for (int c = 0; c < P; c++) { fold.peak[c] = 0; fold.ctot[c] = 0.0; fold.basel[c] = 0.0; fold.nev[c] = 0; }
+        }
+        int nevt[P];
+        bool anyev = false;
+#pragma unroll
+        for (int c = 0; c < P; c++) {
+            nevt[c] = anyok ? fold.nev[c] : 0;
+            anyev |= nevt[c] > 0;
         }
         // ---- phase 6: swap events -> hand-off slot --------------------------------
         if (gi >= 2) bar_sync(kBarEmpty + slot, TM + 32);
         SlotHdr& h = hdr[slot];
-        bool anyev = false;
-#pragma unroll
-        for (int c = 0; c < P; c++) anyev |= nevt[c] > 0;
         if (tid == 0) {
 #pragma unroll
             for (int c = 0; c < P; c++) {
                 h.k[c] = valid[c] ? grp * P + c : LLONG_MAX;
                 h.status[c] = status[c];
-                h.peak[c] = peak[c];
-                h.ctot[c] = ctot[c];
-                h.basel[c] = basel[c];
+                h.peak[c] = fold.peak[c];
+                h.ctot[c] = fold.ctot[c];
+                h.basel[c] = fold.basel[c];
                 h.nev[c] = nevt[c];
                 h.cnt[c] = 0;
                 if (nevt[c] <= pl.evcap) {
@@ -586,7 +626,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 }
             }
             bar_sync(kBarMain, TM);
-            // rank sort (unique keys) + compute-cost prefix before each event
+            // rank sort (unique keys) + compute-cost prefix before each event:
+            // cost of the steps of earlier warps' chunks, earlier lanes of the
+            // same warp, then the steps of the owning chunk before the event
             int tot = 0;
 #pragma unroll
             for (int c = 0; c < P; c++) tot += nevt[c];
@@ -600,8 +642,12 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 for (int j = 0; j < ne; j++) rank += (kin[j] < key);
                 const int32_t stp = (int32_t)(key >> 32);
                 const int32_t th = stp >> lgL;
-                double cb = cofs[th * P + c];
-                for (int32_t i = th * L, jj = 0; i < stp; i++, jj++) cb += Cst[c * Sl + jj * S + th];
+                double cb = fold.woff[c][th >> 5] + cofs[th * P + c];
+                const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT;
+                for (int32_t i = th * L; i < stp; i++) {
+                    const int32_t v = __ldg(Pp + i);
+                    if (v < n || pos[v * P + c] != 0) cb += cost_s[v];
+                }
                 h.key[c][ne + rank] = key;
                 h.cb[c][rank] = cb;
             }
@@ -609,11 +655,13 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         __threadfence_block();
         bar_arrive(kBarFull + slot, TM + 32);
         // reset the per-group control words for the next group, then make sure
-        // every main thread is done with pos / AF / ctl before they are reused
+        // every main thread is done with pos / Fs / ctl before they are reused
         if (tid == 0) {
             for (int c = 0; c < 4; c++) { ctl.flags[c] = 0; ctl.viol[c] = 0; }
             ctl.anysw = 0;
         }
+        // every main thread must be done reading pos (event keys, cost prefix)
+        if (anyev) bar_sync(kBarMain, TM);
         // clear pos so a missing node (duplicate in perm) reads as 0 next group
         {
             const int nb = NT * P * 2;
@@ -625,11 +673,21 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     }
 }
 
+template <int P>
+static const void* kernel_ptr(int lmax) {
+    if (lmax <= 4) return (const void*)eval2_kernel<P, 4>;
+    if (lmax <= 8) return (const void*)eval2_kernel<P, 8>;
+    return (const void*)eval2_kernel<P, 16>;
+}
+
+static const void* kernel_for(const Plan2& pl) {
+    return pl.P == 4 ? kernel_ptr<4>(pl.L) : pl.P == 2 ? kernel_ptr<2>(pl.L) : kernel_ptr<1>(pl.L);
+}
+
 cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
-    cudaError_t e;
-    const void* fn = pl.P == 4 ? (const void*)eval2_kernel<4> : pl.P == 2 ? (const void*)eval2_kernel<2>
-                                                                         : (const void*)eval2_kernel<1>;
-    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_total);
+    if (pl.L > 16) { *blocks = 0; return cudaSuccess; }
+    const void* fn = kernel_for(pl);
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_total);
     if (e != cudaSuccess) return e;
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, TM + 32, pl.smem_total);
 }
@@ -640,16 +698,9 @@ cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, v
     if (K <= 0) return cudaSuccess;
     const int64_t ngroups = (K + pl.P - 1) / pl.P;
     const int gr = (int)std::min<int64_t>(grid, ngroups);
-    if (pl.P == 4)
-        eval2_kernel<4><<<gr, TM + 32, pl.smem_total, stream>>>(g, pl, (const char*)blob, K, perm, dec, status,
-                                                                peak, lat, (char*)ovf);
-    else if (pl.P == 2)
-        eval2_kernel<2><<<gr, TM + 32, pl.smem_total, stream>>>(g, pl, (const char*)blob, K, perm, dec, status,
-                                                                peak, lat, (char*)ovf);
-    else
-        eval2_kernel<1><<<gr, TM + 32, pl.smem_total, stream>>>(g, pl, (const char*)blob, K, perm, dec, status,
-                                                                peak, lat, (char*)ovf);
-    return cudaGetLastError();
+    void* args[] = {(void*)&g, (void*)&pl, (void*)&blob, (void*)&K, (void*)&perm, (void*)&dec,
+                    (void*)&status, (void*)&peak, (void*)&lat, (void*)&ovf};
+    return cudaLaunchKernel(kernel_for(pl), dim3(gr), dim3(TM + 32), args, pl.smem_total, stream);
 }
 
 }  // namespace magis

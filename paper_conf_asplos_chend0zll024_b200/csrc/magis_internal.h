@@ -69,9 +69,10 @@ struct Plan2 {
     uint32_t static_bytes;   // bulk-staged prefix (graph rows + size units)
     uint32_t off_wtab;       // [WM][4]: consumer rows [b, e), input rows [b, e)
     uint32_t off_crow, off_chdr, off_cent;                  // consumer rows: (offset, degree), headers, edges
-    uint32_t off_frow, off_fhdr, off_fsz, off_fcost, off_fent;   // input rows (+ per-node size / cost)
+    uint32_t off_frow, off_fhdr, off_fent;                  // input rows
     uint32_t off_size;       // [NTX] size units
-    uint32_t off_pos, off_last, off_af, off_c, off_dec, off_cofs, off_end, off_ev;
+    uint32_t off_cost;       // [NTX] compute cost (f64; clone = cost(t_r), Store / Load 0)
+    uint32_t off_pos, off_last, off_af, off_dec, off_cofs, off_end, off_ev;   // off_af: free slots
     uint32_t smem_total;
     uint64_t ovf_stride;  // bytes per overflow event region (global)
 };

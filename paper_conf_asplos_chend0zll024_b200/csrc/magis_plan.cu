@@ -146,16 +146,12 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
         wtab[4 * w + 2] = fr.wtab[2 * w];
         wtab[4 * w + 3] = fr.wtab[2 * w + 1];
     }
-    std::vector<uint32_t> fsz(fr.node.size(), 0);
-    std::vector<double> fcost(fr.node.size(), 0.0);
-    for (size_t i = 0; i < fr.node.size(); i++) {
-        const int32_t v = fr.node[i];
-        if (v < 0) continue;
-        fsz[i] = (uint32_t)((uint64_t)sg.size[v] / gg);
-        fcost[i] = (sg.nflag[v] & kFlagCompute) ? sg.cost[v] : 0.0;
-    }
     std::vector<uint32_t> size_u(NTX, 0);
-    for (int32_t v = 0; v < NT; v++) size_u[v] = (uint32_t)((uint64_t)sg.size[v] / gg);
+    std::vector<double> cost_u(NTX, 0.0);
+    for (int32_t v = 0; v < NT; v++) {
+        size_u[v] = (uint32_t)((uint64_t)sg.size[v] / gg);
+        cost_u[v] = (sg.nflag[v] & kFlagCompute) ? sg.cost[v] : 0.0;
+    }
 
     Plan2 p{};
     p.P = P;
@@ -165,7 +161,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     p.R = R;
     p.nU = nU;
     {
-        int32_t Lmin = (NT + kMainThreads2 - 1) / kMainThreads2, lg = 0;
+        int32_t Lmin = std::max(4, (NT + kMainThreads2 - 1) / kMainThreads2), lg = 0;
         while ((1 << lg) < Lmin) lg++;
         p.lgL = lg;
         p.L = 1 << lg;
@@ -180,21 +176,19 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     p.off_cent = (uint32_t)o;  o = a16(o + cr.ent.size() * 4);
     p.off_frow = (uint32_t)o;  o = a16(o + fr.row.size() * 4);
     p.off_fhdr = (uint32_t)o;  o = a16(o + fr.hdr.size() * 4);
-    p.off_fsz = (uint32_t)o;   o = a16(o + fsz.size() * 4);
-    p.off_fcost = (uint32_t)o; o = a16(o + fcost.size() * 8);
     p.off_fent = (uint32_t)o;  o = a16(o + fr.ent.size() * 4);
     p.off_size = (uint32_t)o;  o = a16(o + size_u.size() * 4);
+    p.off_cost = (uint32_t)o;  o = a16(o + cost_u.size() * 8);
     p.static_bytes = (uint32_t)o;
     const size_t Sl = (size_t)p.L * p.S;
     p.off_pos = (uint32_t)o;  o = a16(o + (size_t)NTX * P * 2);
     p.off_last = (uint32_t)o; o = a16(o + (size_t)NTX * P * 2);
-    p.off_af = (uint32_t)o;   o = a16(o + (size_t)P * Sl * 8);
-    p.off_c = (uint32_t)o;    o = a16(o + (size_t)P * Sl * 8);
+    p.off_af = (uint32_t)o;   o = a16(o + (size_t)P * Sl * 4);
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
     p.off_cofs = (uint32_t)o; o = a16(o + (size_t)kMainThreads2 * P * 8);
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
     p.off_ev = (uint32_t)o;
-    int cap = std::min(p.max_events, 192);
+    int cap = std::min(p.max_events, 64);
     while (true) {
         size_t need = o + (size_t)2 * P * (size_t)std::max(cap, 1) * 24;
         if (need <= smem_cap) { p.smem_total = (uint32_t)a16(need); break; }
@@ -214,10 +208,9 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     put(p.off_cent, cr.ent.data(), cr.ent.size() * 4);
     put(p.off_frow, fr.row.data(), fr.row.size() * 4);
     put(p.off_fhdr, fr.hdr.data(), fr.hdr.size() * 4);
-    put(p.off_fsz, fsz.data(), fsz.size() * 4);
-    put(p.off_fcost, fcost.data(), fcost.size() * 8);
     put(p.off_fent, fr.ent.data(), fr.ent.size() * 4);
     put(p.off_size, size_u.data(), size_u.size() * 4);
+    put(p.off_cost, cost_u.data(), cost_u.size() * 8);
     return true;
 }
 
