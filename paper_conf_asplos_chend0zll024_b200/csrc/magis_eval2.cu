@@ -177,7 +177,7 @@ struct Fold {
     double ctot[4];
     double basel[4];
     int nev[4];
-    double woff[4][WM];     // exclusive compute-cost prefix per warp
+    double woff[WM];        // exclusive compute-cost prefix of each warp within its team
 };
 
 constexpr long long kNegInf = -(1ll << 62);
@@ -195,9 +195,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     __shared__ SlotHdr hdr[2];
     __shared__ Ctl ctl;
     __shared__ Fold fold;
-    __shared__ long long agg_s[WM][P];
-    __shared__ long long agg_m[WM][P];
-    __shared__ double agg_c[WM][P];
+    __shared__ long long agg_s[WM];
+    __shared__ long long agg_m[WM];
+    __shared__ double agg_c[WM];
     __shared__ double agg_b[WM][P];
     __shared__ int agg_n[WM][P];
 
@@ -209,17 +209,17 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const uint32_t* wtab = (const uint32_t*)(sm + pl.off_wtab);   // [WM][4]: consumer rows, input rows
     const uint2* crow = (const uint2*)(sm + pl.off_crow);
     const uint32_t* chdr = (const uint32_t*)(sm + pl.off_chdr);
-    const uint32_t* cent = (const uint32_t*)(sm + pl.off_cent);
+    const uint16_t* cent = (const uint16_t*)(sm + pl.off_cent);
     const uint2* frow = (const uint2*)(sm + pl.off_frow);
     const uint32_t* fhdr = (const uint32_t*)(sm + pl.off_fhdr);
-    const uint32_t* fent = (const uint32_t*)(sm + pl.off_fent);
+    const uint16_t* fent = (const uint16_t*)(sm + pl.off_fent);
     const uint32_t* size_s = (const uint32_t*)(sm + pl.off_size);
     const double* cost_s = (const double*)(sm + pl.off_cost);
     uint16_t* pos = (uint16_t*)(sm + pl.off_pos);
     uint16_t* last = (uint16_t*)(sm + pl.off_last);
     uint32_t* Fs = (uint32_t*)(sm + pl.off_af);           // [P][Sl] bytes freed after each step (units)
     uint8_t* dec_s = (uint8_t*)(sm + pl.off_dec);
-    double* cofs = (double*)(sm + pl.off_cofs);           // [TM][P] cost prefix within the warp
+    double* cofs = (double*)(sm + pl.off_cofs);           // [TM] cost prefix within the warp
     double* endb_all = (double*)(sm + pl.off_end);
     unsigned long long* evk_s = (unsigned long long*)(sm + pl.off_ev);               // [2][P][2*cap]
     double* evcb_s = (double*)(sm + pl.off_ev + (size_t)2 * P * 2 * pl.evcap * 8);  // [2][P][cap]
@@ -290,7 +290,11 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     }
 
     // ========================= main warps =====================================
-    const int32_t lo = tid * L;                 // this thread's step chunk [lo, lo + L)
+    // phases 1 and 5: candidate cm of the group is handled by team cm (TPC
+    // threads, WT warps); thread tt of the team owns steps [lo, lo + L)
+    constexpr int TPC = TM / P, WT = WM / P;
+    const int cm = tid / TPC, tt = tid - cm * TPC;
+    const int32_t lo = tt * L;
     const bool vec4 = (NT & 3) == 0;
     for (int gi = 0; gi < ncta; gi++) {
         const int64_t grp = blockIdx.x + (int64_t)gi * gridDim.x;
@@ -316,16 +320,18 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 if (bad[c]) atomicOr(&ctl.flags[c], MAGIS_ST_BAD_DEC);
         }
         // ---- phase 1: inverse permutation (pos stored +1); this thread's
-        //      chunk of every candidate's perm stays in registers for the scan
-        int32_t pr[P][LMAX];
-#pragma unroll
-        for (int c = 0; c < P; c++) {
-            const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT + lo;
+        //      chunk of its team's candidate stays in registers for the scan
+        int32_t pr[LMAX];
+        {
+            const int32_t* Pp = perm + (grp * P + cm) * (int64_t)NT + lo;
             int bad = 0;
+            bool vc = false;
+#pragma unroll
+            for (int c = 0; c < P; c++) vc |= (c == cm) && valid[c];
 #pragma unroll
             for (int j = 0; j < LMAX; j += 4) {
                 int4 v = make_int4(-1, -1, -1, -1);
-                if (valid[c] && j < L && lo + j < NT) {
+                if (vc && j < L && lo + j < NT) {
                     if (vec4) {
                         v = __ldcs(reinterpret_cast<const int4*>(Pp + j));
                     } else {
@@ -335,23 +341,23 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         if (lo + j + 3 < NT) v.w = __ldcs(Pp + j + 3);
                     }
                     const uint32_t i0 = (uint32_t)(lo + j);
-                    if ((uint32_t)v.x < (uint32_t)NT) pos[v.x * P + c] = (uint16_t)(i0 + 1); else bad = 1;
+                    if ((uint32_t)v.x < (uint32_t)NT) pos[v.x * P + cm] = (uint16_t)(i0 + 1); else bad = 1;
                     if (i0 + 1 < (uint32_t)NT) {
-                        if ((uint32_t)v.y < (uint32_t)NT) pos[v.y * P + c] = (uint16_t)(i0 + 2); else bad = 1;
+                        if ((uint32_t)v.y < (uint32_t)NT) pos[v.y * P + cm] = (uint16_t)(i0 + 2); else bad = 1;
                     }
                     if (i0 + 2 < (uint32_t)NT) {
-                        if ((uint32_t)v.z < (uint32_t)NT) pos[v.z * P + c] = (uint16_t)(i0 + 3); else bad = 1;
+                        if ((uint32_t)v.z < (uint32_t)NT) pos[v.z * P + cm] = (uint16_t)(i0 + 3); else bad = 1;
                     }
                     if (i0 + 3 < (uint32_t)NT) {
-                        if ((uint32_t)v.w < (uint32_t)NT) pos[v.w * P + c] = (uint16_t)(i0 + 4); else bad = 1;
+                        if ((uint32_t)v.w < (uint32_t)NT) pos[v.w * P + cm] = (uint16_t)(i0 + 4); else bad = 1;
                     }
                 }
-                pr[c][j] = v.x;
-                if (j + 1 < LMAX) pr[c][j + 1] = v.y;
-                if (j + 2 < LMAX) pr[c][j + 2] = v.z;
-                if (j + 3 < LMAX) pr[c][j + 3] = v.w;
+                pr[j] = v.x;
+                if (j + 1 < LMAX) pr[j + 1] = v.y;
+                if (j + 2 < LMAX) pr[j + 2] = v.z;
+                if (j + 3 < LMAX) pr[j + 3] = v.w;
             }
-            if (bad) atomicOr(&ctl.flags[c], MAGIS_ST_NOT_PERM);
+            if (bad) atomicOr(&ctl.flags[cm], MAGIS_ST_NOT_PERM);
         }
         bar_sync(kBarMain, TM);
         const bool anysw = ctl.anysw != 0;
@@ -360,32 +366,33 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         int nev[P];
 #pragma unroll
         for (int c = 0; c < P; c++) { bl[c] = 0.0; nev[c] = 0; }
-        for (int32_t r = tid; r < R; r += TM) {
+        for (int q = tid; q < P * R; q += TM) {
+            const int c = q / R, r = q - c * R;
             const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
 #pragma unroll
-            for (int c = 0; c < P; c++) {
-                if (!valid[c]) continue;
-                const uint8_t d = dec_s[c * R + r];
+            for (int cc = 0; cc < P; cc++) {
+                if (cc != c || !valid[cc]) continue;
+                const uint8_t d = dec_s[cc * R + r];
 #pragma unroll
                 for (int o = 0; o < 3; o++) {
                     const int32_t id = n + 3 * r + o;
-                    const uint32_t p = pos[id * P + c];
+                    const uint32_t p = pos[id * P + cc];
                     if (p == 0) {
-                        atomicOr(&ctl.flags[c], MAGIS_ST_NOT_PERM);
+                        atomicOr(&ctl.flags[cc], MAGIS_ST_NOT_PERM);
                         continue;
                     }
                     const bool act = (o == 0) ? (d == 1) : (d == 2);
                     if (!act) {
                         const uint32_t st = p - 1;
-                        Fs[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = 0u;
-                        pos[id * P + c] = 0;
+                        Fs[cc * Sl + (st & (L - 1)) * S + (st >> lgL)] = 0u;
+                        pos[id * P + cc] = 0;
                     }
                 }
-                if (d == 1) bl[c] += __ldg(g.tcost + r);
-                if (d == 2) nev[c] += 3 + (u1 - u0);
+                if (d == 1) bl[cc] += __ldg(g.tcost + r);
+                if (d == 2) nev[cc] += 3 + (u1 - u0);
                 for (int32_t j = u0; j < u1; j++) {
                     const int32_t b = __ldg(g.U_idx + j);
-                    pos[(NT + j) * P + c] = (d == 0) ? pos[b * P + c] : (uint16_t)0;
+                    pos[(NT + j) * P + cc] = (d == 0) ? pos[b * P + cc] : (uint16_t)0;
                 }
             }
         }
@@ -400,7 +407,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const uint32_t kind = h >> kKindShift, id = h & kIdMask;
                 const V p = PK::load(pos, id);
                 V lst = p, mn = PK::ones();
-                const uint32_t* ent = cent + rw.x + lane;
+                const uint16_t* ent = cent + rw.x + lane;
 #pragma unroll 4
                 for (uint32_t j = 0; j < rw.y; j++) {
                     const V q = PK::load(pos, ent[j * 32]);
@@ -460,7 +467,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 #pragma unroll
                         for (int c = 0; c < P; c++) fr[c] *= A;
                     }
-                    const uint32_t* ent = fent + rw.x + lane;
+                    const uint16_t* ent = fent + rw.x + lane;
 #pragma unroll 4
                     for (uint32_t j = 0; j < rw.y; j++) {
                         const uint32_t u = ent[j * 32];
@@ -486,36 +493,29 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 }
             }
             bar_sync(kBarMain, TM);
-            // ---- phase 5: scan of the (sum, max-prefix) monoid per candidate ----
-            //      alloc = size of the op at each step (perm chunk in registers),
-            //      free = Fs slot; compute cost per step for the swap sweep
-            long long s[P], m[P];
-            double cs_[P];
-#pragma unroll
-            for (int c = 0; c < P; c++) { s[c] = 0; m[c] = kNegInf; cs_[c] = 0.0; }
+            // ---- phase 5: scan of the (sum, max-prefix) monoid ------------------
+            //      team cm scans candidate cm: alloc = size of the op at each step
+            //      (perm chunk in registers), free = Fs slot, compute cost per step
+            long long s1 = 0, m1 = kNegInf;
+            double cs1 = 0.0;
 #pragma unroll
             for (int j = 0; j < LMAX; j++) {
                 if (j < L && lo + j < NT) {
-#pragma unroll
-                    for (int c = 0; c < P; c++) {
-                        const int32_t v = pr[c][j];
-                        if ((uint32_t)v >= (uint32_t)NT) continue;     // invalid candidate: ignored later
-                        const bool act = v < n || pos[v * P + c] != 0;
+                    const int32_t v = pr[j];
+                    if ((uint32_t)v < (uint32_t)NT) {                // else: invalid candidate, ignored
+                        const bool act = v < n || pos[v * P + cm] != 0;
                         const uint32_t A = act ? size_s[v] : 0u;
-                        s[c] += A;
-                        m[c] = max(m[c], s[c]);
-                        s[c] -= Fs[c * Sl + j * S + tid];
-                        if (anysw && act) cs_[c] += cost_s[v];
+                        s1 += A;
+                        m1 = max(m1, s1);
+                        s1 -= Fs[cm * Sl + j * S + tt];
+                        if (anysw && act) cs1 += cost_s[v];
                     }
                 }
             }
-            // warp-level monoid scan: (s1, m1) then (s2, m2) = (s1 + s2, max(m1, s1 + m2))
-            double bi[P];
-            int ni[P];
-#pragma unroll
-            for (int c = 0; c < P; c++) {
-                long long ss = s[c], mm = m[c];
-                double cc = cs_[c];
+            {
+                // warp-level monoid scan: (s1, m1) then (s2, m2) = (s1 + s2, max(m1, s1 + m2))
+                long long ss = s1, mm = m1;
+                double cc = cs1;
 #pragma unroll
                 for (int o = 1; o < 32; o <<= 1) {
                     const long long ps = __shfl_up_sync(0xffffffffu, ss, o);
@@ -523,46 +523,50 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     const double pc = __shfl_up_sync(0xffffffffu, cc, o);
                     if (lane >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
                 }
-                if (anysw) cofs[tid * P + c] = cc - cs_[c];
-                if (lane == 31) { agg_s[warp][c] = ss; agg_m[warp][c] = mm; agg_c[warp][c] = cc; }
-                double b = bl[c];
-                int nn = nev[c];
+                if (anysw) cofs[tid] = cc - cs1;
+                if (lane == 31) { agg_s[warp] = ss; agg_m[warp] = mm; agg_c[warp] = cc; }
 #pragma unroll
-                for (int o = 16; o > 0; o >>= 1) {
-                    b += __shfl_xor_sync(0xffffffffu, b, o);
-                    nn += __shfl_xor_sync(0xffffffffu, nn, o);
+                for (int c = 0; c < P; c++) {
+                    double b = bl[c];
+                    int nn = nev[c];
+#pragma unroll
+                    for (int o = 16; o > 0; o >>= 1) {
+                        b += __shfl_xor_sync(0xffffffffu, b, o);
+                        nn += __shfl_xor_sync(0xffffffffu, nn, o);
+                    }
+                    if (lane == 0) { agg_b[warp][c] = b; agg_n[warp][c] = nn; }
                 }
-                bi[c] = b;
-                ni[c] = nn;
-            }
-            if (lane == 0) {
-#pragma unroll
-                for (int c = 0; c < P; c++) { agg_b[warp][c] = bi[c]; agg_n[warp][c] = ni[c]; }
             }
             bar_sync(kBarMain, TM);
             if (warp == 0) {
-                // fold the WM warp aggregates (lanes >= WM hold the identity)
+                // fold the WT warp aggregates of each team (segments of WT lanes)
+                long long ss = lane < WM ? agg_s[lane] : 0;
+                long long mm = lane < WM ? agg_m[lane] : kNegInf;
+                double cc = lane < WM ? agg_c[lane] : 0.0;
+                const double c0 = cc;
+#pragma unroll
+                for (int o = 1; o < WT; o <<= 1) {
+                    const long long ps = __shfl_up_sync(0xffffffffu, ss, o, WT);
+                    const long long pm = __shfl_up_sync(0xffffffffu, mm, o, WT);
+                    const double pc = __shfl_up_sync(0xffffffffu, cc, o, WT);
+                    if ((lane % WT) >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
+                }
+                if (lane < WM) fold.woff[lane] = cc - c0;
+                if (lane < WM && (lane % WT) == WT - 1) {
+                    const int c = lane / WT;
+                    fold.peak[c] = mm;
+                    fold.ctot[c] = cc;
+                }
 #pragma unroll
                 for (int c = 0; c < P; c++) {
-                    long long ss = lane < WM ? agg_s[lane][c] : 0;
-                    long long mm = lane < WM ? agg_m[lane][c] : kNegInf;
-                    double cc = lane < WM ? agg_c[lane][c] : 0.0;
                     double b = lane < WM ? agg_b[lane][c] : 0.0;
                     int nn = lane < WM ? agg_n[lane][c] : 0;
-                    const double c0 = cc;
 #pragma unroll
-                    for (int o = 1; o < 32; o <<= 1) {
-                        const long long ps = __shfl_up_sync(0xffffffffu, ss, o);
-                        const long long pm = __shfl_up_sync(0xffffffffu, mm, o);
-                        const double pc = __shfl_up_sync(0xffffffffu, cc, o);
-                        if (lane >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
-                        b += __shfl_xor_sync(0xffffffffu, b, o == 1 ? 16 : o >> 1);
-                        nn += __shfl_xor_sync(0xffffffffu, nn, o == 1 ? 16 : o >> 1);
+                    for (int o = 16; o > 0; o >>= 1) {
+                        b += __shfl_xor_sync(0xffffffffu, b, o);
+                        nn += __shfl_xor_sync(0xffffffffu, nn, o);
                     }
-                    if (lane < WM) fold.woff[c][lane] = cc - c0;
-                    if (lane == 31) {
-                        fold.peak[c] = mm;
-                        fold.ctot[c] = cc;
+                    if (lane == 0) {
                         fold.basel[c] = g.base_cost + b;
                         fold.nev[c] = (status[c] || !valid[c]) ? 0 : nn;
                     }
@@ -605,12 +609,13 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         if (anyev) {
             bar_sync(kBarMain, TM);
-            for (int32_t r = tid; r < R; r += TM) {
+            for (int q = tid; q < P * R; q += TM) {
+                const int c0 = q / R, r = q - c0 * R;
                 const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
                 const unsigned long long rr = (unsigned long long)r;
 #pragma unroll
                 for (int c = 0; c < P; c++) {
-                    if (nevt[c] == 0 || dec_s[c * R + r] != 2) continue;
+                    if (c != c0 || nevt[c] == 0 || dec_s[c * R + r] != 2) continue;
                     const int b0 = atomicAdd(&h.cnt[c], 3 + (u1 - u0));
                     unsigned long long* kin = h.key[c];
                     const unsigned long long pt = (unsigned long long)pos[__ldg(g.elig + r) * P + c] - 1;
@@ -642,7 +647,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 for (int j = 0; j < ne; j++) rank += (kin[j] < key);
                 const int32_t stp = (int32_t)(key >> 32);
                 const int32_t th = stp >> lgL;
-                double cb = fold.woff[c][th >> 5] + cofs[th * P + c];
+                double cb = fold.woff[c * WT + (th >> 5)] + cofs[c * TPC + th];
                 const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT;
                 for (int32_t i = th * L; i < stp; i++) {
                     const int32_t v = __ldg(Pp + i);

@@ -328,7 +328,12 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
             SuperGraphHost sg{n, R, NT, cons_ptr.data(), cons_ent.data(), in_ptr.data(), in_ent.data(),
                               size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data()};
             const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
+            // pick the packing with the most candidates in flight per SM
+            // (P x resident CTAs; ties go to more CTAs, which hide barriers)
             const int cands[3] = {4, 2, 1};
+            int bestP = 0, bestOcc = 0;
+            Plan2 bestPl{};
+            std::vector<char> bestImg;
             for (int ci = 0; ci < 3; ci++) {
                 const int P = cands[ci];
                 if (pforce && std::atoi(pforce) != P) continue;
@@ -337,25 +342,34 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
                 if (!plan2_build(sg, P, cap, &pl, &img)) continue;
                 int occ = 0;
                 if (eval2_occupancy(pl, &occ) != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
+                if (P * occ > bestP * bestOcc || (P * occ == bestP * bestOcc && occ > bestOcc)) {
+                    bestP = P;
+                    bestOcc = occ;
+                    bestPl = pl;
+                    bestImg.swap(img);
+                }
+            }
+            if (bestP > 0) {
                 void* b2 = nullptr;
                 void* ov = nullptr;
-                const int grid = prop.multiProcessorCount * occ;
-                if (cudaMalloc(&b2, img.size()) != cudaSuccess) { cudaGetLastError(); break; }
-                if (cudaMemcpy(b2, img.data(), img.size(), cudaMemcpyHostToDevice) != cudaSuccess ||
-                    cudaMalloc(&ov, (size_t)grid * 8 * pl.ovf_stride) != cudaSuccess) {
+                const int grid = prop.multiProcessorCount * bestOcc;
+                bool ok = cudaMalloc(&b2, bestImg.size()) == cudaSuccess;
+                ok = ok && cudaMemcpy(b2, bestImg.data(), bestImg.size(), cudaMemcpyHostToDevice) == cudaSuccess;
+                ok = ok && cudaMalloc(&ov, (size_t)grid * 8 * bestPl.ovf_stride) == cudaSuccess;
+                if (ok) {
+                    g->plan2 = bestPl;
+                    g->blob2 = b2;
+                    g->blob2_bytes = bestImg.size();
+                    g->ovf2 = ov;
+                    g->cfg.variant = 2;
+                    g->cfg.grid = grid;
+                    g->cfg.block = kMainThreads2 + 32;
+                    g->cfg.smem = bestPl.smem_total;
+                } else {
                     cudaGetLastError();
-                    cudaFree(b2);
-                    break;
+                    if (b2) cudaFree(b2);
+                    if (ov) cudaFree(ov);
                 }
-                g->plan2 = pl;
-                g->blob2 = b2;
-                g->blob2_bytes = img.size();
-                g->ovf2 = ov;
-                g->cfg.variant = 2;
-                g->cfg.grid = grid;
-                g->cfg.block = kMainThreads2 + 32;
-                g->cfg.smem = pl.smem_total;
-                break;
             }
         }
     }

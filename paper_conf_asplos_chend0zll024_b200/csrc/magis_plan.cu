@@ -35,14 +35,14 @@ size_t a16(size_t x) { return (x + 15) / 16 * 16; }
 struct Rows {
     std::vector<uint32_t> row;   // (offset, degree) pairs
     std::vector<uint32_t> hdr;   // [nrows * 32]
-    std::vector<uint32_t> ent;   // edge entries, lane-major per row
+    std::vector<uint16_t> ent;   // edge entries (node ids), lane-major per row
     std::vector<int32_t> node;   // [nrows * 32] node id or -1
     std::vector<uint32_t> wtab;  // per warp [begin, end) rows
 };
 
 // Group nodes into rows of 32 by descending degree, deal rows onto warps.
 Rows make_rows(const std::vector<std::vector<uint32_t>>& lists, const std::vector<uint32_t>& hdrs,
-               uint32_t nop_entry, uint32_t nop_hdr, int WM) {
+               uint16_t nop_entry, uint32_t nop_hdr, int WM) {
     const int32_t N = (int32_t)lists.size();
     std::vector<int32_t> order(N);
     std::iota(order.begin(), order.end(), 0);
@@ -82,7 +82,8 @@ Rows make_rows(const std::vector<std::vector<uint32_t>>& lists, const std::vecto
                     const int32_t v = order[i];
                     out.hdr.push_back(hdrs[v]);
                     out.node.push_back(v);
-                    for (size_t j = 0; j < lists[v].size(); j++) out.ent[off + j * 32 + l] = lists[v][j];
+                    for (size_t j = 0; j < lists[v].size(); j++)
+                        out.ent[off + j * 32 + l] = (uint16_t)(lists[v][j] & 0xffffu);
                 } else {
                     out.hdr.push_back(nop_hdr);
                     out.node.push_back(-1);
@@ -135,7 +136,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     }
     const int WM = kMainThreads2 / 32;
     const uint32_t dummy = (uint32_t)(NTX - 1);
-    const uint32_t nop = (kEdge << kKindShift) | dummy;
+    const uint16_t nop = (uint16_t)dummy;
     const uint32_t nophdr = (kNop << kKindShift) | dummy;
     Rows cr = make_rows(cons, hdrs, nop, nophdr, WM);
     Rows fr = make_rows(ins, hdrs, nop, nophdr, WM);
@@ -161,7 +162,8 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     p.R = R;
     p.nU = nU;
     {
-        int32_t Lmin = std::max(4, (NT + kMainThreads2 - 1) / kMainThreads2), lg = 0;
+        const int32_t tpc = kMainThreads2 / P;          // threads per candidate in the scan
+        int32_t Lmin = std::max(4, (NT + tpc - 1) / tpc), lg = 0;
         while ((1 << lg) < Lmin) lg++;
         p.lgL = lg;
         p.L = 1 << lg;
@@ -173,10 +175,10 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     p.off_wtab = (uint32_t)o;  o = a16(o + wtab.size() * 4);
     p.off_crow = (uint32_t)o;  o = a16(o + cr.row.size() * 4);
     p.off_chdr = (uint32_t)o;  o = a16(o + cr.hdr.size() * 4);
-    p.off_cent = (uint32_t)o;  o = a16(o + cr.ent.size() * 4);
+    p.off_cent = (uint32_t)o;  o = a16(o + cr.ent.size() * 2);
     p.off_frow = (uint32_t)o;  o = a16(o + fr.row.size() * 4);
     p.off_fhdr = (uint32_t)o;  o = a16(o + fr.hdr.size() * 4);
-    p.off_fent = (uint32_t)o;  o = a16(o + fr.ent.size() * 4);
+    p.off_fent = (uint32_t)o;  o = a16(o + fr.ent.size() * 2);
     p.off_size = (uint32_t)o;  o = a16(o + size_u.size() * 4);
     p.off_cost = (uint32_t)o;  o = a16(o + cost_u.size() * 8);
     p.static_bytes = (uint32_t)o;
@@ -185,7 +187,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     p.off_last = (uint32_t)o; o = a16(o + (size_t)NTX * P * 2);
     p.off_af = (uint32_t)o;   o = a16(o + (size_t)P * Sl * 4);
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
-    p.off_cofs = (uint32_t)o; o = a16(o + (size_t)kMainThreads2 * P * 8);
+    p.off_cofs = (uint32_t)o; o = a16(o + (size_t)kMainThreads2 * 8);
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
     p.off_ev = (uint32_t)o;
     int cap = std::min(p.max_events, 64);
@@ -205,10 +207,10 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     put(p.off_wtab, wtab.data(), wtab.size() * 4);
     put(p.off_crow, cr.row.data(), cr.row.size() * 4);
     put(p.off_chdr, cr.hdr.data(), cr.hdr.size() * 4);
-    put(p.off_cent, cr.ent.data(), cr.ent.size() * 4);
+    put(p.off_cent, cr.ent.data(), cr.ent.size() * 2);
     put(p.off_frow, fr.row.data(), fr.row.size() * 4);
     put(p.off_fhdr, fr.hdr.data(), fr.hdr.size() * 4);
-    put(p.off_fent, fr.ent.data(), fr.ent.size() * 4);
+    put(p.off_fent, fr.ent.data(), fr.ent.size() * 2);
     put(p.off_size, size_u.data(), size_u.size() * 4);
     put(p.off_cost, cost_u.data(), cost_u.size() * 8);
     return true;
