@@ -25,6 +25,8 @@
 //    to the next group while it runs.
 #include <climits>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 
 #include "magis_internal.h"
 
@@ -694,6 +696,14 @@ cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
     const void* fn = kernel_for(pl);
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_total);
     if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
+    if (e != cudaSuccess) return e;
+    if (std::getenv("MAGIS_DEBUG")) {
+        cudaFuncAttributes fa;
+        cudaFuncGetAttributes(&fa, fn);
+        std::fprintf(stderr, "[magis] eval2 P=%d regs=%d static_smem=%zu local=%zu\n", pl.P, fa.numRegs,
+                     fa.sharedSizeBytes, fa.localSizeBytes);
+    }
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, TM + 32, pl.smem_total);
 }
 

@@ -9,6 +9,7 @@
 // activation gate so that one static CSR serves every decision vector.
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <numeric>
@@ -326,7 +327,7 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
         cudaDeviceProp prop;
         if (allow2 && cudaGetDeviceProperties(&prop, device) == cudaSuccess) {
             SuperGraphHost sg{n, R, NT, cons_ptr.data(), cons_ent.data(), in_ptr.data(), in_ent.data(),
-                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data()};
+                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data(), r_of.data()};
             const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
             // pick the packing with the most candidates in flight per SM
             // (P x resident CTAs; ties go to more CTAs, which hide barriers)
@@ -341,7 +342,11 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
                 std::vector<char> img;
                 if (!plan2_build(sg, P, cap, &pl, &img)) continue;
                 int occ = 0;
-                if (eval2_occupancy(pl, &occ) != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
+                cudaError_t oe = eval2_occupancy(pl, &occ);
+                if (std::getenv("MAGIS_DEBUG"))
+                    std::fprintf(stderr, "[magis] plan P=%d L=%d S=%d smem=%u static=%u occ=%d err=%d\n", P, pl.L,
+                                 pl.S, pl.smem_total, pl.static_bytes, occ, (int)oe);
+                if (oe != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
                 if (P * occ > bestP * bestOcc || (P * occ == bestP * bestOcc && occ > bestOcc)) {
                     bestP = P;
                     bestOcc = occ;
