@@ -327,7 +327,7 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
         cudaDeviceProp prop;
         if (allow2 && cudaGetDeviceProperties(&prop, device) == cudaSuccess) {
             SuperGraphHost sg{n, R, NT, cons_ptr.data(), cons_ent.data(), in_ptr.data(), in_ent.data(),
-                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data(), r_of.data()};
+                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data()};
             const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
             // pick the packing with the most candidates in flight per SM
             // (P x resident CTAs; ties go to more CTAs, which hide barriers)
