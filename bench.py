@@ -84,39 +84,57 @@ REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_c
 
 
 class ClockSampler:
+    """SM clocks and throttle reasons sampled through NVML every ~2 ms while
+    the timed region runs (nvidia-smi's >= 100 ms period is longer than a
+    short timed region)."""
+
     def __init__(self, index: int):
         self.index = index
         self.rows = []
-        self.proc = None
+        self.stop = threading.Event()
+        self.h = None
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active",
-                 "--format=csv,noheader,nounits", "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL,
-                text=True)
-            self.thr = threading.Thread(target=self._read, daemon=True)
+            import pynvml
+            pynvml.nvmlInit()
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            idx = int(vis.split(",")[self.index]) if vis and vis.split(",")[0].isdigit() else self.index
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self.nv = pynvml
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self._sample()
+            self.thr = threading.Thread(target=self._run, daemon=True)
             self.thr.start()
         except Exception:
-            self.proc = None
+            self.h = None
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            parts = [p.strip() for p in line.split(",")]
-            if len(parts) >= 3:
-                try:
-                    self.rows.append((float(parts[0]), float(parts[1]), int(parts[2], 16)))
-                except ValueError:
-                    pass
+    def _sample(self):
+        nv = self.nv
+        sm = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+        try:
+            rs = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        except Exception:
+            rs = nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+        self.rows.append((float(sm), float(self.max_mhz), int(rs)))
+
+    def _run(self):
+        while not self.stop.is_set():
+            try:
+                self._sample()
+            except Exception:
+                return
+            time.sleep(0.002)
 
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
+        self.stop.set()
+        if self.h is not None:
+            self.thr.join(1.0)
             try:
-                self.proc.wait(2)
+                self._sample()
             except Exception:
-                self.proc.kill()
+                pass
 
     def summary(self):
         if not self.rows:
@@ -127,7 +145,8 @@ class ClockSampler:
         for r in self.rows:
             mask |= r[2]
         reasons = [name for bit, name in REASONS.items() if mask & bit and name != "gpu_idle"]
-        return {"sm_mhz": sm, "sm_max_mhz": mx, "reasons": reasons, "samples": len(self.rows)}
+        return {"sm_mhz": sm, "sm_max_mhz": mx, "reasons": reasons, "samples": len(self.rows),
+                "source": "NVML during the timed region"}
 
 
 def peaks():
@@ -232,7 +251,8 @@ def main():
     torch.cuda.synchronize()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
+    clk = ClockSampler(local)
+    with clk:
         start.record(stream)
         for i in range(args.steps):
             fr = step(evs[i])
@@ -259,7 +279,8 @@ def main():
     tr = ncu_traffic(cfg)
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak_gbs, "unit": "GB/s",
             "frac": round(achieved / peak_gbs, 4), "traffic": tr, "peak_source": peak_src,
-            "kernel": "magis::eval_kernel", "alg_bytes_per_launch": alg_bytes,
+            "kernel": {0: "magis::eval_kernel<smem>", 1: "magis::eval_kernel<global>", 2: "magis::eval2_kernel"}[g.info["variant"]],
+            "alg_bytes_per_launch": alg_bytes,
             "bytes_per_candidate": bytes_per_cand, "kernel_ms_avg": round(kern_avg, 4),
             "kernel_share_of_step": round(kern_avg / ms_per_step, 4)}
 
