@@ -301,25 +301,24 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     for (int gi = 0; gi < ncta; gi++) {
         const int64_t grp = blockIdx.x + (int64_t)gi * gridDim.x;
         const int slot = gi & 1;
-        bool valid[P];
-#pragma unroll
-        for (int c = 0; c < P; c++) valid[c] = grp * P + c < K;
+        // candidate c of this group exists iff bit c of vmask is set
+        const int64_t kleft = K - grp * P;
+        const uint32_t vmask = kleft >= P ? ((1u << P) - 1u) : ((1u << (uint32_t)kleft) - 1u);
         // ---- phase 0: decisions ---------------------------------------------
         {
-            int sw = 0, bad[P];
-#pragma unroll
-            for (int c = 0; c < P; c++) bad[c] = 0;
+            int sw = 0;
+            uint32_t badm = 0;
             for (int i = tid; i < P * R; i += TM) {
                 const int c = i / R, r = i - c * R;
-                const uint8_t d = valid[c] ? dec[(grp * P + c) * (int64_t)R + r] : 0;
+                const uint8_t d = ((vmask >> c) & 1u) ? dec[(grp * P + c) * (int64_t)R + r] : 0;
                 dec_s[i] = d;
                 sw |= (d == 2);
-                if ((d > 2) | ((d == 1) & !(__ldg(g.rflag + r) & kRHasInput))) bad[c] = 1;
+                if ((d > 2) | ((d == 1) & !(__ldg(g.rflag + r) & kRHasInput))) badm |= 1u << c;
             }
             if (sw) atomicOr(&ctl.anysw, 1);
 #pragma unroll
             for (int c = 0; c < P; c++)
-                if (bad[c]) atomicOr(&ctl.flags[c], MAGIS_ST_BAD_DEC);
+                if ((badm >> c) & 1u) atomicOr(&ctl.flags[c], MAGIS_ST_BAD_DEC);
         }
         // ---- phase 1: inverse permutation (pos stored +1); this thread's
         //      chunk of its team's candidate stays in registers for the scan
@@ -327,9 +326,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         {
             const int32_t* Pp = perm + (grp * P + cm) * (int64_t)NT + lo;
             int bad = 0;
-            bool vc = false;
-#pragma unroll
-            for (int c = 0; c < P; c++) vc |= (c == cm) && valid[c];
+            const bool vc = (vmask >> cm) & 1u;
 #pragma unroll
             for (int j = 0; j < LMAX; j += 4) {
                 int4 v = make_int4(-1, -1, -1, -1);
@@ -373,7 +370,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
 #pragma unroll
             for (int cc = 0; cc < P; cc++) {
-                if (cc != c || !valid[cc]) continue;
+                if (cc != c || !((vmask >> cc) & 1u)) continue;
                 const uint8_t d = dec_s[cc * R + r];
 #pragma unroll
                 for (int o = 0; o < 3; o++) {
@@ -437,14 +434,16 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             }
         }
         bar_sync(kBarMain, TM);
-        int status[P];
-        bool anyok = false;
+        // per-candidate status, 4 bits each; okm: valid candidates with status 0
+        uint32_t stm = 0, okm = 0;
 #pragma unroll
         for (int c = 0; c < P; c++) {
             const int f = ctl.flags[c];
-            status[c] = valid[c] ? (f ? f : ctl.viol[c]) : 0;
-            anyok |= valid[c] && status[c] == 0;
+            const uint32_t st = ((vmask >> c) & 1u) ? (uint32_t)(f ? f : ctl.viol[c]) : 0u;
+            stm |= st << (4 * c);
+            if (((vmask >> c) & 1u) && st == 0) okm |= 1u << c;
         }
+        const bool anyok = okm != 0;
         if (anyok) {
             // ---- phase 4: frees over the input rows -> per-step slots ------------
             {
@@ -487,7 +486,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 #pragma unroll
                         for (int c = 0; c < P; c++) {
                             const uint32_t pc = PK::get(p, c);
-                            if (pc == 0 || status[c] || !valid[c]) continue;
+                            if (pc == 0 || !((okm >> c) & 1u)) continue;
                             const uint32_t st = pc - 1;
                             Fs[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = fr[c];
                         }
@@ -570,7 +569,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     }
                     if (lane == 0) {
                         fold.basel[c] = g.base_cost + b;
-                        fold.nev[c] = (status[c] || !valid[c]) ? 0 : nn;
+                        fold.nev[c] = ((okm >> c) & 1u) ? nn : 0;
                     }
                 }
             }
@@ -592,8 +591,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         if (tid == 0) {
 #pragma unroll
             for (int c = 0; c < P; c++) {
-                h.k[c] = valid[c] ? grp * P + c : LLONG_MAX;
-                h.status[c] = status[c];
+                h.k[c] = ((vmask >> c) & 1u) ? grp * P + c : LLONG_MAX;
+                h.status[c] = (int)((stm >> (4 * c)) & 15u);
                 h.peak[c] = fold.peak[c];
                 h.ctot[c] = fold.ctot[c];
                 h.basel[c] = fold.basel[c];
