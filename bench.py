@@ -223,6 +223,17 @@ def main():
     g = Graph.from_workload(wl, device=local)
     load_s = time.perf_counter() - t0
     R, NT = g.R, g.n_total
+    # device candidate generator (§8(a) a1), timed separately from evaluation
+    Pg, Dg = g.generate_candidates(rank * K, K, seed=args.seed)          # warm-up / scratch allocation
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    g.generate_candidates(rank * K, K, seed=args.seed, perm=Pg, dec=Dg)
+    e1.record()
+    torch.cuda.synchronize()
+    gen_dev_ms = e0.elapsed_time(e1)
+    gen_match = bool(torch.equal(Pg, P) and (R == 0 or torch.equal(Dg[:, :R], D[:, :R])))
+    del Pg, Dg
     stream = torch.cuda.current_stream()
     st = torch.empty(K, dtype=torch.uint8, device=dev)
     pk = torch.empty(K, dtype=torch.int64, device=dev)
@@ -340,6 +351,9 @@ def main():
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk.summary(),
                 "gpu_launches": gpu_launches,
                 "setup": {"candidate_gen_s": round(gen_s, 3), "graph_load_s": round(load_s, 3),
+                          "device_gen_ms": round(gen_dev_ms, 3),
+                          "device_gen_cand_per_s": round(K / (gen_dev_ms / 1e3), 1),
+                          "device_gen_matches_host": gen_match,
                           "eval_variant": g.info["variant"], "grid": g.info["grid"], "block": g.info["block"],
                           "smem_bytes": g.info["smem_bytes"]}}
         print(json.dumps(line), flush=True)

@@ -167,6 +167,35 @@ int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_t* h_perm,
                               double* h_latency, void* cuda_stream);
 
 /*
+ * Seeded candidate generation on the device.  Candidate k
+ * (global id id0 + i) depends only on (spec->seed, k), so ranks generate
+ * their shards independently.  The recipe stands in for MAGIS's rule
+ * application + re-ordering (§5.2, Alg. 2; DESIGN.md
+ * §5): per eligible tensor a decision (re-mat with probability
+ * p_remat/10000 if the tensor has inputs, else swap with p_swap/10000);
+ * pct_random % random-priority Kahn orders, pct_local % local moves (a window
+ * of <= wmax natural-order steps re-ordered by the same keyed Kahn), the rest
+ * a random order with one random transposition (may be invalid); Stores right
+ * after their producer, Loads / clones 0..slack steps before the
+ * first late user, inactive optional nodes last.
+ * d_perm [K x n_total] int32, d_dec [K x max(R,1)] uint8: device memory, caller-owned.
+ * Asynchronous on the stream.  The first call allocates graph-owned scratch.
+ * Errors: MAGIS_E_INVAL (K < 0, null pointer, bad spec), MAGIS_E_NOMEM / MAGIS_E_CUDA.
+ */
+typedef struct magis_gen_spec {
+    uint64_t seed;
+    int32_t pct_random;   /* % random topological orders                       */
+    int32_t pct_local;    /* % local moves; the rest: one random transposition */
+    int32_t p_remat;      /* per 10000 eligible tensors                         */
+    int32_t p_swap;       /* per 10000 eligible tensors                         */
+    int32_t wmax;         /* max local-move window (>= 2)                       */
+    int32_t slack;        /* Load / clone placement slack in steps (>= 0)       */
+} magis_gen_spec;
+
+int magis_generate_candidates(magis_graph* g, const magis_gen_spec* spec, uint64_t id0, int64_t K,
+                              int32_t* d_perm, uint8_t* d_dec, void* cuda_stream);
+
+/*
  * Pareto front of (peak, latency) over valid points,
  * plus the BetterThan-best point of Alg. 3 in both optimisation
  * modes.  a dominates b iff a.peak <= b.peak, a.lat <= b.lat and

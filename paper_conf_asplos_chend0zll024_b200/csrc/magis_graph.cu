@@ -273,6 +273,10 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     size_t o_xfer = add(xfer.data(), xfer.size() * 8);
     size_t o_tcost = add(tcost.data(), tcost.size() * 8);
     size_t o_rflag = add(rflag.data(), rflag.size());
+    size_t o_sp = add(succ_ptr.data(), succ_ptr.size() * 4);
+    size_t o_s = add(succ.data(), succ.size() * 4);
+    size_t o_pp = add(pred_ptr.data(), pred_ptr.size() * 4);
+    size_t o_p = add(pred.data(), pred.size() * 4);
     g->blob_bytes = off;
     cudaError_t e = cudaMalloc(&g->blob, off);
     if (e != cudaSuccess) {
@@ -311,6 +315,10 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     dg.tcost = (const double*)(b + o_tcost);
     dg.rflag = (const uint8_t*)(b + o_rflag);
     dg.base_cost = base_cost;
+    g->gen.succ_ptr = (const int32_t*)(b + o_sp);
+    g->gen.succ = (const int32_t*)(b + o_s);
+    g->gen.pred_ptr = (const int32_t*)(b + o_pp);
+    g->gen.pred = (const int32_t*)(b + o_p);
 
     e = eval_configure(dg, device, &g->cfg);
     if (e != cudaSuccess) {
@@ -401,6 +409,7 @@ extern "C" int magis_graph_free(magis_graph* g) {
     if (g->gws) cudaFree(g->gws);
     if (g->blob2) cudaFree(g->blob2);
     if (g->ovf2) cudaFree(g->ovf2);
+    if (g->gen_scratch) cudaFree(g->gen_scratch);
     for (int i = 0; i < 2; i++) {
         if (g->stage[i]) cudaFree(g->stage[i]);
         if (g->ev_h2d[i]) cudaEventDestroy(g->ev_h2d[i]);
@@ -511,6 +520,33 @@ extern "C" int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_
         CK(cudaEventRecord(g->ev_done[b], s0));
     }
     CK(cudaStreamSynchronize(s0));
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* spec, uint64_t id0, int64_t K,
+                                         int32_t* d_perm, uint8_t* d_dec, void* cuda_stream) {
+    clear_error();
+    if (!g || !spec) return set_error(MAGIS_E_INVAL, "null argument");
+    if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
+    if (K == 0) return MAGIS_SUCCESS;
+    if (!d_perm || !d_dec) return set_error(MAGIS_E_INVAL, "null device pointer");
+    if (spec->pct_random < 0 || spec->pct_local < 0 || spec->pct_random + spec->pct_local > 100 ||
+        spec->p_remat < 0 || spec->p_swap < 0 || spec->p_remat + spec->p_swap > 10000 || spec->wmax < 2 ||
+        spec->slack < 0)
+        return set_error(MAGIS_E_INVAL, "bad generator spec");
+    DeviceGuard guard(g->device);
+    if (!g->gen_scratch) {
+        const int64_t T = gen_threads(g->device);
+        CK(cudaMalloc(&g->gen_scratch, gen_scratch_bytes(g->dev, T)));
+        g->gen_T = T;
+    }
+    GenSpec sp{spec->seed, spec->pct_random, spec->pct_local, spec->p_remat, spec->p_swap, spec->wmax, spec->slack};
+    cudaError_t e = gen_launch(g->dev, g->gen, sp, id0, K, d_perm, d_dec, g->gen_scratch, g->gen_T,
+                               (cudaStream_t)cuda_stream);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return set_error(MAGIS_E_CUDA, std::string("generator launch: ") + cudaGetErrorString(e));
+    }
     return MAGIS_SUCCESS;
 }
 

@@ -77,6 +77,24 @@ struct Plan2 {
     uint64_t ovf_stride;  // bytes per overflow event region (global)
 };
 
+// Base-graph adjacency for the device candidate generator (magis_gen.cu).
+struct GenTables {
+    const int32_t* succ_ptr;   // [n+1]
+    const int32_t* succ;
+    const int32_t* pred_ptr;   // [n+1]
+    const int32_t* pred;
+};
+
+struct GenSpec {
+    uint64_t seed;
+    int32_t pct_random, pct_local, p_remat, p_swap, wmax, slack;
+};
+
+size_t gen_scratch_bytes(const DevGraph& g, int64_t T);
+int64_t gen_threads(int device);
+cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp, uint64_t id0, int64_t K,
+                       int32_t* perm, uint8_t* dec, void* scratch, int64_t T, cudaStream_t stream);
+
 struct EvalConfig {
     int variant;          // 0: per-candidate state in shared memory, 1: in global workspace,
                           // 2: packed streams (magis_eval2.cu)
@@ -146,6 +164,9 @@ struct magis_graph {
     void* blob2 = nullptr;         // variant 2 static shared-memory image
     size_t blob2_bytes = 0;
     void* ovf2 = nullptr;          // variant 2 event overflow scratch
+    magis::GenTables gen{};        // base-graph adjacency (device)
+    void* gen_scratch = nullptr;   // candidate generator scratch (lazily allocated)
+    int64_t gen_T = 0;
     size_t gws_bytes = 0;
     int64_t n_edges = 0;
     int64_t n_super_edges = 0;

@@ -23,7 +23,7 @@ ST_NOT_PERM, ST_EDGE, ST_BAD_DEC = 1, 2, 4
 # names declared in include/magis.h (checked by tests/test_abi.py)
 EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magis_eval_schedules",
            "magis_eval_schedules_host", "magis_pareto_workspace_size", "magis_pareto_merge",
-           "magis_last_error", "magis_abi_version", "magis_device_supported"]
+           "magis_last_error", "magis_abi_version", "magis_device_supported", "magis_generate_candidates"]
 
 
 class MagisError(RuntimeError):
@@ -39,6 +39,12 @@ class GraphDesc(ctypes.Structure):
                 ("eligible_tensor", ctypes.c_void_p), ("late_user_ptr", ctypes.c_void_p),
                 ("late_user_idx", ctypes.c_void_p), ("swap_bytes_per_s", ctypes.c_double),
                 ("swap_latency_s", ctypes.c_double)]
+
+
+class GenSpec(ctypes.Structure):
+    _fields_ = [("seed", ctypes.c_uint64), ("pct_random", ctypes.c_int32), ("pct_local", ctypes.c_int32),
+                ("p_remat", ctypes.c_int32), ("p_swap", ctypes.c_int32), ("wmax", ctypes.c_int32),
+                ("slack", ctypes.c_int32)]
 
 
 class GraphInfo(ctypes.Structure):
@@ -80,6 +86,8 @@ def lib() -> ctypes.CDLL:
     L.magis_abi_version.restype = ctypes.c_int
     L.magis_device_supported.argtypes = [ctypes.c_int]
     L.magis_device_supported.restype = ctypes.c_int
+    L.magis_generate_candidates.argtypes = [P, ctypes.POINTER(GenSpec), ctypes.c_uint64, i64, P, P, P]
+    L.magis_generate_candidates.restype = ctypes.c_int
     _lib = L
     return L
 
@@ -176,6 +184,20 @@ class Graph:
                                             _tptr(status), _tptr(peak), _tptr(latency),
                                             _stream_ptr(stream)))
         return status, peak, latency
+
+    def generate_candidates(self, id0: int, K: int, seed: int = 1, pct_random: int = 75, pct_local: int = 24,
+                            p_remat: int = 500, p_swap: int = 500, wmax: int = 64, slack: int = 8,
+                            perm=None, dec=None, stream=None):
+        """Device candidate generator (magis_generate_candidates): returns
+        (perm int32 [K, n_total], dec uint8 [K, max(R,1)]) cuda tensors."""
+        import torch
+        dev = torch.device("cuda", self.device)
+        perm = torch.empty((K, self.n_total), dtype=torch.int32, device=dev) if perm is None else perm
+        dec = torch.empty((K, max(self.R, 1)), dtype=torch.uint8, device=dev) if dec is None else dec
+        spec = GenSpec(int(seed), pct_random, pct_local, p_remat, p_swap, wmax, slack)
+        _check(self._L.magis_generate_candidates(self._h, ctypes.byref(spec), int(id0), int(K), _tptr(perm),
+                                                 _tptr(dec), _stream_ptr(stream)))
+        return perm, dec
 
     def eval_schedules_host(self, perm: np.ndarray, dec: Optional[np.ndarray] = None, out=None,
                             stream=None):

@@ -300,3 +300,42 @@ def test_pareto_shard_merge_identical_to_single():
     # and the GPU front equals the oracle's front of the GPU values
     ref = oracle.pareto(pk, lt, st)
     np.testing.assert_array_equal(single[1], ref)
+
+
+# --------------------------------------------------- device generator (a1) --
+
+@pytest.mark.parametrize("cfg", ["c2", "c3", "c5"])
+def test_device_generator_bit_exact(cfg):
+    """magis_generate_candidates == the CPU generator (magis_inputs) byte for
+    byte, on a shard that does not start at id 0."""
+    wl = build_workload(cfg)
+    spec = CandidateSpec(seed=17)
+    Pc, Dc = CandidateGenerator(wl, spec).generate(1000, 700)
+    g = Graph.from_workload(wl)
+    Pg, Dg = g.generate_candidates(1000, 700, seed=17)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(Pg.cpu().numpy(), Pc)
+    np.testing.assert_array_equal(Dg.cpu().numpy(), Dc)
+
+
+def test_device_generator_small_graphs():
+    rng = np.random.default_rng(8)
+    for trial in range(30):
+        n, edges, size, cost, outs, elig, U, dec = random_case(rng)
+        o, g = both(n, edges, size, outs, cost=cost, elig=elig, U=U)
+        from magis_inputs.graph import Workload
+        wl = Workload("rand", np.asarray(size, np.int64), np.asarray(cost), np.zeros(n, np.uint8),
+                      np.asarray([u for u, _ in edges], np.int32), np.asarray([v for _, v in edges], np.int32),
+                      [""] * n, ["op"] * n, np.asarray(elig, np.int32), [list(u) for u in U])
+        for spec in (CandidateSpec(seed=trial, p_remat=3000, p_swap=3000, wmax=4, slack=2),
+                     CandidateSpec(seed=trial + 100, pct_random=0, pct_local=50)):
+            Pc, Dc = CandidateGenerator(wl, spec).generate(5, 64)
+            Pg, Dg = g.generate_candidates(5, 64, seed=spec.seed, pct_random=spec.pct_random,
+                                           pct_local=spec.pct_local, p_remat=spec.p_remat, p_swap=spec.p_swap,
+                                           wmax=spec.wmax, slack=spec.slack)
+            torch.cuda.synchronize()
+            np.testing.assert_array_equal(Pg.cpu().numpy(), Pc)
+            np.testing.assert_array_equal(Dg.cpu().numpy()[:, :len(elig)], Dc[:, :len(elig)])
+            # and the generated candidates evaluate identically on both sides
+            R = len(elig)
+            assert_parity(*gpu_eval(g, Pc, Dc[:, :R] if R else None), *o.eval_batch(Pc, Dc[:, :R] if R else None))
