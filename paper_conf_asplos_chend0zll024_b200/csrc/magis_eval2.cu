@@ -205,6 +205,14 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int32_t NT = pl.NT, R = pl.R, n = pl.n;
+    // optional phase profile (MAGIS_PROFILE=1): cycles between marks, thread 0
+    // of the main warps and lane 0 of the latency warp, summed over CTAs
+    const bool prof = pl.prof && (tid == 0 || tid == TM);
+    unsigned long long pt[16];
+#pragma unroll
+    for (int i = 0; i < 16; i++) pt[i] = 0;
+    long long plast = clock64();
+#define PROF_MARK(k) do { if (prof) { const long long _t = clock64(); pt[k] += _t - plast; plast = _t; } } while (0)
     const int32_t L = pl.L, S = pl.S, Sl = pl.L * pl.S, lgL = pl.lgL;
 
     bulk_stage(sm, blob, pl.static_bytes, &mbar);
@@ -216,10 +224,11 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const uint32_t* fhdr = (const uint32_t*)(sm + pl.off_fhdr);
     const uint16_t* fent = (const uint16_t*)(sm + pl.off_fent);
     const uint32_t* size_s = (const uint32_t*)(sm + pl.off_size);
+    const double2* rtab = (const double2*)(sm + pl.off_rtab);       // [R] (cost(t_r), swap transfer time)
     const double* cost_s = (const double*)(sm + pl.off_cost);
     uint16_t* pos = (uint16_t*)(sm + pl.off_pos);
     uint16_t* last = (uint16_t*)(sm + pl.off_last);
-    uint32_t* Fs = (uint32_t*)(sm + pl.off_af);           // [P][Sl] bytes freed after each step (units)
+    uint2* AF = (uint2*)(sm + pl.off_af);                 // [P][Sl] (alloc, free) size units per step
     uint8_t* dec_s = (uint8_t*)(sm + pl.off_dec);
     double* cofs = (double*)(sm + pl.off_cofs);           // [TM] cost prefix within the warp
     double* endb_all = (double*)(sm + pl.off_end);
@@ -241,7 +250,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         // ================= latency sweep warp (reading P7) ==================
         for (int gi = 0; gi < ncta; gi++) {
             const int slot = gi & 1;
+            PROF_MARK(13);
             bar_sync(kBarFull + slot, TM + 32);
+            PROF_MARK(14);
             const SlotHdr& h = hdr[slot];
             if (lane < P) {
                 const long long k = h.k[lane];
@@ -258,20 +269,22 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         const double* cb = h.cb[lane];
                         double* endb = endb_all + (size_t)lane * 3 * R;
                         double D = 0.0, Td = 0.0, Th = 0.0;
+                        // end of producer / Store / Load of r at endb[3r + 0 / 1 / 2]
                         for (int e = 0; e < ne; e++) {
                             const unsigned long long kk = key[e];
                             const uint32_t type = (uint32_t)(kk >> 24) & 0xff;
                             const int32_t r = (int32_t)(kk & 0xffffff);
                             const double c = cb[e];
+                            const double2 tx = rtab[r];                 // (cost(t_r), transfer time)
                             if (type == kEvStall) {
                                 D = fmax(D, endb[3 * r + 2] - c);
                             } else if (type == kEvProduce) {
-                                endb[3 * r + 0] = c + D + __ldg(g.tcost + r);
+                                endb[3 * r + 0] = c + D + tx.x;
                             } else if (type == kEvStore) {
-                                Td = fmax(Td, endb[3 * r + 0]) + __ldg(g.xfer + r);
+                                Td = fmax(Td, endb[3 * r + 0]) + tx.y;
                                 endb[3 * r + 1] = Td;
                             } else {
-                                Th = fmax(Th, endb[3 * r + 1]) + __ldg(g.xfer + r);
+                                Th = fmax(Th, endb[3 * r + 1]) + tx.y;
                                 endb[3 * r + 2] = Th;
                             }
                         }
@@ -283,11 +296,15 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 }
             }
             __syncwarp();
+            PROF_MARK(15);
             if (gi + 2 < ncta) {
                 __threadfence_block();
                 bar_arrive(kBarEmpty + slot, TM + 32);
             }
         }
+        if (prof)
+#pragma unroll
+            for (int i = 13; i < 16; i++) atomicAdd((unsigned long long*)(ovf + pl.prof_off) + i, pt[i]);
         return;
     }
 
@@ -359,6 +376,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             if (bad) atomicOr(&ctl.flags[cm], MAGIS_ST_NOT_PERM);
         }
         bar_sync(kBarMain, TM);
+        PROF_MARK(1);
         const bool anysw = ctl.anysw != 0;
         // ---- phase 2: optional nodes, virtual late-user slots ------------------
         double bl[P];
@@ -383,7 +401,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     const bool act = (o == 0) ? (d == 1) : (d == 2);
                     if (!act) {
                         const uint32_t st = p - 1;
-                        Fs[cc * Sl + (st & (L - 1)) * S + (st >> lgL)] = 0u;
+                        AF[cc * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
                         pos[id * P + cc] = 0;
                     }
                 }
@@ -396,6 +414,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             }
         }
         bar_sync(kBarMain, TM);
+        PROF_MARK(2);
         // ---- phase 3: validity + last use over the consumer rows -----------------
         {
             int nperm = 0, viol = 0;
@@ -434,6 +453,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             }
         }
         bar_sync(kBarMain, TM);
+        PROF_MARK(3);
         // per-candidate status, 4 bits each; okm: valid candidates with status 0
         uint32_t stm = 0, okm = 0;
 #pragma unroll
@@ -454,19 +474,12 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     const uint32_t kind = h >> kKindShift, id = h & kIdMask;
                     const V p = PK::load(pos, id);
                     const V lv = PK::load(last, id);
+                    const uint32_t A = size_s[id];
                     uint32_t fr[P];
-                    bool selff = false;
 #pragma unroll
                     for (int c = 0; c < P; c++) {
                         const uint32_t pc = PK::get(p, c);
-                        const bool m = pc != 0 && PK::get(lv, c) == pc;    // no reader: freed after own step
-                        selff |= m;
-                        fr[c] = m ? 1u : 0u;
-                    }
-                    if (selff) {
-                        const uint32_t A = size_s[id];
-#pragma unroll
-                        for (int c = 0; c < P; c++) fr[c] *= A;
+                        fr[c] = (pc != 0 && PK::get(lv, c) == pc) ? A : 0u;   // no reader: freed after own step
                     }
                     const uint16_t* ent = fent + rw.x + lane;
 #pragma unroll 4
@@ -488,28 +501,29 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                             const uint32_t pc = PK::get(p, c);
                             if (pc == 0 || !((okm >> c) & 1u)) continue;
                             const uint32_t st = pc - 1;
-                            Fs[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = fr[c];
+                            AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(A, fr[c]);
                         }
                     }
                 }
             }
             bar_sync(kBarMain, TM);
+            PROF_MARK(4);
             // ---- phase 5: scan of the (sum, max-prefix) monoid ------------------
             //      team cm scans candidate cm: alloc = size of the op at each step
             //      (perm chunk in registers), free = Fs slot, compute cost per step
             long long s1 = 0, m1 = kNegInf;
             double cs1 = 0.0;
+            const int32_t nst = ((okm >> cm) & 1u) ? min(L, NT - lo) : 0;   // steps of this chunk
 #pragma unroll
             for (int j = 0; j < LMAX; j++) {
-                if (j < L && lo + j < NT) {
-                    const int32_t v = pr[j];
-                    if ((uint32_t)v < (uint32_t)NT) {                // else: invalid candidate, ignored
-                        const bool act = v < n || pos[v * P + cm] != 0;
-                        const uint32_t A = act ? size_s[v] : 0u;
-                        s1 += A;
-                        m1 = max(m1, s1);
-                        s1 -= Fs[cm * Sl + j * S + tt];
-                        if (anysw && act) cs1 += cost_s[v];
+                if (j < nst) {
+                    const uint2 af = AF[cm * Sl + j * S + tt];     // alloc / free of the step (units)
+                    s1 += af.x;
+                    m1 = max(m1, s1);
+                    s1 -= af.y;
+                    if (anysw) {
+                        const int32_t v = pr[j];
+                        if (v < n || pos[v * P + cm] != 0) cs1 += cost_s[v];
                     }
                 }
             }
@@ -539,6 +553,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 }
             }
             bar_sync(kBarMain, TM);
+            PROF_MARK(5);
             if (warp == 0) {
                 // fold the WT warp aggregates of each team (segments of WT lanes)
                 long long ss = lane < WM ? agg_s[lane] : 0;
@@ -574,6 +589,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 }
             }
             bar_sync(kBarMain, TM);
+            PROF_MARK(6);
         } else if (tid == 0) {
 #pragma unroll
             for (int c = 0; c < P; c++) { fold.peak[c] = 0; fold.ctot[c] = 0.0; fold.basel[c] = 0.0; fold.nev[c] = 0; }
@@ -587,6 +603,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         // ---- phase 6: swap events -> hand-off slot --------------------------------
         if (gi >= 2) bar_sync(kBarEmpty + slot, TM + 32);
+        PROF_MARK(7);
         SlotHdr& h = hdr[slot];
         if (tid == 0) {
 #pragma unroll
@@ -610,6 +627,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         if (anyev) {
             bar_sync(kBarMain, TM);
+            PROF_MARK(8);
             for (int q = tid; q < P * R; q += TM) {
                 const int c0 = q / R, r = q - c0 * R;
                 const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
@@ -632,6 +650,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 }
             }
             bar_sync(kBarMain, TM);
+            PROF_MARK(9);
             // rank sort (unique keys) + compute-cost prefix before each event:
             // cost of the steps of earlier warps' chunks, earlier lanes of the
             // same warp, then the steps of the owning chunk before the event
@@ -649,8 +668,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const int32_t stp = (int32_t)(key >> 32);
                 const int32_t th = stp >> lgL;
                 double cb = fold.woff[c * WT + (th >> 5)] + cofs[c * TPC + th];
-                const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT;
-                for (int32_t i = th * L; i < stp; i++) {
+                const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT + th * L;
+                const int32_t nb = stp - th * L;
+#pragma unroll 4
+                for (int32_t i = 0; i < nb; i++) {
                     const int32_t v = __ldg(Pp + i);
                     if (v < n || pos[v * P + c] != 0) cb += cost_s[v];
                 }
@@ -660,6 +681,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         __threadfence_block();
         bar_arrive(kBarFull + slot, TM + 32);
+        PROF_MARK(10);
         // reset the per-group control words for the next group, then make sure
         // every main thread is done with pos / Fs / ctl before they are reused
         if (tid == 0) {
@@ -668,6 +690,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         // every main thread must be done reading pos (event keys, cost prefix)
         if (anyev) bar_sync(kBarMain, TM);
+        PROF_MARK(11);
         // clear pos so a missing node (duplicate in perm) reads as 0 next group
         {
             const int nb = NT * P * 2;
@@ -676,7 +699,11 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             for (int i = ((nb >> 4) << 3) + tid; i < NT * P; i += TM) pos[i] = 0;
         }
         bar_sync(kBarMain, TM);
+        PROF_MARK(12);
     }
+    if (prof)
+#pragma unroll
+        for (int i = 1; i < 13; i++) atomicAdd((unsigned long long*)(ovf + pl.prof_off) + i, pt[i]);
 }
 
 template <int P>

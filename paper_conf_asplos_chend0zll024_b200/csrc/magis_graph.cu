@@ -72,8 +72,23 @@ size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
 cudaError_t dispatch_eval(const magis_graph* g, int64_t K, const int32_t* perm, const uint8_t* dec,
                           uint8_t* st, int64_t* pk, double* lt, cudaStream_t s) {
-    if (g->cfg.variant == 2)
-        return eval2_launch(g->dev, g->plan2, g->blob2, g->ovf2, g->cfg.grid, K, perm, dec, st, pk, lt, s);
+    if (g->cfg.variant == 2) {
+        cudaError_t e = eval2_launch(g->dev, g->plan2, g->blob2, g->ovf2, g->cfg.grid, K, perm, dec, st, pk, lt, s);
+        if (e == cudaSuccess && g->plan2.prof) {
+            // diagnostics only: per-phase cycles summed over CTAs (thread 0 / latency lane 0)
+            unsigned long long h[16];
+            cudaStreamSynchronize(s);
+            cudaMemcpy(h, (char*)g->ovf2 + g->plan2.prof_off, 128, cudaMemcpyDeviceToHost);
+            cudaMemset((char*)g->ovf2 + g->plan2.prof_off, 0, 128);
+            unsigned long long tot = 0;
+            for (int i = 1; i < 13; i++) tot += h[i];
+            std::fprintf(stderr, "[magis-prof] main:");
+            for (int i = 1; i < 13; i++) std::fprintf(stderr, " p%d=%.1f%%", i, tot ? 100.0 * h[i] / tot : 0.0);
+            std::fprintf(stderr, " | sweep wait=%llu busy=%llu arrive=%llu (main total %llu)\n", h[14], h[15],
+                         h[13], tot);
+        }
+        return e;
+    }
     return eval_launch(g->dev, g->cfg, g->gws, K, perm, dec, st, pk, lt, s);
 }
 
@@ -334,8 +349,10 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
         const bool allow2 = !(force && std::atoi(force) != 2);
         cudaDeviceProp prop;
         if (allow2 && cudaGetDeviceProperties(&prop, device) == cudaSuccess) {
+            std::vector<double> rtab((size_t)2 * R);
+            for (int32_t r = 0; r < R; r++) { rtab[2 * r] = tcost[r]; rtab[2 * r + 1] = xfer[r]; }
             SuperGraphHost sg{n, R, NT, cons_ptr.data(), cons_ent.data(), in_ptr.data(), in_ent.data(),
-                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data()};
+                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data(), rtab.data()};
             const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
             // pick the packing with the most candidates in flight per SM
             // (P x resident CTAs; ties go to more CTAs, which hide barriers)
@@ -368,7 +385,10 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
                 const int grid = prop.multiProcessorCount * bestOcc;
                 bool ok = cudaMalloc(&b2, bestImg.size()) == cudaSuccess;
                 ok = ok && cudaMemcpy(b2, bestImg.data(), bestImg.size(), cudaMemcpyHostToDevice) == cudaSuccess;
-                ok = ok && cudaMalloc(&ov, (size_t)grid * 8 * bestPl.ovf_stride) == cudaSuccess;
+                bestPl.prof = std::getenv("MAGIS_PROFILE") ? 1 : 0;
+                bestPl.prof_off = (uint64_t)grid * 8 * bestPl.ovf_stride;
+                ok = ok && cudaMalloc(&ov, bestPl.prof_off + 256) == cudaSuccess;
+                ok = ok && cudaMemset(ov, 0, bestPl.prof_off + 256) == cudaSuccess;
                 if (ok) {
                     g->plan2 = bestPl;
                     g->blob2 = b2;

@@ -71,10 +71,13 @@ struct Plan2 {
     uint32_t off_crow, off_chdr, off_cent;                  // consumer rows: (offset, degree), headers, edges
     uint32_t off_frow, off_fhdr, off_fent;                  // input rows
     uint32_t off_size;       // [NTX] size units
+    uint32_t off_rtab;       // [R] double2 (cost(t_r), swap transfer time)
     uint32_t off_cost;       // [NTX] compute cost (f64; clone = cost(t_r), Store / Load 0)
     uint32_t off_pos, off_last, off_af, off_dec, off_cofs, off_end, off_ev;   // off_af: free slots
     uint32_t smem_total;
     uint64_t ovf_stride;  // bytes per overflow event region (global)
+    int32_t prof;         // MAGIS_PROFILE: accumulate per-phase cycles
+    uint64_t prof_off;    // byte offset of the 16 u64 phase counters in the overflow buffer
 };
 
 // Base-graph adjacency for the device candidate generator (magis_gen.cu).
@@ -122,6 +125,7 @@ struct SuperGraphHost {
     const uint8_t* nflag;      // [NT]
     const int32_t* U_ptr;      // [R+1]
     const int32_t* U_idx;
+    const double* rtab;        // [R][2] (cost(t_r), swap transfer time)
 };
 
 // Build the variant-2 plan and its static shared-memory image for a given P.

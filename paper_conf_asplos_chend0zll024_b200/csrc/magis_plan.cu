@@ -181,11 +181,12 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     p.off_fent = (uint32_t)o;  o = a16(o + fr.ent.size() * 2);
     p.off_size = (uint32_t)o;  o = a16(o + size_u.size() * 4);
     p.off_cost = (uint32_t)o;  o = a16(o + cost_u.size() * 8);
+    p.off_rtab = (uint32_t)o;  o = a16(o + (size_t)std::max(R, 1) * 16);
     p.static_bytes = (uint32_t)o;
     const size_t Sl = (size_t)p.L * p.S;
     p.off_pos = (uint32_t)o;  o = a16(o + (size_t)NTX * P * 2);
     p.off_last = (uint32_t)o; o = a16(o + (size_t)NTX * P * 2);
-    p.off_af = (uint32_t)o;   o = a16(o + (size_t)P * Sl * 4);
+    p.off_af = (uint32_t)o;   o = a16(o + (size_t)P * Sl * 8);
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
     p.off_cofs = (uint32_t)o; o = a16(o + (size_t)kMainThreads2 * 8);
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
@@ -213,6 +214,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     put(p.off_fent, fr.ent.data(), fr.ent.size() * 2);
     put(p.off_size, size_u.data(), size_u.size() * 4);
     put(p.off_cost, cost_u.data(), cost_u.size() * 8);
+    put(p.off_rtab, sg.rtab, (size_t)R * 16);
     return true;
 }
 
