@@ -184,12 +184,14 @@ struct Fold {
 
 constexpr long long kNegInf = -(1ll << 62);
 
-template <int P, int LMAX>
+// MODE 0: graph tables and step slots in shared memory; 1: tables read from
+// the global image; 2: tables and step slots in global memory (large graphs)
+template <int P, int LMAX, int MODE>
 __global__ void __launch_bounds__(TM + 32, 1)
 eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
              const int32_t* __restrict__ perm, const uint8_t* __restrict__ dec,
              uint8_t* __restrict__ out_status, int64_t* __restrict__ out_peak,
-             double* __restrict__ out_lat, char* __restrict__ ovf) {
+             double* __restrict__ out_lat, char* __restrict__ ovf, char* __restrict__ afg) {
     using PK = Pk<P>;
     using V = typename PK::V;
     extern __shared__ __align__(128) char sm[];
@@ -215,20 +217,24 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 #define PROF_MARK(k) do { if (prof) { const long long _t = clock64(); pt[k] += _t - plast; plast = _t; } } while (0)
     const int32_t L = pl.L, S = pl.S, Sl = pl.L * pl.S, lgL = pl.lgL;
 
-    bulk_stage(sm, blob, pl.static_bytes, &mbar);
-    const uint32_t* wtab = (const uint32_t*)(sm + pl.off_wtab);   // [WM][4]: consumer rows, input rows
-    const uint2* crow = (const uint2*)(sm + pl.off_crow);
-    const uint32_t* chdr = (const uint32_t*)(sm + pl.off_chdr);
-    const uint16_t* cent = (const uint16_t*)(sm + pl.off_cent);
-    const uint2* frow = (const uint2*)(sm + pl.off_frow);
-    const uint32_t* fhdr = (const uint32_t*)(sm + pl.off_fhdr);
-    const uint16_t* fent = (const uint16_t*)(sm + pl.off_fent);
-    const uint32_t* size_s = (const uint32_t*)(sm + pl.off_size);
-    const double2* rtab = (const double2*)(sm + pl.off_rtab);       // [R] (cost(t_r), swap transfer time)
-    const double* cost_s = (const double*)(sm + pl.off_cost);
+    // graph tables: staged into shared memory once per CTA (bulk copy), or
+    // read in place from the global image when they do not fit
+    const char* sb = MODE ? blob : sm;
+    if (MODE == 0) bulk_stage(sm, blob, pl.static_bytes, &mbar);
+    const uint32_t* wtab = (const uint32_t*)(sb + pl.off_wtab);   // [WM][4]: consumer rows, input rows
+    const uint2* crow = (const uint2*)(sb + pl.off_crow);
+    const uint32_t* chdr = (const uint32_t*)(sb + pl.off_chdr);
+    const uint16_t* cent = (const uint16_t*)(sb + pl.off_cent);
+    const uint2* frow = (const uint2*)(sb + pl.off_frow);
+    const uint32_t* fhdr = (const uint32_t*)(sb + pl.off_fhdr);
+    const uint16_t* fent = (const uint16_t*)(sb + pl.off_fent);
+    const uint32_t* size_s = (const uint32_t*)(sb + pl.off_size);
+    const double2* rtab = (const double2*)(sb + pl.off_rtab);       // [R] (cost(t_r), swap transfer time)
+    const double* cost_s = (const double*)(sb + pl.off_cost);
     uint16_t* pos = (uint16_t*)(sm + pl.off_pos);
     uint16_t* last = (uint16_t*)(sm + pl.off_last);
-    uint2* AF = (uint2*)(sm + pl.off_af);                 // [P][Sl] (alloc, free) size units per step
+    uint2* AF = MODE == 2 ? (uint2*)(afg + (size_t)blockIdx.x * pl.af_bytes)   // [P][Sl] (alloc, free)
+                          : (uint2*)(sm + pl.off_af);                           // size units per step
     uint8_t* dec_s = (uint8_t*)(sm + pl.off_dec);
     double* cofs = (double*)(sm + pl.off_cofs);           // [TM] cost prefix within the warp
     double* endb_all = (double*)(sm + pl.off_end);
@@ -339,7 +345,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         // ---- phase 1: inverse permutation (pos stored +1); this thread's
         //      chunk of its team's candidate stays in registers for the scan
-        int32_t pr[LMAX];
+        constexpr int LR = LMAX <= 16 ? LMAX : 1;      // perm chunk kept in registers when short
+        int32_t pr[LR];
         {
             const int32_t* Pp = perm + (grp * P + cm) * (int64_t)NT + lo;
             int bad = 0;
@@ -368,10 +375,12 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         if ((uint32_t)v.w < (uint32_t)NT) pos[v.w * P + cm] = (uint16_t)(i0 + 4); else bad = 1;
                     }
                 }
-                pr[j] = v.x;
-                if (j + 1 < LMAX) pr[j + 1] = v.y;
-                if (j + 2 < LMAX) pr[j + 2] = v.z;
-                if (j + 3 < LMAX) pr[j + 3] = v.w;
+                if (LMAX <= 16) {
+                    pr[j % LR] = v.x;
+                    if (j + 1 < LR) pr[(j + 1) % LR] = v.y;
+                    if (j + 2 < LR) pr[(j + 2) % LR] = v.z;
+                    if (j + 3 < LR) pr[(j + 3) % LR] = v.w;
+                }
             }
             if (bad) atomicOr(&ctl.flags[cm], MAGIS_ST_NOT_PERM);
         }
@@ -522,7 +531,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     m1 = max(m1, s1);
                     s1 -= af.y;
                     if (anysw) {
-                        const int32_t v = pr[j];
+                        const int32_t v = LMAX <= 16 ? pr[j % LR]
+                                                     : __ldg(perm + (grp * P + cm) * (int64_t)NT + lo + j);
                         if (v < n || pos[v * P + cm] != 0) cs1 += cost_s[v];
                     }
                 }
@@ -706,19 +716,32 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         for (int i = 1; i < 13; i++) atomicAdd((unsigned long long*)(ovf + pl.prof_off) + i, pt[i]);
 }
 
-template <int P>
+template <int P, int MODE>
 static const void* kernel_ptr(int lmax) {
-    if (lmax <= 4) return (const void*)eval2_kernel<P, 4>;
-    if (lmax <= 8) return (const void*)eval2_kernel<P, 8>;
-    return (const void*)eval2_kernel<P, 16>;
+    if constexpr (MODE == 0) {
+        if (lmax <= 4) return (const void*)eval2_kernel<P, 4, 0>;
+        if (lmax <= 8) return (const void*)eval2_kernel<P, 8, 0>;
+        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, 0>;
+        return (const void*)eval2_kernel<P, 32, 0>;
+    } else {
+        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, MODE>;
+        if (lmax <= 32) return (const void*)eval2_kernel<P, 32, MODE>;
+        return (const void*)eval2_kernel<P, 64, MODE>;
+    }
+}
+
+template <int MODE>
+static const void* kernel_mode(const Plan2& pl) {
+    return pl.P == 4 ? kernel_ptr<4, MODE>(pl.L) : pl.P == 2 ? kernel_ptr<2, MODE>(pl.L) : kernel_ptr<1, MODE>(pl.L);
 }
 
 static const void* kernel_for(const Plan2& pl) {
-    return pl.P == 4 ? kernel_ptr<4>(pl.L) : pl.P == 2 ? kernel_ptr<2>(pl.L) : kernel_ptr<1>(pl.L);
+    const int mode = pl.gmem_af ? 2 : (pl.gmem_static ? 1 : 0);
+    return mode == 0 ? kernel_mode<0>(pl) : mode == 1 ? kernel_mode<1>(pl) : kernel_mode<2>(pl);
 }
 
 cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
-    if (pl.L > 16) { *blocks = 0; return cudaSuccess; }
+    if (pl.L > 64 || (!pl.gmem_static && pl.L > 32)) { *blocks = 0; return cudaSuccess; }
     const void* fn = kernel_for(pl);
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_total);
     if (e != cudaSuccess) return e;
@@ -733,14 +756,14 @@ cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, TM + 32, pl.smem_total);
 }
 
-cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, int grid,
+cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,
                          int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status,
                          int64_t* peak, double* lat, cudaStream_t stream) {
     if (K <= 0) return cudaSuccess;
     const int64_t ngroups = (K + pl.P - 1) / pl.P;
     const int gr = (int)std::min<int64_t>(grid, ngroups);
     void* args[] = {(void*)&g, (void*)&pl, (void*)&blob, (void*)&K, (void*)&perm, (void*)&dec,
-                    (void*)&status, (void*)&peak, (void*)&lat, (void*)&ovf};
+                    (void*)&status, (void*)&peak, (void*)&lat, (void*)&ovf, (void*)&afg};
     return cudaLaunchKernel(kernel_for(pl), dim3(gr), dim3(TM + 32), args, pl.smem_total, stream);
 }
 

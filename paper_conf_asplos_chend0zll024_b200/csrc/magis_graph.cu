@@ -73,7 +73,8 @@ size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 cudaError_t dispatch_eval(const magis_graph* g, int64_t K, const int32_t* perm, const uint8_t* dec,
                           uint8_t* st, int64_t* pk, double* lt, cudaStream_t s) {
     if (g->cfg.variant == 2) {
-        cudaError_t e = eval2_launch(g->dev, g->plan2, g->blob2, g->ovf2, g->cfg.grid, K, perm, dec, st, pk, lt, s);
+        cudaError_t e = eval2_launch(g->dev, g->plan2, g->blob2, g->ovf2, g->afg2, g->cfg.grid, K, perm, dec, st, pk,
+                                     lt, s);
         if (e == cudaSuccess && g->plan2.prof) {
             // diagnostics only: per-phase cycles summed over CTAs (thread 0 / latency lane 0)
             unsigned long long h[16];
@@ -355,28 +356,33 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
                               size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data(), rtab.data()};
             const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
             // pick the packing with the most candidates in flight per SM
-            // (P x resident CTAs; ties go to more CTAs, which hide barriers)
+            // (P x resident CTAs; ties go to more CTAs, which hide barriers).
+            // Tiers, in order: graph tables and step slots in shared memory;
+            // tables read from global (L2); tables and slots in global.
             const int cands[3] = {4, 2, 1};
             int bestP = 0, bestOcc = 0;
             Plan2 bestPl{};
             std::vector<char> bestImg;
-            for (int ci = 0; ci < 3; ci++) {
-                const int P = cands[ci];
-                if (pforce && std::atoi(pforce) != P) continue;
-                Plan2 pl;
-                std::vector<char> img;
-                if (!plan2_build(sg, P, cap, &pl, &img)) continue;
-                int occ = 0;
-                cudaError_t oe = eval2_occupancy(pl, &occ);
-                if (std::getenv("MAGIS_DEBUG"))
-                    std::fprintf(stderr, "[magis] plan P=%d L=%d S=%d smem=%u static=%u occ=%d err=%d\n", P, pl.L,
-                                 pl.S, pl.smem_total, pl.static_bytes, occ, (int)oe);
-                if (oe != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
-                if (P * occ > bestP * bestOcc || (P * occ == bestP * bestOcc && occ > bestOcc)) {
-                    bestP = P;
-                    bestOcc = occ;
-                    bestPl = pl;
-                    bestImg.swap(img);
+            for (int tier = 0; tier < 3 && bestP == 0; tier++) {
+                const bool gs = tier >= 1, ga = tier >= 2;
+                for (int ci = 0; ci < 3; ci++) {
+                    const int P = cands[ci];
+                    if (pforce && std::atoi(pforce) != P) continue;
+                    Plan2 pl;
+                    std::vector<char> img;
+                    if (!plan2_build(sg, P, gs, ga, cap, &pl, &img)) continue;
+                    int occ = 0;
+                    cudaError_t oe = eval2_occupancy(pl, &occ);
+                    if (std::getenv("MAGIS_DEBUG"))
+                        std::fprintf(stderr, "[magis] plan tier=%d P=%d L=%d S=%d smem=%u static=%u occ=%d err=%d\n",
+                                     tier, P, pl.L, pl.S, pl.smem_total, pl.static_bytes, occ, (int)oe);
+                    if (oe != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
+                    if (P * occ > bestP * bestOcc || (P * occ == bestP * bestOcc && occ > bestOcc)) {
+                        bestP = P;
+                        bestOcc = occ;
+                        bestPl = pl;
+                        bestImg.swap(img);
+                    }
                 }
             }
             if (bestP > 0) {
@@ -389,6 +395,9 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
                 bestPl.prof_off = (uint64_t)grid * 8 * bestPl.ovf_stride;
                 ok = ok && cudaMalloc(&ov, bestPl.prof_off + 256) == cudaSuccess;
                 ok = ok && cudaMemset(ov, 0, bestPl.prof_off + 256) == cudaSuccess;
+                void* ag = nullptr;
+                if (ok && bestPl.gmem_af) ok = cudaMalloc(&ag, (size_t)grid * bestPl.af_bytes) == cudaSuccess;
+                g->afg2 = ag;
                 if (ok) {
                     g->plan2 = bestPl;
                     g->blob2 = b2;
@@ -429,6 +438,7 @@ extern "C" int magis_graph_free(magis_graph* g) {
     if (g->gws) cudaFree(g->gws);
     if (g->blob2) cudaFree(g->blob2);
     if (g->ovf2) cudaFree(g->ovf2);
+    if (g->afg2) cudaFree(g->afg2);
     if (g->gen_scratch) cudaFree(g->gen_scratch);
     for (int i = 0; i < 2; i++) {
         if (g->stage[i]) cudaFree(g->stage[i]);

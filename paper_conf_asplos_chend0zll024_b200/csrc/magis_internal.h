@@ -76,6 +76,10 @@ struct Plan2 {
     uint32_t off_pos, off_last, off_af, off_dec, off_cofs, off_end, off_ev;   // off_af: free slots
     uint32_t smem_total;
     uint64_t ovf_stride;  // bytes per overflow event region (global)
+    int32_t gmem_static;  // graph tables read from the global image instead of shared memory
+    int32_t gmem_af;      // per-step slots in a per-CTA global slice (af_bytes each)
+    uint32_t state_base;  // offset of the per-candidate state in shared memory
+    uint64_t af_bytes;
     int32_t prof;         // MAGIS_PROFILE: accumulate per-phase cycles
     uint64_t prof_off;    // byte offset of the 16 u64 phase counters in the overflow buffer
 };
@@ -131,9 +135,9 @@ struct SuperGraphHost {
 // Build the variant-2 plan and its static shared-memory image for a given P.
 // Returns false if the graph does not fit (ids >= 65535, sizes beyond u32
 // units, or shared memory).
-bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* plan,
+bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af, size_t smem_cap, Plan2* plan,
                  std::vector<char>* image);
-cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, int grid,
+cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,
                          int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status,
                          int64_t* peak, double* lat, cudaStream_t stream);
 cudaError_t eval2_occupancy(const Plan2& pl, int* blocks_per_sm);
@@ -168,6 +172,7 @@ struct magis_graph {
     void* blob2 = nullptr;         // variant 2 static shared-memory image
     size_t blob2_bytes = 0;
     void* ovf2 = nullptr;          // variant 2 event overflow scratch
+    void* afg2 = nullptr;          // variant 2 per-CTA global step slots (gmem_af)
     magis::GenTables gen{};        // base-graph adjacency (device)
     void* gen_scratch = nullptr;   // candidate generator scratch (lazily allocated)
     int64_t gen_T = 0;

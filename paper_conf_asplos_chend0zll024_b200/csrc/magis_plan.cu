@@ -96,7 +96,8 @@ Rows make_rows(const std::vector<std::vector<uint32_t>>& lists, const std::vecto
 }
 }  // namespace
 
-bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, std::vector<char>* img) {
+bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af, size_t smem_cap, Plan2* pl,
+                 std::vector<char>* img) {
     const int32_t NT = sg.NT, n = sg.n, R = sg.R;
     const int32_t nU = R > 0 ? sg.U_ptr[R] : 0;
     const int64_t NTX = (int64_t)NT + nU + 1;
@@ -165,6 +166,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
         const int32_t tpc = kMainThreads2 / P;          // threads per candidate in the scan
         int32_t Lmin = std::max(4, (NT + tpc - 1) / tpc), lg = 0;
         while ((1 << lg) < Lmin) lg++;
+        if (lg > 6) return false;                       // LMAX <= 64 steps per thread
         p.lgL = lg;
         p.L = 1 << lg;
         p.S = (NT + p.L - 1) / p.L;
@@ -183,10 +185,18 @@ bool plan2_build(const SuperGraphHost& sg, int P, size_t smem_cap, Plan2* pl, st
     p.off_cost = (uint32_t)o;  o = a16(o + cost_u.size() * 8);
     p.off_rtab = (uint32_t)o;  o = a16(o + (size_t)std::max(R, 1) * 16);
     p.static_bytes = (uint32_t)o;
+    // graph tables in shared memory (staged) or read from the global image
+    // (L1/L2; the row reads stay coalesced); per-step slots in shared memory or
+    // in a per-CTA global slice
+    p.gmem_static = gmem_static ? 1 : 0;
+    p.gmem_af = gmem_af ? 1 : 0;
     const size_t Sl = (size_t)p.L * p.S;
+    p.af_bytes = (uint64_t)((P * Sl * 8 + 255) / 256 * 256);
+    if (gmem_static) o = 0;
+    p.state_base = (uint32_t)o;
     p.off_pos = (uint32_t)o;  o = a16(o + (size_t)NTX * P * 2);
     p.off_last = (uint32_t)o; o = a16(o + (size_t)NTX * P * 2);
-    p.off_af = (uint32_t)o;   o = a16(o + (size_t)P * Sl * 8);
+    p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * 8));
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
     p.off_cofs = (uint32_t)o; o = a16(o + (size_t)kMainThreads2 * 8);
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
