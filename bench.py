@@ -43,6 +43,8 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU-baseline wall time")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--windows", action="store_true",
+                    help="local-move candidates scored by windowed delta evaluation (NEXT-1); default config c5, K=1M")
     return ap.parse_args()
 
 
@@ -178,6 +180,8 @@ def main():
 
     from magis_inputs import CONFIGS, CandidateGenerator, CandidateSpec, build_workload
     cfg = args.config.lower()
+    if args.windows and "--config" not in " ".join(sys.argv):
+        cfg = "c5"
     K = args.K or CONFIGS[cfg]["K"]
     if cfg == "c5" and not args.K:
         K = 65536          # C5's 1M local moves are evaluated in 16 chunks of 64k; one chunk per step
@@ -199,6 +203,10 @@ def main():
 
     if args.impl == "reference":
         return run_reference(args, wl, K, workload, pool, ncores, rank, world)
+    if args.windows:
+        if pool is not None:
+            pool.close()
+        return run_windows(args, wl, cfg, rank, world, local)
 
     import torch
     import torch.distributed as dist
@@ -356,6 +364,95 @@ def main():
                           "device_gen_matches_host": gen_match,
                           "eval_variant": g.info["variant"], "grid": g.info["grid"], "block": g.info["block"],
                           "smem_bytes": g.info["smem_bytes"]}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_windows(args, wl, cfg, rank, world, local):
+    """Local-move sweep (SURVEY config 5, NEXT-1): a base schedule with swaps,
+    K window candidates (w <= 64) scored by magis_eval_windows; local fronts
+    merged across ranks like the full path."""
+    import torch
+    import torch.distributed as dist
+    from magis_inputs import CandidateGenerator, CandidateSpec, WindowGenerator
+    from paper_conf_asplos_chend0zll024_b200 import Base, Graph, pareto_merge
+    from paper_conf_asplos_chend0zll024_b200.distributed import global_front
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    K = args.K or 1 << 20
+    g = Graph.from_workload(wl, device=local)
+    P, D = CandidateGenerator(wl, CandidateSpec(seed=args.seed)).generate(0, 64)
+    Pd, Dd = torch.from_numpy(P).to(dev), torch.from_numpy(D).to(dev)
+    st, pk, lt = g.eval_schedules(Pd, Dd if wl.R else None)
+    st = st.cpu().numpy()
+    ok = np.nonzero((st == 0) & (D[:, :max(wl.R, 1)] == 2).any(axis=1))[0]
+    bi = int(ok[0]) if len(ok) else int(np.argmax(st == 0))
+    base = Base(g, Pd[bi].contiguous(), Dd[bi].contiguous() if wl.R else None)
+    t0 = time.perf_counter()
+    wg = WindowGenerator(wl, P[bi], D[bi], seed=args.seed + 1)
+    ws, wln, wp = wg.generate(rank * K, K)
+    gen_s = time.perf_counter() - t0
+    wsd, wld, wpd = (torch.from_numpy(a).to(dev) for a in (ws, wln, wp))
+    st = torch.empty(K, dtype=torch.uint8, device=dev)
+    pk = torch.empty(K, dtype=torch.int64, device=dev)
+    lt = torch.empty(K, dtype=torch.float64, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step(evp=None):
+        if evp:
+            evp[0].record(stream)
+        base.eval_windows(wsd, wld, wpd, st, pk, lt, stream=stream)
+        if evp:
+            evp[1].record(stream)
+        fr = pareto_merge(pk, lt, st, id_base=rank * K, cap=args.cap, stream=stream)
+        if world > 1:
+            fr = global_front(fr, args.cap)
+        return fr
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clk = ClockSampler(local)
+    with clk:
+        start.record(stream)
+        for i in range(args.steps):
+            fr = step(evs[i])
+        end.record(stream)
+        torch.cuda.synchronize()
+    t = torch.tensor([start.elapsed_time(end), statistics.mean(a.elapsed_time(b) for a, b in evs)],
+                     dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms, kern = t.tolist()
+    ms_per_step = ms / args.steps
+    value = world * K / (ms_per_step / 1e3)
+    bytes_per_cand = 4 + 4 + 4 * wg.wmax + 17
+    achieved = K * bytes_per_cand / (kern / 1e3) / 1e9
+    peak_gbs, peak_src = peaks()
+    if rank == 0:
+        line = {"metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+                "op_steps_per_s": round(value * wl.n_total, 1),
+                "window_steps_per_s": round(world * float(wln.sum()) / (ms_per_step / 1e3), 1),
+                "config": {"workload": f"{cfg} local-move sweep: {K} windows (w <= {wg.wmax}) over one base schedule, "
+                                       "windowed delta evaluation (NEXT-1)", "graph": wl.name, "n_total": wl.n_total,
+                           "K_per_rank": K, "mean_window": round(float(wln.mean()), 2),
+                           "base_peak_latency": list(base.info()[1:]), "parallelism": f"candidate-dp{world}",
+                           "front_n": int(fr["front_n"].item())},
+                "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak_gbs, "unit": "GB/s",
+                             "frac": round(achieved / peak_gbs, 4), "traffic": None, "peak_source": peak_src,
+                             "kernel": "magis::window_kernel", "bytes_per_candidate": bytes_per_cand,
+                             "kernel_ms_avg": round(kern, 4)},
+                "cpu_baseline": None, "e2e": None, "clocks": clk.summary(), "gpu_launches": args.steps * 7,
+                "setup": {"window_gen_s": round(gen_s, 3)}}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

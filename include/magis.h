@@ -196,6 +196,40 @@ int magis_generate_candidates(magis_graph* g, const magis_gen_spec* spec, uint64
                               int32_t* d_perm, uint8_t* d_dec, void* cuda_stream);
 
 /*
+ * Windowed delta evaluation of local moves (the
+ * incremental-scheduling idea of Alg. 2, applied to scoring).
+ * A base schedule (perm + decisions) is evaluated once into a device-resident
+ * profile; a local-move candidate k re-orders the base steps
+ * [wstart[k], wstart[k] + wlen[k]) and keeps the base decisions.  Outside the
+ * window the memory curve cannot change, so each candidate costs
+ * O(window + incident edges + swap events) and the result equals the full
+ * evaluation of the expanded schedule (tested bit-exactly on peak/status,
+ * 1e-9 on latency).
+ *
+ * magis_base_create: d_perm [n_total] / d_dec [R] device memory (may be
+ *   reused by the caller after the call's stream work completes); the base is
+ *   evaluated asynchronously on the stream.  *out is library-owned.
+ * magis_base_info: synchronises and returns the base's status / peak / latency.
+ * magis_eval_windows: d_wstart [K], d_wlen [K] (1..wmax), d_wperm [K x wmax]
+ *   int32 (the window's super-graph node ids in their new order; entry j of
+ *   row k for j < wlen[k]), device memory; wmax <= 64.  Outputs as
+ *   magis_eval_schedules.  A window that is not a permutation of the base
+ *   window's nodes gets MAGIS_ST_NOT_PERM; a violated dependency inside the
+ *   window MAGIS_ST_EDGE; an invalid base passes its status on.
+ *   Asynchronous on the stream.  Errors: MAGIS_E_INVAL, MAGIS_E_UNSUPPORTED
+ *   (wmax > 64), MAGIS_E_NOMEM, MAGIS_E_CUDA.
+ */
+typedef struct magis_base magis_base;   /* opaque, library-owned */
+
+int magis_base_create(magis_graph* g, const int32_t* d_perm, const uint8_t* d_dec, magis_base** out,
+                      void* cuda_stream);
+int magis_base_info(const magis_base* b, int* status, int64_t* peak, double* latency);
+int magis_base_free(magis_base* b);
+int magis_eval_windows(const magis_base* b, int64_t K, const int32_t* d_wstart, const int32_t* d_wlen,
+                       const int32_t* d_wperm, int32_t wmax, uint8_t* d_status, int64_t* d_peak,
+                       double* d_latency, void* cuda_stream);
+
+/*
  * Pareto front of (peak, latency) over valid points,
  * plus the BetterThan-best point of Alg. 3 in both optimisation
  * modes.  a dominates b iff a.peak <= b.peak, a.lat <= b.lat and

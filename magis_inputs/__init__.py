@@ -9,7 +9,7 @@ evaluation arithmetic.
 from __future__ import annotations
 
 from .graph import Workload, Builder
-from .candidates import CandidateGenerator, CandidateSpec
+from .candidates import CandidateGenerator, CandidateSpec, WindowGenerator
 from . import models, ftrans, eligible
 
 # SURVEY §8 config sheet.  R_max per config; n_ftrans where applicable.
@@ -48,5 +48,5 @@ def build_workload(cfg: str, **kw) -> Workload:
     return eligible.select(wl, R_max)
 
 
-__all__ = ["Workload", "Builder", "CandidateGenerator", "CandidateSpec", "CONFIGS",
+__all__ = ["Workload", "Builder", "CandidateGenerator", "CandidateSpec", "WindowGenerator", "CONFIGS",
            "build_workload", "models", "ftrans", "eligible"]

@@ -37,6 +37,8 @@ def _load():
         lib.candgen.argtypes = [i32, i32, P, P, P, P, P, P, P, u64, i32, i32, i32, i32, i32, i32,
                                 u64, i64, P, P, i32]
         lib.candgen.restype = None
+        lib.wingen.argtypes = [i32, i32, P, P, P, P, P, P, P, P, P, P, u64, i32, i32, u64, i64, P, P, P]
+        lib.wingen.restype = None
         _lib = lib
     return _lib
 
@@ -99,3 +101,51 @@ class CandidateGenerator:
                     sp.pct_random, sp.pct_local, sp.p_remat, sp.p_swap, sp.wmax, sp.slack,
                     ctypes.c_uint64(id0), K, p(perms), p(decs), int(nthreads))
         return perms, decs
+
+
+class WindowGenerator:
+    """Local-move candidates over a base schedule (csrc/candgen.c wingen):
+    candidate k re-orders base steps [wstart, wstart + wlen) by the keyed Kahn
+    over the window's dependencies under the base decisions; pct_bad % get the
+    window's two ends swapped (may be invalid)."""
+
+    def __init__(self, wl: Workload, base_perm, base_dec=None, seed: int = 1, wmax: int = 64, pct_bad: int = 1):
+        self.wl = wl
+        self.NT = wl.n_total
+        self.bperm = np.ascontiguousarray(base_perm, np.int32)
+        self.bpos = np.empty(self.NT, np.int32)
+        self.bpos[self.bperm] = np.arange(self.NT, dtype=np.int32)
+        self.bdec = np.ascontiguousarray(base_dec if base_dec is not None else np.zeros(max(wl.R, 1)), np.uint8)
+        self.seed, self.wmax, self.pct_bad = seed, wmax, pct_bad
+        _, _, self.pred_ptr, self.pred_idx = csr(wl.n, wl.src, wl.dst)
+        self.U_ptr, self.U_idx = wl.U_arrays()
+        lu = [[] for _ in range(wl.n)]
+        for r, us in enumerate(wl.U):
+            for b in us:
+                lu[b].append(r)
+        self.lu_ptr = np.zeros(wl.n + 1, np.int64)
+        for v in range(wl.n):
+            self.lu_ptr[v + 1] = self.lu_ptr[v] + len(lu[v])
+        self.lu_idx = np.ascontiguousarray(np.concatenate([np.asarray(x, np.int32) for x in lu])
+                                           if self.lu_ptr[-1] else np.zeros(0, np.int32), np.int32)
+        self.elig = np.ascontiguousarray(wl.elig, np.int32)
+
+    def generate(self, id0: int, K: int):
+        lib = _load()
+        ws = np.empty(K, np.int32)
+        wln = np.empty(K, np.int32)
+        wp = np.empty((K, self.wmax), np.int32)
+        p = lambda a: a.ctypes.data_as(ctypes.c_void_p)
+        lib.wingen(self.wl.n, self.wl.R, p(self.pred_ptr), p(self.pred_idx), p(self.elig), p(self.U_ptr),
+                   p(self.U_idx), p(self.lu_ptr), p(self.lu_idx), p(self.bperm), p(self.bpos), p(self.bdec),
+                   ctypes.c_uint64(self.seed), self.wmax, self.pct_bad, ctypes.c_uint64(id0), K, p(ws), p(wln), p(wp))
+        return ws, wln, wp
+
+    def expand(self, ws, wln, wp):
+        """Full perms of window candidates (for the oracle)."""
+        K = len(ws)
+        out = np.repeat(self.bperm[None, :], K, axis=0)
+        for k in range(K):
+            b, w = int(ws[k]), int(wln[k])
+            out[k, b:b + w] = wp[k, :w]
+        return out

@@ -270,3 +270,106 @@ void candgen(int32_t n, int32_t R, const int64_t *succ_ptr, const int32_t *succ_
     for (t = 0; t < nthreads; t++) pthread_create(&th[t], NULL, worker, &jobs[t]);
     for (t = 0; t < nthreads; t++) pthread_join(th[t], NULL);
 }
+
+/*
+ * Local-move (window) candidates over a base schedule (INPUT GENERATION):
+ * candidate k re-orders the base steps [b, b+w) and keeps the base
+ * decisions.  w = 2 + rnd(WIN,0) % (wmax-1) (<= NT), b = rnd(WIN,1) % (NT-w+1);
+ * the window's nodes are re-ordered by the keyed Kahn (key = rnd(KEY,node))
+ * over the window's dependencies under the base decisions (Fig. 8 rules: a
+ * late user reads t_r, its clone or its Load by dec[r]; the clone reads
+ * pre(t_r); t_r -> Store -> Load).  With probability pct_bad/100 the two
+ * ends of the window are swapped afterwards (may be invalid).
+ * Outputs: wstart[K], wlen[K], wperm[K x wmax] (unused entries -1).
+ */
+typedef struct {
+    int32_t n, R, NT;
+    const int64_t *pred_ptr;  const int32_t *pred_idx;   /* base graph */
+    const int32_t *elig;      const int64_t *U_ptr; const int32_t *U_idx;
+    const int64_t *lu_ptr;    const int32_t *lu_idx;     /* per original node: r with node in U_r */
+    const int32_t *bperm, *bpos; const uint8_t *bdec;
+    uint64_t seed; int32_t wmax, pct_bad;
+} win_cfg;
+
+static int in_win(const win_cfg *c, int32_t v, int32_t b, int32_t w)
+{
+    int32_t p = c->bpos[v];
+    return p >= b && p < b + w;
+}
+
+static void win_one(const win_cfg *c, uint64_t k, int32_t *ws, int32_t *wl, int32_t *wp)
+{
+    const int32_t n = c->n, NT = c->NT;
+    int32_t w = 2 + (int32_t)(rnd(c->seed, k, S_WIN, 0) % (uint64_t)(c->wmax - 1));
+    int32_t b, i, j, m = 0;
+    uint64_t pre[64], done = 0;
+    int64_t e, f;
+    if (w > NT) w = NT;
+    b = (int32_t)(rnd(c->seed, k, S_WIN, 1) % (uint64_t)(NT - w + 1));
+    for (i = 0; i < w; i++) {
+        int32_t v = c->bperm[b + i];
+        uint64_t msk = 0;
+        if (v < n) {
+            for (e = c->pred_ptr[v]; e < c->pred_ptr[v + 1]; e++) {
+                int32_t u = c->pred_idx[e], moved = 0;
+                for (f = c->lu_ptr[v]; f < c->lu_ptr[v + 1]; f++) {
+                    int32_t r = c->lu_idx[f];
+                    if (c->elig[r] == u && c->bdec[r] != 0) moved = 1;
+                }
+                if (!moved && in_win(c, u, b, w)) msk |= 1ull << (c->bpos[u] - b);
+            }
+            for (f = c->lu_ptr[v]; f < c->lu_ptr[v + 1]; f++) {
+                int32_t r = c->lu_idx[f], src = -1;
+                if (c->bdec[r] == 1) src = n + 3 * r;
+                if (c->bdec[r] == 2) src = n + 3 * r + 2;
+                if (src >= 0 && in_win(c, src, b, w)) msk |= 1ull << (c->bpos[src] - b);
+            }
+        } else {
+            int32_t r = (v - n) / 3, kd = (v - n) % 3, t = c->elig[r];
+            if (kd == 0 && c->bdec[r] == 1) {
+                for (e = c->pred_ptr[t]; e < c->pred_ptr[t + 1]; e++)
+                    if (in_win(c, c->pred_idx[e], b, w)) msk |= 1ull << (c->bpos[c->pred_idx[e]] - b);
+            } else if (kd == 1 && c->bdec[r] == 2) {
+                if (in_win(c, t, b, w)) msk |= 1ull << (c->bpos[t] - b);
+            } else if (kd == 2 && c->bdec[r] == 2) {
+                if (in_win(c, n + 3 * r + 1, b, w)) msk |= 1ull << (c->bpos[n + 3 * r + 1] - b);
+            }
+        }
+        pre[i] = msk;
+    }
+    /* keyed Kahn over the window: repeatedly take the ready slot with the smallest key */
+    for (m = 0; m < w; m++) {
+        int32_t best = -1;
+        uint64_t bk = 0;
+        for (i = 0; i < w; i++) {
+            uint64_t key;
+            if ((done >> i) & 1ull) continue;
+            if ((pre[i] & ~done) != 0) continue;
+            key = ((rnd(c->seed, k, S_KEY, (uint64_t)c->bperm[b + i]) >> 32) << 32) | (uint32_t)c->bperm[b + i];
+            if (best < 0 || key < bk) { best = i; bk = key; }
+        }
+        done |= 1ull << best;
+        wp[m] = c->bperm[b + best];
+    }
+    if ((int32_t)(rnd(c->seed, k, S_TRN, 0) % 100u) < c->pct_bad) {
+        int32_t t = wp[0]; wp[0] = wp[w - 1]; wp[w - 1] = t;
+    }
+    for (j = w; j < c->wmax; j++) wp[j] = -1;
+    *ws = b;
+    *wl = w;
+}
+
+void wingen(int32_t n, int32_t R, const int64_t *pred_ptr, const int32_t *pred_idx, const int32_t *elig,
+            const int64_t *U_ptr, const int32_t *U_idx, const int64_t *lu_ptr, const int32_t *lu_idx,
+            const int32_t *bperm, const int32_t *bpos, const uint8_t *bdec, uint64_t seed, int32_t wmax,
+            int32_t pct_bad, uint64_t id0, int64_t K, int32_t *wstart, int32_t *wlen, int32_t *wperm)
+{
+    win_cfg c;
+    int64_t k;
+    c.n = n; c.R = R; c.NT = n + 3 * R;
+    c.pred_ptr = pred_ptr; c.pred_idx = pred_idx; c.elig = elig; c.U_ptr = U_ptr; c.U_idx = U_idx;
+    c.lu_ptr = lu_ptr; c.lu_idx = lu_idx; c.bperm = bperm; c.bpos = bpos; c.bdec = bdec;
+    c.seed = seed; c.wmax = wmax < 2 ? 2 : (wmax > 64 ? 64 : wmax); c.pct_bad = pct_bad;
+    for (k = 0; k < K; k++)
+        win_one(&c, id0 + (uint64_t)k, wstart + k, wlen + k, wperm + k * (int64_t)c.wmax);
+}

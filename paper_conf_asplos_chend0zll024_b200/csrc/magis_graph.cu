@@ -580,6 +580,88 @@ extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* s
     return MAGIS_SUCCESS;
 }
 
+// ------------------------------------------------ windowed delta evaluation --
+extern "C" int magis_base_create(magis_graph* g, const int32_t* d_perm, const uint8_t* d_dec, magis_base** out,
+                                 void* cuda_stream) {
+    clear_error();
+    if (!out) return set_error(MAGIS_E_INVAL, "out is NULL");
+    *out = nullptr;
+    if (!g || !d_perm) return set_error(MAGIS_E_INVAL, "null argument");
+    if (g->dev.R > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R > 0");
+    DeviceGuard guard(g->device);
+    magis_base* b = new (std::nothrow) magis_base();
+    if (!b) return set_error(MAGIS_E_NOMEM, "host allocation failed");
+    b->g = g;
+    b->grid = window_grid(g->device);
+    const size_t wsb = (size_t)b->grid * 8 * 3 * std::max(g->dev.R, 1) * sizeof(double);
+    if (cudaMalloc(&b->mem, base_bytes(g->dev)) != cudaSuccess ||
+        cudaMalloc((void**)&b->endb_ws, wsb) != cudaSuccess) {
+        cudaGetLastError();
+        if (b->mem) cudaFree(b->mem);
+        delete b;
+        return set_error(MAGIS_E_NOMEM, "cudaMalloc base failed");
+    }
+    b->dev = base_layout(g->dev, b->mem);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    cudaMemsetAsync(b->dev.endb, 0, (size_t)std::max(g->dev.R, 1) * 24, s);
+    cudaError_t e = base_launch(g->dev, b->dev, d_perm, d_dec ? d_dec : (const uint8_t*)b->dev.dec, s);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(b->mem);
+        cudaFree(b->endb_ws);
+        delete b;
+        return set_error(MAGIS_E_CUDA, std::string("base launch: ") + cudaGetErrorString(e));
+    }
+    *out = b;
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int magis_base_info(const magis_base* b, int* status, int64_t* peak, double* latency) {
+    clear_error();
+    if (!b) return set_error(MAGIS_E_INVAL, "base is NULL");
+    DeviceGuard guard(b->g->device);
+    BaseHdr h;
+    CK(cudaDeviceSynchronize());
+    CK(cudaMemcpy(&h, b->dev.hdr, sizeof(h), cudaMemcpyDeviceToHost));
+    if (status) *status = h.status;
+    if (peak) *peak = h.status ? -1 : h.peak;
+    if (latency) *latency = h.status ? INFINITY : h.latency;
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int magis_base_free(magis_base* b) {
+    clear_error();
+    if (!b) return MAGIS_SUCCESS;
+    DeviceGuard guard(b->g->device);
+    cudaDeviceSynchronize();
+    cudaFree(b->mem);
+    cudaFree(b->endb_ws);
+    cudaGetLastError();
+    delete b;
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int magis_eval_windows(const magis_base* b, int64_t K, const int32_t* d_wstart, const int32_t* d_wlen,
+                                  const int32_t* d_wperm, int32_t wmax, uint8_t* d_status, int64_t* d_peak,
+                                  double* d_latency, void* cuda_stream) {
+    clear_error();
+    if (!b) return set_error(MAGIS_E_INVAL, "base is NULL");
+    if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
+    if (K == 0) return MAGIS_SUCCESS;
+    if (!d_wstart || !d_wlen || !d_wperm || !d_status || !d_peak || !d_latency)
+        return set_error(MAGIS_E_INVAL, "null device pointer");
+    if (wmax < 1) return set_error(MAGIS_E_INVAL, "wmax < 1");
+    if (wmax > window_wmax_supported()) return set_error(MAGIS_E_UNSUPPORTED, "wmax > 64");
+    DeviceGuard guard(b->g->device);
+    cudaError_t e = window_launch(b->g->dev, b->dev, b->grid, b->endb_ws, K, d_wstart, d_wlen, d_wperm, wmax,
+                                  d_status, d_peak, d_latency, (cudaStream_t)cuda_stream);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return set_error(MAGIS_E_CUDA, std::string("window launch: ") + cudaGetErrorString(e));
+    }
+    return MAGIS_SUCCESS;
+}
+
 extern "C" int64_t magis_pareto_workspace_size(int64_t n) {
     return n < 0 ? 0 : pareto_workspace_size(n);
 }

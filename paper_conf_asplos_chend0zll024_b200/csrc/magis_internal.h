@@ -102,6 +102,39 @@ int64_t gen_threads(int device);
 cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp, uint64_t id0, int64_t K,
                        int32_t* perm, uint8_t* dec, void* scratch, int64_t T, cudaStream_t stream);
 
+// Base schedule for windowed delta evaluation (magis_window.cu).
+struct BaseHdr {
+    int status;
+    int nev;
+    long long peak;
+    double latency;
+    double ctot;
+};
+struct BaseDev {
+    BaseHdr* hdr;
+    int32_t* perm;      // [NT] step -> node
+    int32_t* pos;       // [NT] node -> step
+    int32_t* last;      // [NT] last reader step (NT for outputs, own step if none, -1 inactive)
+    uint8_t* active;    // [NT]
+    long long* carry;   // [NT+1] bytes live entering step i (before its allocation)
+    long long* pm;      // [NT+1] max_{j<i} M_j (-1 if none)
+    long long* sm;      // [NT+1] max_{j>=i} M_j (-1 if none)
+    double* cb;         // [NT+1] compute cost before step i
+    long long* mstep;   // [NT] M_i
+    uint8_t* dec;       // [R]
+    double* endb;       // [3R] scratch of the base sweep
+    unsigned long long* evk;   // swap events of the base, step order
+};
+size_t base_bytes(const DevGraph& g);
+BaseDev base_layout(const DevGraph& g, void* mem);
+cudaError_t base_launch(const DevGraph& g, const BaseDev& b, const int32_t* perm, const uint8_t* dec,
+                        cudaStream_t s);
+int window_grid(int device);
+int window_wmax_supported();
+cudaError_t window_launch(const DevGraph& g, const BaseDev& b, int grid, double* endb_ws, int64_t K,
+                          const int32_t* wstart, const int32_t* wlen, const int32_t* wperm, int32_t wmax,
+                          uint8_t* st, int64_t* pk, double* lt, cudaStream_t s);
+
 struct EvalConfig {
     int variant;          // 0: per-candidate state in shared memory, 1: in global workspace,
                           // 2: packed streams (magis_eval2.cu)
@@ -185,4 +218,12 @@ struct magis_graph {
     void* stage[2] = {nullptr, nullptr};
     cudaEvent_t ev_h2d[2] = {nullptr, nullptr};
     cudaEvent_t ev_done[2] = {nullptr, nullptr};
+};
+
+struct magis_base {
+    const magis_graph* g = nullptr;
+    void* mem = nullptr;
+    magis::BaseDev dev{};
+    double* endb_ws = nullptr;
+    int grid = 0;
 };

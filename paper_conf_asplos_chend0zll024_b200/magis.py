@@ -23,7 +23,8 @@ ST_NOT_PERM, ST_EDGE, ST_BAD_DEC = 1, 2, 4
 # names declared in include/magis.h (checked by tests/test_abi.py)
 EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magis_eval_schedules",
            "magis_eval_schedules_host", "magis_pareto_workspace_size", "magis_pareto_merge",
-           "magis_last_error", "magis_abi_version", "magis_device_supported", "magis_generate_candidates"]
+           "magis_last_error", "magis_abi_version", "magis_device_supported", "magis_generate_candidates",
+           "magis_base_create", "magis_base_info", "magis_base_free", "magis_eval_windows"]
 
 
 class MagisError(RuntimeError):
@@ -88,6 +89,14 @@ def lib() -> ctypes.CDLL:
     L.magis_device_supported.restype = ctypes.c_int
     L.magis_generate_candidates.argtypes = [P, ctypes.POINTER(GenSpec), ctypes.c_uint64, i64, P, P, P]
     L.magis_generate_candidates.restype = ctypes.c_int
+    L.magis_base_create.argtypes = [P, P, P, ctypes.POINTER(P), P]
+    L.magis_base_create.restype = ctypes.c_int
+    L.magis_base_info.argtypes = [P, ctypes.POINTER(ctypes.c_int), ctypes.POINTER(i64), ctypes.POINTER(d)]
+    L.magis_base_info.restype = ctypes.c_int
+    L.magis_base_free.argtypes = [P]
+    L.magis_base_free.restype = ctypes.c_int
+    L.magis_eval_windows.argtypes = [P, i64, P, P, P, i32, P, P, P, P]
+    L.magis_eval_windows.restype = ctypes.c_int
     _lib = L
     return L
 
@@ -221,6 +230,50 @@ class Graph:
         _check(self._L.magis_eval_schedules_host(self._h, K, _np_ptr(p), _np_ptr(dd), _np_ptr(st),
                                                  _np_ptr(pk), _np_ptr(lt), _stream_ptr(stream)))
         return st, pk, lt
+
+
+class Base:
+    """A base schedule evaluated once for windowed delta evaluation
+    (magis_base_create / magis_eval_windows)."""
+
+    def __init__(self, graph: "Graph", perm, dec=None, stream=None):
+        import torch
+        self._L = graph._L
+        self.graph = graph
+        self._keep = (perm, dec)
+        h = ctypes.c_void_p()
+        _check(self._L.magis_base_create(graph._h, _tptr(perm), _tptr(dec) if graph.R else None,
+                                         ctypes.byref(h), _stream_ptr(stream)))
+        self._h = h
+
+    def info(self):
+        st, pk, lt = ctypes.c_int(), ctypes.c_int64(), ctypes.c_double()
+        _check(self._L.magis_base_info(self._h, ctypes.byref(st), ctypes.byref(pk), ctypes.byref(lt)))
+        return st.value, pk.value, lt.value
+
+    def eval_windows(self, wstart, wlen, wperm, status=None, peak=None, latency=None, stream=None):
+        """wstart/wlen int32 [K], wperm int32 [K, wmax] cuda tensors."""
+        import torch
+        K = int(wstart.shape[0])
+        dev = wstart.device
+        status = torch.empty(K, dtype=torch.uint8, device=dev) if status is None else status
+        peak = torch.empty(K, dtype=torch.int64, device=dev) if peak is None else peak
+        latency = torch.empty(K, dtype=torch.float64, device=dev) if latency is None else latency
+        _check(self._L.magis_eval_windows(self._h, K, _tptr(wstart), _tptr(wlen), _tptr(wperm),
+                                          int(wperm.shape[1]), _tptr(status), _tptr(peak), _tptr(latency),
+                                          _stream_ptr(stream)))
+        return status, peak, latency
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._L.magis_base_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 def pareto_workspace_size(n: int) -> int:
