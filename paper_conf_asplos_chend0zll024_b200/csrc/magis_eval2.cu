@@ -19,10 +19,14 @@
 //  * alloc/free amounts land in per-step slots (u32 size units) in a
 //    transposed layout, so the scan's per-thread contiguous chunks read
 //    conflict-free;
-//  * the swap-latency sweep (the three in-order queues of reading P7) runs in
-//    a dedicated warp, one lane per candidate, fed through a double-buffered
-//    shared-memory hand-off guarded by named barriers, so the main warps go on
-//    to the next group while it runs.
+//  * swap latency (the three in-order queues of reading P7): the steps that
+//    raise swap events are marked in a per-candidate bitmap while the gates
+//    are resolved (phase 2); the scan threads emit their marked steps with the
+//    compute-cost prefix in step order (a warp scan of mark counts gives each
+//    thread its slot, so no sort is needed), and one latency warp per
+//    candidate walks them.  The hand-off is double-buffered in shared memory
+//    and guarded by named barriers, so the main warps go on to the next group
+//    while the latency warps run.
 #include <climits>
 #include <cmath>
 #include <cstdio>
@@ -155,55 +159,136 @@ __device__ __forceinline__ void bulk_stage(void* smem_dst, const void* gsrc, uin
 }
 
 // ------------------------------------------------------------ hand-off --
+// Main warps -> latency warp, one slot per group parity.  Per candidate: the
+// steps that raise swap events, in step order, as (step << 32 | node) keys
+// with the compute-cost prefix before the step minus the exclusive prefix of
+// the owning warp (woff, added by the latency warp), plus the decisions.
 struct SlotHdr {
     long long k[4];
     long long peak[4];      // in size units
-    double ctot[4];         // sum of compute costs (from the per-step scan)
-    double basel[4];        // base + clone costs (swap-free latency)
-    unsigned long long* key[4];   // [2 * cap]: unsorted keys, then sorted keys
-    double* cb[4];                // compute-cost prefix before each sorted event
+    double ctot[4];         // sum of compute costs (swapping candidates)
     int status[4];
     int nev[4];
-    int cnt[4];             // gather counters
+    int swp[4];             // candidate swaps some tensor
+    double woff[WM];        // exclusive compute-cost prefix of each warp within its team
 };
 
 struct Ctl {
     int flags[4];           // per-candidate status bits (atomicOr)
     int viol[4];
-    int anysw;
-};
-
-// per-group results of the cross-warp fold (written by warp 0)
-struct Fold {
-    long long peak[4];
-    double ctot[4];
-    double basel[4];
-    int nev[4];
-    double woff[WM];        // exclusive compute-cost prefix of each warp within its team
+    int swm;                // bit c: candidate c swaps some tensor
 };
 
 constexpr long long kNegInf = -(1ll << 62);
 
+// mark bits of steps [lo, lo + L) (L a power of two, lo a multiple of L)
+__device__ __forceinline__ unsigned long long mark_bits(const uint32_t* m, int32_t lo, int32_t L) {
+    if (L >= 64) return (unsigned long long)m[lo >> 5] | ((unsigned long long)m[(lo >> 5) + 1] << 32);
+    const uint32_t w = m[lo >> 5] >> (lo & 31);
+    return L == 32 ? w : (w & ((1u << L) - 1u));
+}
+
+// The three in-order queues of reading P7 over one candidate's event steps
+// (in step order): at a compute op, stalls on the Loads of the swapped
+// tensors it reads, then the end of the op if it produces a swapped tensor;
+// Store / Load ops on the D2H / H2D queues.  endb[3r + 0 / 1 / 2] = end of
+// producer / Store / Load of tensor r.
+struct WalkTabs {
+    const uint2* ninfo;
+    const uint16_t* lul;
+    const double2* rtab;
+    int32_t n, lgL;
+};
+
+// What a compute step of a swapping candidate does on the queues, resolved
+// by the main warp that emits it: bits 0-30 = which of the node's late-user
+// tensors (ninfo list order) are swapped, bit 31 = it produces a swapped
+// tensor, bits 32-47 = that tensor, bits 48-63 = offset of the list in lul.
+__device__ __forceinline__ unsigned long long step_info(int32_t v, int32_t n, const uint8_t* dd, const uint2* ninfo,
+                                                        const uint16_t* lul) {
+    if (v >= n) return 0ull;
+    const uint2 x = ninfo[v];
+    const uint32_t rt = x.x & 0xffffu, cnt = x.x >> 16;
+    uint32_t m = 0;
+    for (uint32_t i = 0; i < cnt; i++) m |= (uint32_t)(dd[lul[x.y + i]] == 2) << i;
+    const bool prod = rt && dd[rt - 1] == 2;
+    return (unsigned long long)m | ((unsigned long long)prod << 31) |
+           ((unsigned long long)(prod ? rt - 1 : 0) << 32) | ((unsigned long long)x.y << 48);
+}
+
+__device__ __forceinline__ void walk_events(const unsigned long long* key, const double* cbp,
+                                            const unsigned long long* info, int ne,
+                                            double* endb, const WalkTabs& t, double& D, double& Td, double& Th) {
+    unsigned long long kn = ne > 0 ? key[0] : 0ull, in_ = ne > 0 ? info[0] : 0ull;
+    double cn = ne > 0 ? cbp[0] : 0.0;
+    for (int e = 0; e < ne; e++) {
+        const unsigned long long kk = kn, inf = in_;
+        const double cp = cn;
+        if (e + 1 < ne) { kn = key[e + 1]; cn = cbp[e + 1]; in_ = info[e + 1]; }   // next event step in flight
+        const int32_t w = (int32_t)(kk & 0xffffffffu);
+        const double cw = cp;                                         // compute-cost prefix before the step
+        if (w < t.n) {
+            uint32_t m = (uint32_t)inf & 0x7fffffffu;
+            const uint32_t off = (uint32_t)(inf >> 48);
+            while (m) {                                               // stalls on the Loads it reads
+                const uint32_t i = __ffs(m) - 1;
+                m &= m - 1;
+                const uint32_t r = t.lul[off + i];
+                D = fmax(D, endb[3 * r + 2] - cw);
+            }
+            if ((inf >> 31) & 1ull) {                                 // producer of a swapped tensor ends
+                const uint32_t r = (uint32_t)(inf >> 32) & 0xffffu;
+                endb[3 * r] = cw + D + t.rtab[r].x;
+            }
+        } else {
+            const uint32_t q = (uint32_t)(w - t.n), r = q / 3, o = q - 3 * r;
+            if (o == 1) { Td = fmax(Td, endb[3 * r]) + t.rtab[r].y; endb[3 * r + 1] = Td; }      // Store
+            else { Th = fmax(Th, endb[3 * r + 1]) + t.rtab[r].y; endb[3 * r + 2] = Th; }       // Load
+        }
+    }
+}
+
+// Latency of one swapping candidate from its event steps (key, cb in step
+// order): the warp resolves every step in parallel (cost prefix completed
+// with its warp offset, swap bits via step_info), then lane 0 walks them.
+__device__ __forceinline__ double candidate_latency(unsigned long long* key, double* cbp, unsigned long long* inf,
+                                                    int ne, const double* woff, const uint8_t* dd, double* endb,
+                                                    const WalkTabs& t, double ctot, int lane) {
+    for (int e = lane; e < ne; e += 32) {
+        const unsigned long long kk = key[e];
+        const int32_t stp = (int32_t)(kk >> 32), w = (int32_t)(kk & 0xffffffffu);
+        cbp[e] += woff[(stp >> t.lgL) >> 5];
+        inf[e] = step_info(w, t.n, dd, t.ninfo, t.lul);
+    }
+    __syncwarp();
+    double lat = 0.0;
+    if (lane == 0) {
+        double D = 0.0, Td = 0.0, Th = 0.0;
+        walk_events(key, cbp, inf, ne, endb, t, D, Td, Th);
+        lat = fmax(fmax(ctot + D, Td), Th);
+    }
+    return lat;
+}
+
 // MODE 0: graph tables and step slots in shared memory; 1: tables read from
 // the global image; 2: tables and step slots in global memory (large graphs)
 template <int P, int LMAX, int MODE>
-__global__ void __launch_bounds__(TM + 32, 1)
+__global__ void __launch_bounds__(TM + 32 * P, 1)
 eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
              const int32_t* __restrict__ perm, const uint8_t* __restrict__ dec,
              uint8_t* __restrict__ out_status, int64_t* __restrict__ out_peak,
              double* __restrict__ out_lat, char* __restrict__ ovf, char* __restrict__ afg) {
     using PK = Pk<P>;
     using V = typename PK::V;
+    constexpr int TL = 32 * P;                 // latency warps: one per candidate of a group
     extern __shared__ __align__(128) char sm[];
     __shared__ uint64_t mbar;
     __shared__ SlotHdr hdr[2];
-    __shared__ Ctl ctl;
-    __shared__ Fold fold;
+    __shared__ Ctl ctl[2];                     // per group parity (reset one group ahead)
     __shared__ long long agg_s[WM];
     __shared__ long long agg_m[WM];
     __shared__ double agg_c[WM];
-    __shared__ double agg_b[WM][P];
-    __shared__ int agg_n[WM][P];
+    __shared__ int wcnt[WM];                   // event steps per warp chunk
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int32_t NT = pl.NT, R = pl.R, n = pl.n;
@@ -231,73 +316,79 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const uint32_t* size_s = (const uint32_t*)(sb + pl.off_size);
     const double2* rtab = (const double2*)(sb + pl.off_rtab);       // [R] (cost(t_r), swap transfer time)
     const double* cost_s = (const double*)(sb + pl.off_cost);
+    const uint2* ninfo = (const uint2*)(sb + pl.off_ninfo);
+    const uint16_t* lul = (const uint16_t*)(sb + pl.off_lul);
     uint16_t* pos = (uint16_t*)(sm + pl.off_pos);
     uint16_t* last = (uint16_t*)(sm + pl.off_last);
     uint2* AF = MODE == 2 ? (uint2*)(afg + (size_t)blockIdx.x * pl.af_bytes)   // [P][Sl] (alloc, free)
                           : (uint2*)(sm + pl.off_af);                           // size units per step
     uint8_t* dec_s = (uint8_t*)(sm + pl.off_dec);
-    double* cofs = (double*)(sm + pl.off_cofs);           // [TM] cost prefix within the warp
-    double* endb_all = (double*)(sm + pl.off_end);
-    unsigned long long* evk_s = (unsigned long long*)(sm + pl.off_ev);               // [2][P][2*cap]
-    double* evcb_s = (double*)(sm + pl.off_ev + (size_t)2 * P * 2 * pl.evcap * 8);  // [2][P][cap]
+    uint32_t* evm = (uint32_t*)(sm + pl.off_evm);          // [P][nwm] event-step marks
+    uint8_t* sdec = (uint8_t*)(sm + pl.off_sdec);          // [2][P][Rw] decisions for the latency warp
+    const int32_t Rw = (R + 15) & ~15;                     // padded row of sdec
+    const int32_t nwm = pl.nwm, cap = pl.evcap;
+    unsigned long long* evk_s = (unsigned long long*)(sm + pl.off_ev);             // [2][P][cap]
+    double* evc_s = (double*)(sm + pl.off_ev + (size_t)2 * P * cap * 8);          // [2][P][cap]
+    unsigned long long* evi_s = (unsigned long long*)(sm + pl.off_ev + (size_t)2 * P * cap * 16);   // [2][P][cap]
 
     // pos / last of the virtual and dummy slots start (and the dummy stays) 0
     for (int i = tid; i < pl.NTX * P; i += blockDim.x) { pos[i] = 0; last[i] = 0; }
+    for (int i = tid; i < P * nwm; i += blockDim.x) evm[i] = 0;
     if (tid == 0) {
-        for (int c = 0; c < 4; c++) { ctl.flags[c] = 0; ctl.viol[c] = 0; }
-        ctl.anysw = 0;
+        for (int b = 0; b < 2; b++) {
+            for (int c = 0; c < 4; c++) ctl[b].flags[c] = ctl[b].viol[c] = 0;
+            ctl[b].swm = 0;
+        }
     }
     __syncthreads();
 
     const int64_t ngroups = (K + P - 1) / P;
     const int ncta = (blockIdx.x < ngroups) ? (int)((ngroups - 1 - blockIdx.x) / gridDim.x + 1) : 0;
+    constexpr int TPC = TM / P, WT = WM / P;
 
-    if (warp == WM) {
-        // ================= latency sweep warp (reading P7) ==================
+    if (warp >= WM) {
+        // ================= latency warps (reading P7) ======================
+        //      warp WM + c walks the event steps of candidate c of each group
+        const int c = warp - WM;
+        double* endb = (double*)(sm + pl.off_end) + (size_t)c * 3 * R;
+        const WalkTabs wt{ninfo, lul, rtab, n, lgL};
         for (int gi = 0; gi < ncta; gi++) {
             const int slot = gi & 1;
             PROF_MARK(13);
-            bar_sync(kBarFull + slot, TM + 32);
+            bar_sync(kBarFull + slot, TM + TL);
             PROF_MARK(14);
             const SlotHdr& h = hdr[slot];
-            if (lane < P) {
-                const long long k = h.k[lane];
-                if (k < K) {
-                    const int st = h.status[lane];
-                    double lat;
-                    if (st) {
-                        lat = __longlong_as_double(0x7ff0000000000000ll);
-                    } else if (h.nev[lane] == 0) {
-                        lat = h.basel[lane];
+            const long long k = h.k[c];
+            if (k < K) {
+                const int st = h.status[c];
+                const uint8_t* dd = sdec + (size_t)(slot * P + c) * Rw;
+                double lat = __longlong_as_double(0x7ff0000000000000ll);
+                if (st) {
+                } else if (!h.swp[c]) {
+                    double bl = 0.0;                 // no swap: base cost + re-computations
+                    for (int r = lane; r < R; r += 32)
+                        if (dd[r] == 1) bl += rtab[r].x;
+#pragma unroll
+                    for (int o = 16; o > 0; o >>= 1) bl += __shfl_xor_sync(0xffffffffu, bl, o);
+                    lat = g.base_cost + bl;
+                } else {
+                    const double* woff = h.woff + c * WT;
+                    const int ne = h.nev[c];
+                    if (ne <= cap) {
+                        const size_t b0 = (size_t)(slot * P + c) * cap;
+                        lat = candidate_latency(evk_s + b0, evc_s + b0, evi_s + b0, ne, woff, dd, endb, wt, h.ctot[c],
+                                                lane);
                     } else {
-                        const int ne = h.nev[lane];
-                        const unsigned long long* key = h.key[lane] + ne;
-                        const double* cb = h.cb[lane];
-                        double* endb = endb_all + (size_t)lane * 3 * R;
-                        double D = 0.0, Td = 0.0, Th = 0.0;
-                        // end of producer / Store / Load of r at endb[3r + 0 / 1 / 2]
-                        for (int e = 0; e < ne; e++) {
-                            const unsigned long long kk = key[e];
-                            const uint32_t type = (uint32_t)(kk >> 24) & 0xff;
-                            const int32_t r = (int32_t)(kk & 0xffffff);
-                            const double c = cb[e];
-                            const double2 tx = rtab[r];                 // (cost(t_r), transfer time)
-                            if (type == kEvStall) {
-                                D = fmax(D, endb[3 * r + 2] - c);
-                            } else if (type == kEvProduce) {
-                                endb[3 * r + 0] = c + D + tx.x;
-                            } else if (type == kEvStore) {
-                                Td = fmax(Td, endb[3 * r + 0]) + tx.y;
-                                endb[3 * r + 1] = Td;
-                            } else {
-                                Th = fmax(Th, endb[3 * r + 1]) + tx.y;
-                                endb[3 * r + 2] = Th;
-                            }
-                        }
-                        lat = fmax(fmax(h.ctot[lane] + D, Td), Th);
+                        char* ob = ovf + ((size_t)blockIdx.x * 8 + slot * 4 + c) * pl.ovf_stride;
+                        const size_t me = (size_t)pl.max_events;
+                        lat = candidate_latency((unsigned long long*)ob, (double*)(ob + me * 8),
+                                                (unsigned long long*)(ob + me * 16), ne, woff, dd, endb, wt, h.ctot[c],
+                                                lane);
                     }
+                }
+                if (lane == 0) {
                     out_status[k] = (uint8_t)st;
-                    out_peak[k] = st ? -1 : h.peak[lane] * pl.unit;
+                    out_peak[k] = st ? -1 : h.peak[c] * pl.unit;
                     out_lat[k] = lat;
                 }
             }
@@ -305,7 +396,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             PROF_MARK(15);
             if (gi + 2 < ncta) {
                 __threadfence_block();
-                bar_arrive(kBarEmpty + slot, TM + 32);
+                bar_arrive(kBarEmpty + slot, TM + TL);
             }
         }
         if (prof)
@@ -317,31 +408,30 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // ========================= main warps =====================================
     // phases 1 and 5: candidate cm of the group is handled by team cm (TPC
     // threads, WT warps); thread tt of the team owns steps [lo, lo + L)
-    constexpr int TPC = TM / P, WT = WM / P;
     const int cm = tid / TPC, tt = tid - cm * TPC;
     const int32_t lo = tt * L;
     const bool vec4 = (NT & 3) == 0;
     for (int gi = 0; gi < ncta; gi++) {
         const int64_t grp = blockIdx.x + (int64_t)gi * gridDim.x;
         const int slot = gi & 1;
+        Ctl& cl = ctl[slot];
         // candidate c of this group exists iff bit c of vmask is set
         const int64_t kleft = K - grp * P;
         const uint32_t vmask = kleft >= P ? ((1u << P) - 1u) : ((1u << (uint32_t)kleft) - 1u);
         // ---- phase 0: decisions ---------------------------------------------
         {
-            int sw = 0;
-            uint32_t badm = 0;
+            uint32_t badm = 0, swm = 0;
             for (int i = tid; i < P * R; i += TM) {
                 const int c = i / R, r = i - c * R;
                 const uint8_t d = ((vmask >> c) & 1u) ? dec[(grp * P + c) * (int64_t)R + r] : 0;
                 dec_s[i] = d;
-                sw |= (d == 2);
+                if (d == 2) swm |= 1u << c;
                 if ((d > 2) | ((d == 1) & !(__ldg(g.rflag + r) & kRHasInput))) badm |= 1u << c;
             }
-            if (sw) atomicOr(&ctl.anysw, 1);
+            if (swm) atomicOr(&cl.swm, (int)swm);
 #pragma unroll
             for (int c = 0; c < P; c++)
-                if ((badm >> c) & 1u) atomicOr(&ctl.flags[c], MAGIS_ST_BAD_DEC);
+                if ((badm >> c) & 1u) atomicOr(&cl.flags[c], MAGIS_ST_BAD_DEC);
         }
         // ---- phase 1: inverse permutation (pos stored +1); this thread's
         //      chunk of its team's candidate stays in registers for the scan
@@ -382,43 +472,53 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     if (j + 3 < LR) pr[(j + 3) % LR] = v.w;
                 }
             }
-            if (bad) atomicOr(&ctl.flags[cm], MAGIS_ST_NOT_PERM);
+            if (bad) atomicOr(&cl.flags[cm], MAGIS_ST_NOT_PERM);
+        }
+        // the control words of the next group (last read one group ago)
+        if (tid == 0) {
+            Ctl& cn = ctl[slot ^ 1];
+            for (int c = 0; c < 4; c++) { cn.flags[c] = 0; cn.viol[c] = 0; }
+            cn.swm = 0;
         }
         bar_sync(kBarMain, TM);
         PROF_MARK(1);
-        const bool anysw = ctl.anysw != 0;
-        // ---- phase 2: optional nodes, virtual late-user slots ------------------
-        double bl[P];
-        int nev[P];
-#pragma unroll
-        for (int c = 0; c < P; c++) { bl[c] = 0.0; nev[c] = 0; }
+        // ---- phase 2: optional nodes, virtual late-user slots, swap-event
+        //      steps (producer, Store, Load and late users of swapped tensors)
         for (int q = tid; q < P * R; q += TM) {
             const int c = q / R, r = q - c * R;
+            if (!((vmask >> c) & 1u)) continue;
             const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
 #pragma unroll
             for (int cc = 0; cc < P; cc++) {
-                if (cc != c || !((vmask >> cc) & 1u)) continue;
+                if (cc != c) continue;
                 const uint8_t d = dec_s[cc * R + r];
+                uint32_t* em = evm + cc * nwm;
 #pragma unroll
                 for (int o = 0; o < 3; o++) {
                     const int32_t id = n + 3 * r + o;
                     const uint32_t p = pos[id * P + cc];
                     if (p == 0) {
-                        atomicOr(&ctl.flags[cc], MAGIS_ST_NOT_PERM);
+                        atomicOr(&cl.flags[cc], MAGIS_ST_NOT_PERM);
                         continue;
                     }
                     const bool act = (o == 0) ? (d == 1) : (d == 2);
+                    const uint32_t st = p - 1;
                     if (!act) {
-                        const uint32_t st = p - 1;
                         AF[cc * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
                         pos[id * P + cc] = 0;
+                    } else if (o > 0) {
+                        atomicOr(em + (st >> 5), 1u << (st & 31));
                     }
                 }
-                if (d == 1) bl[cc] += __ldg(g.tcost + r);
-                if (d == 2) nev[cc] += 3 + (u1 - u0);
+                if (d == 2) {
+                    const uint32_t pt_ = pos[__ldg(g.elig + r) * P + cc];
+                    if (pt_) atomicOr(em + ((pt_ - 1) >> 5), 1u << ((pt_ - 1) & 31));
+                }
                 for (int32_t j = u0; j < u1; j++) {
                     const int32_t b = __ldg(g.U_idx + j);
-                    pos[(NT + j) * P + cc] = (d == 0) ? pos[b * P + cc] : (uint16_t)0;
+                    const uint32_t pb = pos[b * P + cc];
+                    pos[(NT + j) * P + cc] = (d == 0) ? (uint16_t)pb : (uint16_t)0;
+                    if (d == 2 && pb) atomicOr(em + ((pb - 1) >> 5), 1u << ((pb - 1) & 31));
                 }
             }
         }
@@ -457,8 +557,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             }
 #pragma unroll
             for (int c = 0; c < P; c++) {
-                if (nperm & (1 << c)) atomicOr(&ctl.flags[c], MAGIS_ST_NOT_PERM);
-                if (viol & (1 << c)) atomicOr(&ctl.viol[c], MAGIS_ST_EDGE);
+                if (nperm & (1 << c)) atomicOr(&cl.flags[c], MAGIS_ST_NOT_PERM);
+                if (viol & (1 << c)) atomicOr(&cl.viol[c], MAGIS_ST_EDGE);
             }
         }
         bar_sync(kBarMain, TM);
@@ -467,62 +567,103 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         uint32_t stm = 0, okm = 0;
 #pragma unroll
         for (int c = 0; c < P; c++) {
-            const int f = ctl.flags[c];
-            const uint32_t st = ((vmask >> c) & 1u) ? (uint32_t)(f ? f : ctl.viol[c]) : 0u;
+            const int f = cl.flags[c];
+            const uint32_t st = ((vmask >> c) & 1u) ? (uint32_t)(f ? f : cl.viol[c]) : 0u;
             stm |= st << (4 * c);
             if (((vmask >> c) & 1u) && st == 0) okm |= 1u << c;
         }
-        const bool anyok = okm != 0;
-        if (anyok) {
+        const uint32_t swm = (uint32_t)cl.swm & okm;       // valid candidates with swaps
+        const bool mysw = (swm >> cm) & 1u;
+        // event steps of this thread's chunk and their order within the warp
+        const int32_t nst = ((okm >> cm) & 1u) ? max(0, min(L, NT - lo)) : 0;   // steps of this chunk
+        const unsigned long long mbits =
+            (mysw && nst > 0) ? mark_bits(evm + cm * nwm, lo, L) & (~0ull >> (64 - nst)) : 0ull;
+        int evx = __popcll(mbits);
+        {
+            int inc = evx;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int x = __shfl_up_sync(0xffffffffu, inc, o);
+                if (lane >= o) inc += x;
+            }
+            if (lane == 31) wcnt[warp] = inc;
+            evx = inc - evx;
+        }
+        if (okm != 0) {
             // ---- phase 4: frees over the input rows -> per-step slots ------------
-            {
-                const uint32_t r0 = wtab[warp * 4 + 2], r1 = wtab[warp * 4 + 3];
-                for (uint32_t r = r0; r < r1; r++) {
-                    const uint2 rw = frow[r];
-                    const uint32_t h = fhdr[r * 32 + lane];
-                    const uint32_t kind = h >> kKindShift, id = h & kIdMask;
-                    const V p = PK::load(pos, id);
-                    const V lv = PK::load(last, id);
-                    const uint32_t A = size_s[id];
-                    uint32_t fr[P];
+            const uint32_t r0 = wtab[warp * 4 + 2], r1 = wtab[warp * 4 + 3];
+            for (uint32_t r = r0; r < r1; r++) {
+                const uint2 rw = frow[r];
+                const uint32_t h = fhdr[r * 32 + lane];
+                const uint32_t kind = h >> kKindShift, id = h & kIdMask;
+                const V p = PK::load(pos, id);
+                const V lv = PK::load(last, id);
+                const uint32_t A = size_s[id];
+                uint32_t fr[P];
 #pragma unroll
-                    for (int c = 0; c < P; c++) {
-                        const uint32_t pc = PK::get(p, c);
-                        fr[c] = (pc != 0 && PK::get(lv, c) == pc) ? A : 0u;   // no reader: freed after own step
-                    }
-                    const uint16_t* ent = fent + rw.x + lane;
+                for (int c = 0; c < P; c++) {
+                    const uint32_t pc = PK::get(p, c);
+                    fr[c] = (pc != 0 && PK::get(lv, c) == pc) ? A : 0u;   // no reader: freed after own step
+                }
+                const uint16_t* ent = fent + rw.x + lane;
 #pragma unroll 4
-                    for (uint32_t j = 0; j < rw.y; j++) {
-                        const uint32_t u = ent[j * 32];
-                        const V l = PK::load(last, u);
-                        if (PK::maybe_eq(l, p)) {
-                            const uint32_t su = size_s[u];
-#pragma unroll
-                            for (int c = 0; c < P; c++) {
-                                const uint32_t pc = PK::get(p, c);
-                                if (pc != 0 && PK::get(l, c) == pc) fr[c] += su;
-                            }
-                        }
-                    }
-                    if (kind != kNop) {
+                for (uint32_t j = 0; j < rw.y; j++) {
+                    const uint32_t u = ent[j * 32];
+                    const V l = PK::load(last, u);
+                    if (PK::maybe_eq(l, p)) {
+                        const uint32_t su = size_s[u];
 #pragma unroll
                         for (int c = 0; c < P; c++) {
                             const uint32_t pc = PK::get(p, c);
-                            if (pc == 0 || !((okm >> c) & 1u)) continue;
-                            const uint32_t st = pc - 1;
-                            AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(A, fr[c]);
+                            if (pc != 0 && PK::get(l, c) == pc) fr[c] += su;
                         }
                     }
                 }
+                if (kind != kNop) {
+#pragma unroll
+                    for (int c = 0; c < P; c++) {
+                        const uint32_t pc = PK::get(p, c);
+                        if (pc == 0 || !((okm >> c) & 1u)) continue;
+                        const uint32_t st = pc - 1;
+                        AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(A, fr[c]);
+                    }
+                }
             }
-            bar_sync(kBarMain, TM);
-            PROF_MARK(4);
+        }
+        // the slot of this group parity is free once the latency warp is done
+        // with group gi - 2
+        PROF_MARK(9);
+        if (gi >= 2) bar_sync(kBarEmpty + slot, TM + TL);
+        else bar_sync(kBarMain, TM);
+        PROF_MARK(4);
+        SlotHdr& h = hdr[slot];
+        // event list of candidate cm: shared-memory slot, or global overflow
+        int ntot = 0, wpre = 0;
+#pragma unroll
+        for (int w = 0; w < WT; w++) {
+            const int x = wcnt[cm * WT + w];
+            ntot += x;
+            if (w < warp - cm * WT) wpre += x;
+        }
+        unsigned long long* kout;
+        double* cout_;
+        if (ntot <= cap) {
+            kout = evk_s + (size_t)(slot * P + cm) * cap;
+            cout_ = evc_s + (size_t)(slot * P + cm) * cap;
+        } else {
+            char* ob = ovf + ((size_t)blockIdx.x * 8 + slot * 4 + cm) * pl.ovf_stride;
+            kout = (unsigned long long*)ob;
+            cout_ = (double*)(ob + (size_t)pl.max_events * 8);
+        }
+        if (okm != 0) {
             // ---- phase 5: scan of the (sum, max-prefix) monoid ------------------
-            //      team cm scans candidate cm: alloc = size of the op at each step
-            //      (perm chunk in registers), free = Fs slot, compute cost per step
+            //      team cm scans candidate cm: alloc = size of the op at each step,
+            //      free = slot; with swaps also the compute-cost prefix, and the
+            //      event steps of the chunk are emitted in order
             long long s1 = 0, m1 = kNegInf;
             double cs1 = 0.0;
-            const int32_t nst = ((okm >> cm) & 1u) ? min(L, NT - lo) : 0;   // steps of this chunk
+            int o = wpre + evx;
+            const int o0 = o;
 #pragma unroll
             for (int j = 0; j < LMAX; j++) {
                 if (j < nst) {
@@ -530,9 +671,14 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     s1 += af.x;
                     m1 = max(m1, s1);
                     s1 -= af.y;
-                    if (anysw) {
+                    if (mysw) {
                         const int32_t v = LMAX <= 16 ? pr[j % LR]
                                                      : __ldg(perm + (grp * P + cm) * (int64_t)NT + lo + j);
+                        if ((mbits >> j) & 1ull) {
+                            kout[o] = ((unsigned long long)(lo + j) << 32) | (uint32_t)v;
+                            cout_[o] = cs1;
+                            o++;
+                        }
                         if (v < n || pos[v * P + cm] != 0) cs1 += cost_s[v];
                     }
                 }
@@ -542,174 +688,80 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 long long ss = s1, mm = m1;
                 double cc = cs1;
 #pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const long long ps = __shfl_up_sync(0xffffffffu, ss, o);
-                    const long long pm = __shfl_up_sync(0xffffffffu, mm, o);
-                    const double pc = __shfl_up_sync(0xffffffffu, cc, o);
-                    if (lane >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
+                for (int o2 = 1; o2 < 32; o2 <<= 1) {
+                    const long long ps = __shfl_up_sync(0xffffffffu, ss, o2);
+                    const long long pm = __shfl_up_sync(0xffffffffu, mm, o2);
+                    const double pc = __shfl_up_sync(0xffffffffu, cc, o2);
+                    if (lane >= o2) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
                 }
-                if (anysw) cofs[tid] = cc - cs1;
                 if (lane == 31) { agg_s[warp] = ss; agg_m[warp] = mm; agg_c[warp] = cc; }
-#pragma unroll
-                for (int c = 0; c < P; c++) {
-                    double b = bl[c];
-                    int nn = nev[c];
-#pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) {
-                        b += __shfl_xor_sync(0xffffffffu, b, o);
-                        nn += __shfl_xor_sync(0xffffffffu, nn, o);
-                    }
-                    if (lane == 0) { agg_b[warp][c] = b; agg_n[warp][c] = nn; }
-                }
+                // add the lane's exclusive cost prefix within the warp to its events
+                const double pre = cc - cs1;
+                for (int e = o0; e < o; e++) cout_[e] += pre;
             }
-            bar_sync(kBarMain, TM);
-            PROF_MARK(5);
-            if (warp == 0) {
-                // fold the WT warp aggregates of each team (segments of WT lanes)
-                long long ss = lane < WM ? agg_s[lane] : 0;
-                long long mm = lane < WM ? agg_m[lane] : kNegInf;
-                double cc = lane < WM ? agg_c[lane] : 0.0;
-                const double c0 = cc;
+        }
+        bar_sync(kBarMain, TM);
+        PROF_MARK(5);
+        // ---- phase 6: fold the team aggregates, hand-off to the latency warp ------
+        if (warp == 0) {
+            long long ss = lane < WM ? agg_s[lane] : 0;
+            long long mm = lane < WM ? agg_m[lane] : kNegInf;
+            double cc = lane < WM ? agg_c[lane] : 0.0;
+            const double c0 = cc;
 #pragma unroll
-                for (int o = 1; o < WT; o <<= 1) {
-                    const long long ps = __shfl_up_sync(0xffffffffu, ss, o, WT);
-                    const long long pm = __shfl_up_sync(0xffffffffu, mm, o, WT);
-                    const double pc = __shfl_up_sync(0xffffffffu, cc, o, WT);
-                    if ((lane % WT) >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
-                }
-                if (lane < WM) fold.woff[lane] = cc - c0;
-                if (lane < WM && (lane % WT) == WT - 1) {
-                    const int c = lane / WT;
-                    fold.peak[c] = mm;
-                    fold.ctot[c] = cc;
-                }
-#pragma unroll
-                for (int c = 0; c < P; c++) {
-                    double b = lane < WM ? agg_b[lane][c] : 0.0;
-                    int nn = lane < WM ? agg_n[lane][c] : 0;
-#pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) {
-                        b += __shfl_xor_sync(0xffffffffu, b, o);
-                        nn += __shfl_xor_sync(0xffffffffu, nn, o);
-                    }
-                    if (lane == 0) {
-                        fold.basel[c] = g.base_cost + b;
-                        fold.nev[c] = ((okm >> c) & 1u) ? nn : 0;
-                    }
-                }
+            for (int o = 1; o < WT; o <<= 1) {
+                const long long ps = __shfl_up_sync(0xffffffffu, ss, o, WT);
+                const long long pm = __shfl_up_sync(0xffffffffu, mm, o, WT);
+                const double pc = __shfl_up_sync(0xffffffffu, cc, o, WT);
+                if ((lane % WT) >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
             }
-            bar_sync(kBarMain, TM);
-            PROF_MARK(6);
-        } else if (tid == 0) {
+            if (lane < WM) h.woff[lane] = cc - c0;
+            // team totals sit in lane c * WT + WT - 1
+            const int src = (lane < P ? lane : 0) * WT + WT - 1;
+            const long long pk = __shfl_sync(0xffffffffu, mm, src);
+            const double ct = __shfl_sync(0xffffffffu, cc, src);
+            int ne = 0;
 #pragma unroll
-            for (int c = 0; c < P; c++) { fold.peak[c] = 0; fold.ctot[c] = 0.0; fold.basel[c] = 0.0; fold.nev[c] = 0; }
-        }
-        int nevt[P];
-        bool anyev = false;
-#pragma unroll
-        for (int c = 0; c < P; c++) {
-            nevt[c] = anyok ? fold.nev[c] : 0;
-            anyev |= nevt[c] > 0;
-        }
-        // ---- phase 6: swap events -> hand-off slot --------------------------------
-        if (gi >= 2) bar_sync(kBarEmpty + slot, TM + 32);
-        PROF_MARK(7);
-        SlotHdr& h = hdr[slot];
-        if (tid == 0) {
-#pragma unroll
-            for (int c = 0; c < P; c++) {
+            for (int w = 0; w < WT; w++) ne += wcnt[(lane < P ? lane : 0) * WT + w];
+            if (lane < P) {
+                const int c = lane;
+                const bool ok = (okm >> c) & 1u;
                 h.k[c] = ((vmask >> c) & 1u) ? grp * P + c : LLONG_MAX;
                 h.status[c] = (int)((stm >> (4 * c)) & 15u);
-                h.peak[c] = fold.peak[c];
-                h.ctot[c] = fold.ctot[c];
-                h.basel[c] = fold.basel[c];
-                h.nev[c] = nevt[c];
-                h.cnt[c] = 0;
-                if (nevt[c] <= pl.evcap) {
-                    h.key[c] = evk_s + (size_t)(slot * P + c) * 2 * pl.evcap;
-                    h.cb[c] = evcb_s + (size_t)(slot * P + c) * pl.evcap;
-                } else {
-                    char* ob = ovf + ((size_t)blockIdx.x * 8 + slot * 4 + c) * pl.ovf_stride;
-                    h.key[c] = (unsigned long long*)ob;
-                    h.cb[c] = (double*)(ob + (size_t)2 * pl.max_events * 8);
-                }
+                h.peak[c] = ok ? pk : 0;
+                h.ctot[c] = ok ? ct : 0.0;
+                h.swp[c] = (int)((swm >> c) & 1u);
+                h.nev[c] = ne;
             }
         }
-        if (anyev) {
-            bar_sync(kBarMain, TM);
-            PROF_MARK(8);
-            for (int q = tid; q < P * R; q += TM) {
-                const int c0 = q / R, r = q - c0 * R;
-                const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
-                const unsigned long long rr = (unsigned long long)r;
+        if (R > 0) {
+            // decisions of the group -> the slot (rows padded to 16 bytes)
+            const int nw = Rw >> 2;
+            uint32_t* dst = reinterpret_cast<uint32_t*>(sdec + (size_t)slot * P * Rw);
+            for (int i = tid; i < P * nw; i += TM) {
+                const int c = i / nw, w = i - c * nw;
+                uint32_t x = 0;
 #pragma unroll
-                for (int c = 0; c < P; c++) {
-                    if (c != c0 || nevt[c] == 0 || dec_s[c * R + r] != 2) continue;
-                    const int b0 = atomicAdd(&h.cnt[c], 3 + (u1 - u0));
-                    unsigned long long* kin = h.key[c];
-                    const unsigned long long pt = (unsigned long long)pos[__ldg(g.elig + r) * P + c] - 1;
-                    const unsigned long long ps = (unsigned long long)pos[(n + 3 * r + 1) * P + c] - 1;
-                    const unsigned long long pq = (unsigned long long)pos[(n + 3 * r + 2) * P + c] - 1;
-                    kin[b0 + 0] = (pt << 32) | ((unsigned long long)kEvProduce << 24) | rr;
-                    kin[b0 + 1] = (ps << 32) | ((unsigned long long)kEvStore << 24) | rr;
-                    kin[b0 + 2] = (pq << 32) | ((unsigned long long)kEvLoad << 24) | rr;
-                    for (int32_t j = u0; j < u1; j++) {
-                        const unsigned long long pb = (unsigned long long)pos[__ldg(g.U_idx + j) * P + c] - 1;
-                        kin[b0 + 3 + (j - u0)] = (pb << 32) | ((unsigned long long)kEvStall << 24) | rr;
-                    }
+                for (int b = 0; b < 4; b++) {
+                    const int r = 4 * w + b;
+                    if (r < R) x |= (uint32_t)dec_s[c * R + r] << (8 * b);
                 }
-            }
-            bar_sync(kBarMain, TM);
-            PROF_MARK(9);
-            // rank sort (unique keys) + compute-cost prefix before each event:
-            // cost of the steps of earlier warps' chunks, earlier lanes of the
-            // same warp, then the steps of the owning chunk before the event
-            int tot = 0;
-#pragma unroll
-            for (int c = 0; c < P; c++) tot += nevt[c];
-            for (int q = tid; q < tot; q += TM) {
-                int c = 0, e = q;
-                while (e >= nevt[c]) { e -= nevt[c]; c++; }
-                const unsigned long long* kin = h.key[c];
-                const int ne = nevt[c];
-                const unsigned long long key = kin[e];
-                int rank = 0;
-                for (int j = 0; j < ne; j++) rank += (kin[j] < key);
-                const int32_t stp = (int32_t)(key >> 32);
-                const int32_t th = stp >> lgL;
-                double cb = fold.woff[c * WT + (th >> 5)] + cofs[c * TPC + th];
-                const int32_t* Pp = perm + (grp * P + c) * (int64_t)NT + th * L;
-                const int32_t nb = stp - th * L;
-#pragma unroll 4
-                for (int32_t i = 0; i < nb; i++) {
-                    const int32_t v = __ldg(Pp + i);
-                    if (v < n || pos[v * P + c] != 0) cb += cost_s[v];
-                }
-                h.key[c][ne + rank] = key;
-                h.cb[c][rank] = cb;
+                dst[i] = x;
             }
         }
         __threadfence_block();
-        bar_arrive(kBarFull + slot, TM + 32);
-        PROF_MARK(10);
-        // reset the per-group control words for the next group, then make sure
-        // every main thread is done with pos / Fs / ctl before they are reused
-        if (tid == 0) {
-            for (int c = 0; c < 4; c++) { ctl.flags[c] = 0; ctl.viol[c] = 0; }
-            ctl.anysw = 0;
-        }
-        // every main thread must be done reading pos (event keys, cost prefix)
-        if (anyev) bar_sync(kBarMain, TM);
-        PROF_MARK(11);
-        // clear pos so a missing node (duplicate in perm) reads as 0 next group
+        bar_arrive(kBarFull + slot, TM + TL);
+        PROF_MARK(6);
+        // clear pos and the event marks for the next group
         {
             const int nb = NT * P * 2;
             uint4* p4 = reinterpret_cast<uint4*>(pos);
             for (int i = tid; i < (nb >> 4); i += TM) p4[i] = make_uint4(0u, 0u, 0u, 0u);
             for (int i = ((nb >> 4) << 3) + tid; i < NT * P; i += TM) pos[i] = 0;
+            for (int i = tid; i < P * nwm; i += TM) evm[i] = 0;
         }
         bar_sync(kBarMain, TM);
-        PROF_MARK(12);
+        PROF_MARK(7);
     }
     if (prof)
 #pragma unroll
@@ -753,7 +805,7 @@ cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
         std::fprintf(stderr, "[magis] eval2 P=%d regs=%d static_smem=%zu local=%zu\n", pl.P, fa.numRegs,
                      fa.sharedSizeBytes, fa.localSizeBytes);
     }
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, TM + 32, pl.smem_total);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, TM + 32 * pl.P, pl.smem_total);
 }
 
 cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,
@@ -764,7 +816,7 @@ cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, v
     const int gr = (int)std::min<int64_t>(grid, ngroups);
     void* args[] = {(void*)&g, (void*)&pl, (void*)&blob, (void*)&K, (void*)&perm, (void*)&dec,
                     (void*)&status, (void*)&peak, (void*)&lat, (void*)&ovf, (void*)&afg};
-    return cudaLaunchKernel(kernel_for(pl), dim3(gr), dim3(TM + 32), args, pl.smem_total, stream);
+    return cudaLaunchKernel(kernel_for(pl), dim3(gr), dim3(TM + 32 * pl.P), args, pl.smem_total, stream);
 }
 
 }  // namespace magis

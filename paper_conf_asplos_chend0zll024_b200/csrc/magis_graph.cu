@@ -353,7 +353,8 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
             std::vector<double> rtab((size_t)2 * R);
             for (int32_t r = 0; r < R; r++) { rtab[2 * r] = tcost[r]; rtab[2 * r + 1] = xfer[r]; }
             SuperGraphHost sg{n, R, NT, cons_ptr.data(), cons_ent.data(), in_ptr.data(), in_ent.data(),
-                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data(), rtab.data()};
+                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data(), rtab.data(),
+                              elig.data()};
             const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
             // pick the packing with the most candidates in flight per SM
             // (P x resident CTAs; ties go to more CTAs, which hide barriers).
@@ -405,7 +406,7 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
                     g->ovf2 = ov;
                     g->cfg.variant = 2;
                     g->cfg.grid = grid;
-                    g->cfg.block = kMainThreads2 + 32;
+                    g->cfg.block = kMainThreads2 + 32 * bestPl.P;
                     g->cfg.smem = bestPl.smem_total;
                 } else {
                     cudaGetLastError();

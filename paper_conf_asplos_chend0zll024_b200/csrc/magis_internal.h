@@ -63,7 +63,6 @@ struct Plan2 {
     int32_t NT, NTX, n, R, nU;
     int32_t L, S;         // scan chunk length / slot stride (L * S >= NT, S <= kMainThreads2)
     int64_t unit;         // bytes per size unit (gcd of sizes)
-    int32_t evcap;        // events per candidate held in shared memory
     int32_t max_events;   // 3R + |U|
     int32_t lgL;          // L = 1 << lgL
     uint32_t static_bytes;   // bulk-staged prefix (graph rows + size units)
@@ -73,15 +72,23 @@ struct Plan2 {
     uint32_t off_size;       // [NTX] size units
     uint32_t off_rtab;       // [R] double2 (cost(t_r), swap transfer time)
     uint32_t off_cost;       // [NTX] compute cost (f64; clone = cost(t_r), Store / Load 0)
-    uint32_t off_pos, off_last, off_af, off_dec, off_cofs, off_end, off_ev;   // off_af: free slots
+    uint32_t off_ninfo;      // [n] uint2: x = (r + 1 if node is t_r, else 0) | |{r : node in U_r}| << 16,
+                             //            y = offset of that r list in lul
+    uint32_t off_lul;        // u16 r lists (late-user -> tensors), see off_ninfo
+    uint32_t off_pos, off_last, off_af, off_dec, off_end;
+    uint32_t off_evm;        // [P][NW] swap-event step marks (bit per step)
+    uint32_t off_sdec;       // [2][P][Rw] decisions handed to the latency warp
+    uint32_t off_ev;         // [2][P][evcap] event keys (u64) then [2][P][evcap] cost prefixes (f64)
+    int32_t evcap;           // event steps per candidate held in shared memory
+    int32_t nwm;             // NW: u32 words of marks per candidate
+    uint64_t ovf_stride;     // bytes per overflow event region (global)
     uint32_t smem_total;
-    uint64_t ovf_stride;  // bytes per overflow event region (global)
     int32_t gmem_static;  // graph tables read from the global image instead of shared memory
     int32_t gmem_af;      // per-step slots in a per-CTA global slice (af_bytes each)
     uint32_t state_base;  // offset of the per-candidate state in shared memory
     uint64_t af_bytes;
     int32_t prof;         // MAGIS_PROFILE: accumulate per-phase cycles
-    uint64_t prof_off;    // byte offset of the 16 u64 phase counters in the overflow buffer
+    uint64_t prof_off;    // byte offset of the 16 u64 phase counters in the scratch buffer
 };
 
 // Base-graph adjacency for the device candidate generator (magis_gen.cu).
@@ -163,6 +170,7 @@ struct SuperGraphHost {
     const int32_t* U_ptr;      // [R+1]
     const int32_t* U_idx;
     const double* rtab;        // [R][2] (cost(t_r), swap transfer time)
+    const int32_t* elig;       // [R] t_r
 };
 
 // Build the variant-2 plan and its static shared-memory image for a given P.

@@ -101,7 +101,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
     const int32_t NT = sg.NT, n = sg.n, R = sg.R;
     const int32_t nU = R > 0 ? sg.U_ptr[R] : 0;
     const int64_t NTX = (int64_t)NT + nU + 1;
-    if (NTX >= 65535 || NT < 1) return false;            // u16 positions (stored +1)
+    if (NTX >= 65535 || NT < 1 || R >= 65535) return false;   // u16 positions (stored +1), u16 tensor ids
     // size units
     uint64_t gg = 0;
     for (int32_t v = 0; v < NT; v++) if (sg.size[v] > 0) gg = gcd64(gg, (uint64_t)sg.size[v]);
@@ -184,6 +184,8 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
     p.off_size = (uint32_t)o;  o = a16(o + size_u.size() * 4);
     p.off_cost = (uint32_t)o;  o = a16(o + cost_u.size() * 8);
     p.off_rtab = (uint32_t)o;  o = a16(o + (size_t)std::max(R, 1) * 16);
+    p.off_ninfo = (uint32_t)o; o = a16(o + (size_t)n * 8);
+    p.off_lul = (uint32_t)o;   o = a16(o + (size_t)std::max(nU, 1) * 2);
     p.static_bytes = (uint32_t)o;
     // graph tables in shared memory (staged) or read from the global image
     // (L1/L2; the row reads stay coalesced); per-step slots in shared memory or
@@ -198,17 +200,20 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
     p.off_last = (uint32_t)o; o = a16(o + (size_t)NTX * P * 2);
     p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * 8));
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
-    p.off_cofs = (uint32_t)o; o = a16(o + (size_t)kMainThreads2 * 8);
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
+    p.nwm = (NT + 31) / 32 + 2;
+    p.off_evm = (uint32_t)o;  o = a16(o + (size_t)P * p.nwm * 4);
+    p.off_sdec = (uint32_t)o; o = a16(o + (size_t)2 * P * ((std::max(R, 1) + 15) & ~15));
     p.off_ev = (uint32_t)o;
-    int cap = std::min(p.max_events, 64);
+    // event steps of a candidate: at most the marked steps (<= 3R + |U|)
+    int cap = std::min(std::max(p.max_events, 1), 128);
     while (true) {
-        size_t need = o + (size_t)2 * P * (size_t)std::max(cap, 1) * 24;
+        const size_t need = o + (size_t)2 * P * cap * 24;
         if (need <= smem_cap) { p.smem_total = (uint32_t)a16(need); break; }
-        if (cap <= 16) return false;
+        if (cap <= 8) return false;
         cap /= 2;
     }
-    p.evcap = std::max(cap, 1);
+    p.evcap = cap;
     p.ovf_stride = (uint64_t)((std::max(p.max_events, 1) * 24 + 255) / 256 * 256);
     *pl = p;
     img->assign(p.static_bytes, 0);
@@ -225,6 +230,24 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
     put(p.off_size, size_u.data(), size_u.size() * 4);
     put(p.off_cost, cost_u.data(), cost_u.size() * 8);
     put(p.off_rtab, sg.rtab, (size_t)R * 16);
+    // per original node: the tensor it produces (if eligible) and the eligible
+    // tensors it is a late user of -- the swap events it can raise (reading P7)
+    {
+        std::vector<std::vector<uint16_t>> lu(n);
+        for (int32_t r = 0; r < R; r++)
+            for (int32_t j = sg.U_ptr[r]; j < sg.U_ptr[r + 1]; j++) lu[sg.U_idx[j]].push_back((uint16_t)r);
+        std::vector<uint32_t> ninfo((size_t)2 * n, 0);
+        std::vector<uint16_t> lul;
+        for (int32_t v = 0; v < n; v++) {
+            if (lu[v].size() > 31) return false;       // swapped-late-user mask of the event steps
+            ninfo[2 * v] = (uint32_t)lu[v].size() << 16;
+            ninfo[2 * v + 1] = (uint32_t)lul.size();
+            lul.insert(lul.end(), lu[v].begin(), lu[v].end());
+        }
+        for (int32_t r = 0; r < R; r++) ninfo[2 * sg.elig[r]] |= (uint32_t)(r + 1);
+        put(p.off_ninfo, ninfo.data(), ninfo.size() * 4);
+        put(p.off_lul, lul.data(), lul.size() * 2);
+    }
     return true;
 }
 
