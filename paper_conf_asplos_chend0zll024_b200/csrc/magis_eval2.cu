@@ -411,6 +411,34 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const int cm = tid / TPC, tt = tid - cm * TPC;
     const int32_t lo = tt * L;
     const bool vec4 = (NT & 3) == 0;
+    constexpr int LR = LMAX <= 16 ? LMAX : 1;      // perm chunk kept in registers when short
+    int32_t pr[LR];
+    // this thread's chunk of candidate cm of group grp_ (-1 past the end)
+    auto load_chunk = [&](int64_t grp_) {
+        const bool vc = grp_ * P + cm < K;
+        const int32_t* Pp = perm + (grp_ * P + cm) * (int64_t)NT + lo;
+#pragma unroll
+        for (int j = 0; j < LR; j += 4) {
+            int4 v = make_int4(-1, -1, -1, -1);
+            if (vc && j < L && lo + j < NT) {
+                if (vec4) {
+                    v = __ldcs(reinterpret_cast<const int4*>(Pp + j));
+                } else {
+                    v.x = __ldcs(Pp + j);
+                    if (lo + j + 1 < NT) v.y = __ldcs(Pp + j + 1);
+                    if (lo + j + 2 < NT) v.z = __ldcs(Pp + j + 2);
+                    if (lo + j + 3 < NT) v.w = __ldcs(Pp + j + 3);
+                }
+            }
+            pr[j] = v.x;
+            if (j + 1 < LR) pr[j + 1] = v.y;
+            if (j + 2 < LR) pr[j + 2] = v.z;
+            if (j + 3 < LR) pr[j + 3] = v.w;
+        }
+    };
+    if constexpr (LMAX <= 16) {
+        if (ncta > 0) load_chunk(blockIdx.x);
+    }
     for (int gi = 0; gi < ncta; gi++) {
         const int64_t grp = blockIdx.x + (int64_t)gi * gridDim.x;
         const int slot = gi & 1;
@@ -434,42 +462,45 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 if ((badm >> c) & 1u) atomicOr(&cl.flags[c], MAGIS_ST_BAD_DEC);
         }
         // ---- phase 1: inverse permutation (pos stored +1); this thread's
-        //      chunk of its team's candidate stays in registers for the scan
-        constexpr int LR = LMAX <= 16 ? LMAX : 1;      // perm chunk kept in registers when short
-        int32_t pr[LR];
+        //      chunk of its team's candidate is in registers (loaded during the
+        //      previous group) when short, else streamed here
         {
-            const int32_t* Pp = perm + (grp * P + cm) * (int64_t)NT + lo;
             int bad = 0;
             const bool vc = (vmask >> cm) & 1u;
+            if constexpr (LMAX <= 16) {
 #pragma unroll
-            for (int j = 0; j < LMAX; j += 4) {
-                int4 v = make_int4(-1, -1, -1, -1);
-                if (vc && j < L && lo + j < NT) {
-                    if (vec4) {
-                        v = __ldcs(reinterpret_cast<const int4*>(Pp + j));
-                    } else {
-                        v.x = __ldcs(Pp + j);
-                        if (lo + j + 1 < NT) v.y = __ldcs(Pp + j + 1);
-                        if (lo + j + 2 < NT) v.z = __ldcs(Pp + j + 2);
-                        if (lo + j + 3 < NT) v.w = __ldcs(Pp + j + 3);
-                    }
-                    const uint32_t i0 = (uint32_t)(lo + j);
-                    if ((uint32_t)v.x < (uint32_t)NT) pos[v.x * P + cm] = (uint16_t)(i0 + 1); else bad = 1;
-                    if (i0 + 1 < (uint32_t)NT) {
-                        if ((uint32_t)v.y < (uint32_t)NT) pos[v.y * P + cm] = (uint16_t)(i0 + 2); else bad = 1;
-                    }
-                    if (i0 + 2 < (uint32_t)NT) {
-                        if ((uint32_t)v.z < (uint32_t)NT) pos[v.z * P + cm] = (uint16_t)(i0 + 3); else bad = 1;
-                    }
-                    if (i0 + 3 < (uint32_t)NT) {
-                        if ((uint32_t)v.w < (uint32_t)NT) pos[v.w * P + cm] = (uint16_t)(i0 + 4); else bad = 1;
+                for (int j = 0; j < LMAX; j++) {
+                    if (vc && j < L && lo + j < NT) {
+                        const int32_t v = pr[j];
+                        if ((uint32_t)v < (uint32_t)NT) pos[v * P + cm] = (uint16_t)(lo + j + 1); else bad = 1;
                     }
                 }
-                if (LMAX <= 16) {
-                    pr[j % LR] = v.x;
-                    if (j + 1 < LR) pr[(j + 1) % LR] = v.y;
-                    if (j + 2 < LR) pr[(j + 2) % LR] = v.z;
-                    if (j + 3 < LR) pr[(j + 3) % LR] = v.w;
+            } else {
+                const int32_t* Pp = perm + (grp * P + cm) * (int64_t)NT + lo;
+#pragma unroll
+                for (int j = 0; j < LMAX; j += 4) {
+                    if (vc && j < L && lo + j < NT) {
+                        int4 v = make_int4(-1, -1, -1, -1);
+                        if (vec4) {
+                            v = __ldcs(reinterpret_cast<const int4*>(Pp + j));
+                        } else {
+                            v.x = __ldcs(Pp + j);
+                            if (lo + j + 1 < NT) v.y = __ldcs(Pp + j + 1);
+                            if (lo + j + 2 < NT) v.z = __ldcs(Pp + j + 2);
+                            if (lo + j + 3 < NT) v.w = __ldcs(Pp + j + 3);
+                        }
+                        const uint32_t i0 = (uint32_t)(lo + j);
+                        if ((uint32_t)v.x < (uint32_t)NT) pos[v.x * P + cm] = (uint16_t)(i0 + 1); else bad = 1;
+                        if (i0 + 1 < (uint32_t)NT) {
+                            if ((uint32_t)v.y < (uint32_t)NT) pos[v.y * P + cm] = (uint16_t)(i0 + 2); else bad = 1;
+                        }
+                        if (i0 + 2 < (uint32_t)NT) {
+                            if ((uint32_t)v.z < (uint32_t)NT) pos[v.z * P + cm] = (uint16_t)(i0 + 3); else bad = 1;
+                        }
+                        if (i0 + 3 < (uint32_t)NT) {
+                            if ((uint32_t)v.w < (uint32_t)NT) pos[v.w * P + cm] = (uint16_t)(i0 + 4); else bad = 1;
+                        }
+                    }
                 }
             }
             if (bad) atomicOr(&cl.flags[cm], MAGIS_ST_NOT_PERM);
@@ -699,6 +730,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const double pre = cc - cs1;
                 for (int e = o0; e < o; e++) cout_[e] += pre;
             }
+        }
+        // the next group's chunk is loaded while this group finishes
+        if constexpr (LMAX <= 16) {
+            if (gi + 1 < ncta) load_chunk(grp + gridDim.x);
         }
         bar_sync(kBarMain, TM);
         PROF_MARK(5);

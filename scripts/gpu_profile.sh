@@ -10,3 +10,5 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:eval2_kernel -s 3 -c 1 -o gpurun_out/prof_eval python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/ncu_full.log 2>&1
 tail -c 2500 gpurun_out/bench_full.log
 for f in gpurun_out/bench_c*.log gpurun_out/bench_ref.log; do echo $f; grep -o '"value": [0-9.e+]*, "unit"[^,]*' $f | head -1; grep -o '"frac": [0-9.]*' $f; done
+timeout 600 python bench.py --windows --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/bench_windows.log 2>&1
+grep -o '"value": [0-9.e+]*' gpurun_out/bench_windows.log | head -1
