@@ -56,6 +56,10 @@ def _load():
     lib.orc_graph_n_edges.argtypes = [P]
     lib.orc_eval.argtypes = [P, P, P, P, P, P, P]
     lib.orc_eval_batch.argtypes = [P, ctypes.c_int64, P, P, P, P, P]
+    lib.orc_idom.restype = ctypes.c_int
+    lib.orc_idom.argtypes = [P, P]
+    lib.orc_hotspots.restype = ctypes.c_int
+    lib.orc_hotspots.argtypes = [P, P, P, ctypes.c_int32, P, P, P, P]
     lib.orc_pareto.restype = ctypes.c_int64
     lib.orc_pareto.argtypes = [ctypes.c_int64, P, P, P, P, P]
     lib.orc_best_mem.restype = ctypes.c_int64
@@ -145,6 +149,31 @@ class OracleGraph:
         lt = np.zeros(K, np.float64)
         self._lib.orc_eval_batch(self._h, K, _ptr(perms), _ptr(decs), _ptr(st), _ptr(pk), _ptr(lt))
         return st, pk, lt
+
+    def idom(self):
+        """Immediate dominators of the original graph (-1: only the sources'
+        virtual root dominates), from the plain set definition."""
+        out = np.zeros(max(self.n, 1), np.int32)
+        if self._lib.orc_idom(self._h, _ptr(out)) != 0:
+            raise ValueError("oracle: cyclic graph")
+        return out[:self.n]
+
+    def hotspots(self, perm, dec=None, nsplit: int = 2):
+        """Memory hot-spots H (reading H1) and heat / score
+        (Eq. 3-4) -> (status, peak, hot[n] u8, heat[n] int64, score[n] f64)."""
+        perm = np.ascontiguousarray(perm, dtype=np.int32)
+        assert perm.shape == (self.n_total,)
+        if dec is None or self.R == 0:
+            dec = np.zeros(max(self.R, 1), dtype=np.uint8)
+        dec = np.ascontiguousarray(dec, dtype=np.uint8)
+        m = max(self.n, 1)
+        hot = np.zeros(m, np.uint8)
+        heat = np.zeros(m, np.int64)
+        score = np.zeros(m, np.float64)
+        pk = np.zeros(1, np.int64)
+        st = self._lib.orc_hotspots(self._h, _ptr(perm), _ptr(dec), int(nsplit), _ptr(hot), _ptr(heat),
+                                    _ptr(score), _ptr(pk))
+        return int(st), int(pk[0]), hot[:self.n], heat[:self.n], score[:self.n]
 
 
 def pareto(peak, lat, status, ids=None):

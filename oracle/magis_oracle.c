@@ -18,6 +18,8 @@
  *   4. compaction to the active order                       (reading: inactive nodes are no-ops)
  *   5. lifetimes S_j < i <= F_j, F = last reader            (reading P1, P2)
  *   6. event simulation, M_i, M_peak = max_i M_i, first argmax
+ *   (+) memory hot-spots and F-Trans heat / score over the dominator tree
+ *       (Eq. 3-4; reading H1)       -- orc_hotspots
  *   7. latency: three in-order queues (compute, D2H, H2D)   (reading P7, P8, P9)
  *
  * Super-graph ids: original nodes 0..n-1; for eligible tensor r:
@@ -147,9 +149,9 @@ static int64_t node_bytes(const orc_graph *g, int32_t v)
  * bit2 bad decision), peak bytes (-1 if invalid), latency (+inf if invalid),
  * first compacted step attaining the peak (-1 if invalid).
  */
-void orc_eval(const orc_graph *g, const int32_t *perm, const uint8_t *dec,
-              uint8_t *status_out, int64_t *peak_out, double *lat_out,
-              int64_t *argmax_out)
+static void eval_impl(const orc_graph *g, const int32_t *perm, const uint8_t *dec,
+                      uint8_t *status_out, int64_t *peak_out, double *lat_out,
+                      int64_t *argmax_out, uint8_t *hot_out)
 {
     const int32_t n = g->n, R = g->R, NT = g->NT;
     uint8_t status = 0;
@@ -259,15 +261,27 @@ void orc_eval(const orc_graph *g, const int32_t *perm, const uint8_t *dec,
             if (!active[i]) continue;
             next[i] = head[last[i]]; head[last[i]] = (int32_t)i;
         }
+        int64_t *curve = (int64_t *)malloc(sizeof(int64_t) * (nact ? nact : 1));
         peak = 0; argmax = -1;
         for (i = 0; i < nact; i++) {
             int32_t u;
             if (i > 0)
                 for (u = head[i - 1]; u >= 0; u = next[u]) cur -= node_bytes(g, u);
             cur += node_bytes(g, ord[i]);
+            curve[i] = cur;
             if (i == 0 || cur > peak) { peak = cur; argmax = i; }  /* first argmax (reading P10) */
         }
-        free(head); free(next);
+        /* memory hot-spots H = union of A_i over the steps with M_i = M_peak,
+         * A_i = {u : S_u <= i <= F_u}, by the definition */
+        if (hot_out) {
+            for (i = 0; i < NT; i++) hot_out[i] = 0;
+            for (i = 0; i < nact; i++) {
+                if (curve[i] != peak) continue;
+                for (k = 0; k < NT; k++)
+                    if (active[k] && step[k] <= i && i <= last[k]) hot_out[k] = 1;
+            }
+        }
+        free(head); free(next); free(curve);
     }
 
     /* 7. latency: compute, D2H (Store) and H2D (Load) are three in-order
@@ -323,6 +337,133 @@ done:
     if (argmax_out) *argmax_out = argmax;
     free(seen); free(active); free(pos); free(step); free(ord); free(last);
     free(tsrc); free(tdst);
+}
+
+void orc_eval(const orc_graph *g, const int32_t *perm, const uint8_t *dec,
+              uint8_t *status_out, int64_t *peak_out, double *lat_out,
+              int64_t *argmax_out)
+{
+    eval_impl(g, perm, dec, status_out, peak_out, lat_out, argmax_out, NULL);
+}
+
+/*
+ * Dominators of the original graph G (T = T(G)): u dominates v
+ * iff every path from a source (a node without predecessors) to v passes
+ * through u.  Plain iterative set intersection over a topological order,
+ * Dom(v) = {v} + intersection of Dom(p) over the predecessors p (sources:
+ * {v}), as n x n byte matrices.  dom[u * n + v] = 1 iff u dominates v.
+ * Returns NULL if G has a cycle.
+ */
+static uint8_t *dominators(const orc_graph *g)
+{
+    const int32_t n = g->n;
+    int32_t *indeg = (int32_t *)calloc(n ? n : 1, sizeof(int32_t));
+    int32_t *order = (int32_t *)malloc(sizeof(int32_t) * (n ? n : 1));
+    uint8_t *dom = (uint8_t *)calloc((size_t)n * n + 1, 1);
+    int64_t k;
+    int32_t head = 0, tail = 0, i, v, u;
+    for (k = 0; k < g->ne; k++) indeg[g->dst[k]]++;
+    for (v = 0; v < n; v++) if (indeg[v] == 0) order[tail++] = v;
+    while (head < tail) {
+        v = order[head++];
+        for (k = 0; k < g->ne; k++)
+            if (g->src[k] == v && --indeg[g->dst[k]] == 0) order[tail++] = g->dst[k];
+    }
+    if (tail != n) { free(indeg); free(order); free(dom); return NULL; }
+    for (i = 0; i < n; i++) {
+        int first = 1;
+        v = order[i];
+        for (k = 0; k < g->ne; k++) {
+            if (g->dst[k] != v) continue;
+            u = g->src[k];
+            if (first) {
+                int32_t w;
+                for (w = 0; w < n; w++) dom[(size_t)w * n + v] = dom[(size_t)w * n + u];
+                first = 0;
+            } else {
+                int32_t w;
+                for (w = 0; w < n; w++) dom[(size_t)w * n + v] &= dom[(size_t)w * n + u];
+            }
+        }
+        dom[(size_t)v * n + v] = 1;
+    }
+    free(indeg); free(order);
+    return dom;
+}
+
+/* Immediate dominator of every node (-1: dominated only by the sources'
+ * virtual root).  The strict dominators of v form a chain; idom(v) is the one
+ * dominated by all the others.  Returns 0, or -1 on a cycle. */
+int orc_idom(const orc_graph *g, int32_t *idom)
+{
+    const int32_t n = g->n;
+    uint8_t *dom = dominators(g);
+    int32_t v, u, w;
+    if (!dom) return -1;
+    for (v = 0; v < n; v++) {
+        idom[v] = -1;
+        for (u = 0; u < n; u++) {
+            int all = 1;
+            if (u == v || !dom[(size_t)u * n + v]) continue;
+            for (w = 0; w < n && all; w++)
+                if (w != v && dom[(size_t)w * n + v] && !dom[(size_t)w * n + u]) all = 0;
+            if (all) { idom[v] = u; break; }
+        }
+    }
+    free(dom);
+    return 0;
+}
+
+/*
+ * Memory hot-spots and the F-Trans metrics of one candidate.
+ *   H: the tensors live at some step where M_i = M_peak.  Over
+ *   the original graph (reading H1): a live clone A' or Load of t_r stands for
+ *   t_r; a Store holds no device bytes and does not count.
+ *   heat(v) = sum of |w| over w in H and in T.des(v)          (Eq. 3)
+ *   score(v) = (1 - 1/nsplit) heat(v) - sum of |u| over u in
+ *              G.inps(T.des(v)) minus H                          (Eq. 4)
+ *   where T.des(v) = {w : v dominates w} and G.inps(S) = the nodes outside S
+ *   with an edge into S.
+ * hot[n] u8, heat[n] int64, score[n] double (zeroed if the candidate is
+ * invalid).  Returns the status bits; *peak_out as orc_eval.
+ */
+int orc_hotspots(const orc_graph *g, const int32_t *perm, const uint8_t *dec, int32_t nsplit,
+                 uint8_t *hot, int64_t *heat, double *score, int64_t *peak_out)
+{
+    const int32_t n = g->n, NT = g->NT;
+    uint8_t status;
+    int64_t peak, k;
+    double lat;
+    int32_t v, w, r;
+    uint8_t *hs = (uint8_t *)calloc(NT ? NT : 1, 1);
+    uint8_t *dom, *in_s;
+    eval_impl(g, perm, dec, &status, &peak, &lat, NULL, hs);
+    *peak_out = peak;
+    for (v = 0; v < n; v++) { hot[v] = 0; heat[v] = 0; score[v] = 0.0; }
+    if (status) { free(hs); return status; }
+    for (v = 0; v < n; v++) hot[v] = hs[v];
+    for (r = 0; r < g->R; r++)
+        if (hs[n + 3 * r] || hs[n + 3 * r + 2]) hot[g->elig[r]] = 1;
+    free(hs);
+    dom = dominators(g);
+    in_s = (uint8_t *)malloc(n ? n : 1);
+    for (v = 0; v < n; v++) {
+        int64_t h = 0, inp = 0;
+        for (w = 0; w < n; w++)
+            if (dom[(size_t)v * n + w] && hot[w]) h += g->size[w];
+        /* G.inps(T.des(v)): sources of edges entering T.des(v), each once */
+        for (w = 0; w < n; w++) in_s[w] = 0;
+        for (k = 0; k < g->ne; k++) {
+            int32_t a = g->src[k], b = g->dst[k];
+            if (dom[(size_t)v * n + b] && !dom[(size_t)v * n + a]) in_s[a] = 1;
+        }
+        for (w = 0; w < n; w++)
+            if (in_s[w] && !hot[w]) inp += g->size[w];
+        heat[v] = h;
+        score[v] = (1.0 - 1.0 / (double)nsplit) * (double)h - (double)inp;
+    }
+    free(dom); free(in_s);
+    return status;
 }
 
 /* K candidates back to back: perms is K x NT row-major, decs K x R. */

@@ -141,3 +141,89 @@ def defn_eval(n, edges, size, outputs, elig, U, dec, perm):
             sz[v] = 0 if k == 1 else size[elig[r]]
     pk, _ = interval_peak(order, te, sz, set(outputs))
     return 0, pk
+
+
+# ---- NEXT-3: hot-spots, dominators, heat / score (written from the text) ----
+
+def defn_hotspots(n, edges, size, outputs, elig, U, dec, perm):
+    """H = union of A_i over the steps i with M_i = M_peak, A_i = the tensors
+    with S_u < i <= F_u (P:420-424, reading P1), on the transformed graph;
+    then over the original nodes: a live clone or Load of t_r stands for t_r,
+    a Store does not count (reading H1).  -> set of original nodes, or None
+    if the schedule violates a dependency."""
+    active, te = transformed(n, edges, elig, U, dec)
+    pos = {v: i for i, v in enumerate(perm)}
+    if any(pos[u] >= pos[v] for u, v in te):
+        return None
+    order = [v for v in perm if v in active]
+    sz = {}
+    for v in order:
+        if v < n:
+            sz[v] = size[v]
+        else:
+            r, k = divmod(v - n, 3)
+            sz[v] = 0 if k == 1 else size[elig[r]]
+    S, F = intervals(order, te, set(outputs))
+    curve = [sum(sz[u] for u in order if S[u] < i <= F[u]) for i in range(1, len(order) + 1)]
+    peak = max(curve)
+    Hs = set()
+    for i in range(1, len(order) + 1):
+        if curve[i - 1] == peak:
+            Hs |= {u for u in order if S[u] < i <= F[u]}
+    H = {v for v in Hs if v < n}
+    for v in Hs:
+        if v >= n:
+            r, k = divmod(v - n, 3)
+            if k != 1:
+                H.add(elig[r])
+    return H
+
+
+def brute_dominators(n, edges):
+    """dom[u] = set of nodes v that u dominates: u == v, or v cannot be reached
+    from any source (node without predecessors) once u is removed."""
+    pre = {v: set() for v in range(n)}
+    suc = {v: set() for v in range(n)}
+    for u, v in edges:
+        pre[v].add(u)
+        suc[u].add(v)
+    sources = [v for v in range(n) if not pre[v]]
+    dom = {}
+    for u in range(n):
+        seen = set()
+        stack = [s for s in sources if s != u]
+        while stack:
+            x = stack.pop()
+            if x in seen:
+                continue
+            seen.add(x)
+            stack.extend(y for y in suc[x] if y != u)
+        dom[u] = {v for v in range(n) if v == u or v not in seen}
+    return dom
+
+
+def brute_idom(n, edges):
+    dom = brute_dominators(n, edges)
+    idom = []
+    for v in range(n):
+        strict = [u for u in range(n) if u != v and v in dom[u]]
+        # the strict dominator dominated by every other strict dominator
+        best = [u for u in strict if all(u in dom[w] for w in strict)]
+        idom.append(best[0] if best else -1)
+    return idom
+
+
+def defn_heat_score(n, edges, size, H, nsplit):
+    """Eq. 3 / Eq. 4 literally: heat(v) = sum |w| over w in H and T.des(v);
+    score(v) = (1 - 1/nsplit) heat(v) - sum |u| over the inputs of T.des(v)
+    (nodes outside it with an edge into it) that are not in H."""
+    dom = brute_dominators(n, edges)
+    heat, score = [], []
+    for v in range(n):
+        des = dom[v]
+        h = sum(size[w] for w in des if w in H)
+        inps = {u for (u, w) in edges if w in des and u not in des}
+        inp = sum(size[u] for u in inps if u not in H)
+        heat.append(h)
+        score.append((1.0 - 1.0 / nsplit) * float(h) - float(inp))
+    return heat, score
