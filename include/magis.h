@@ -230,6 +230,40 @@ int magis_eval_windows(const magis_base* b, int64_t K, const int32_t* d_wstart, 
                        double* d_latency, void* cuda_stream);
 
 /*
+ * Memory hot-spots and F-Trans heat / score of K candidate schedules
+ * (Eq. 3-4), for the schedules
+ * the search selects (one CTA per candidate; not the batch hot loop).
+ * H = the tensors live at some step where M_i = M_peak; over the original
+ * graph a live clone or Load of t_r stands for t_r and a Store does not count
+ * (reading H1).  T = the dominator tree of G, sources under a
+ * virtual root (built by magis_graph_load; see magis_graph_idom).
+ *   heat(v)  = sum of |w| over w in H and T.des(v)                      (Eq. 3)
+ *   score(v) = (1 - 1/nsplit) heat(v) - sum of |u| over the inputs of
+ *              T.des(v) not in H                                         (Eq. 4)
+ * d_perm [K x n_total] int32, d_dec [K x R] u8 (may be NULL if R == 0):
+ *             device memory, as magis_eval_schedules.
+ * nsplit      n of Eq. 4 (>= 1; the paper uses 2).
+ * d_status [K] u8, d_peak [K] int64 out: as magis_eval_schedules.
+ * d_hot [K x n_nodes] u8 out: 1 iff original tensor v is a hot-spot.
+ * d_heat [K x n_nodes] int64 out (bytes) or NULL; d_score [K x n_nodes] f64
+ *             out or NULL.  Invalid candidates: status != 0, peak -1, rows 0.
+ * Asynchronous on the stream; the workspace is library-owned (allocated on
+ * first use, freed with the graph).
+ * Errors: MAGIS_E_INVAL, MAGIS_E_NOMEM, MAGIS_E_CUDA.
+ */
+int magis_hotspots(magis_graph* g, int64_t K, const int32_t* d_perm, const uint8_t* d_dec, int32_t nsplit,
+                   uint8_t* d_status, int64_t* d_peak, uint8_t* d_hot, int64_t* d_heat, double* d_score,
+                   void* cuda_stream);
+
+/*
+ * Immediate dominators of the original graph: idom[v] = the
+ * nearest strict dominator of v, or -1 if only the sources' virtual root
+ * dominates it.  idom: host array [n_nodes], caller-owned.
+ * Errors: MAGIS_E_INVAL.
+ */
+int magis_graph_idom(const magis_graph* g, int32_t* idom);
+
+/*
  * Pareto front of (peak, latency) over valid points,
  * plus the BetterThan-best point of Alg. 3 in both optimisation
  * modes.  a dominates b iff a.peak <= b.peak, a.lat <= b.lat and

@@ -149,21 +149,68 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
         }
     }
     // --- acyclicity --------------------------------------------
+    std::vector<int32_t> topo;
+    topo.reserve(n);
     {
         std::vector<int32_t> indeg(n), stack;
         for (int32_t v = 0; v < n; v++) {
             indeg[v] = pred_ptr[v + 1] - pred_ptr[v];
             if (!indeg[v]) stack.push_back(v);
         }
-        int32_t seen = 0;
         while (!stack.empty()) {
             int32_t u = stack.back();
             stack.pop_back();
-            seen++;
+            topo.push_back(u);
             for (int32_t e = succ_ptr[u]; e < succ_ptr[u + 1]; e++)
                 if (--indeg[succ[e]] == 0) stack.push_back(succ[e]);
         }
-        if (seen != n) return set_error(MAGIS_E_CYCLE, "the graph has a cycle");
+        if ((int32_t)topo.size() != n) return set_error(MAGIS_E_CYCLE, "the graph has a cycle");
+    }
+    // --- dominator tree T(G) (for NEXT-3 heat / score) ----------
+    // Sources hang off a virtual root (-1).  On a DAG in topological order the
+    // immediate dominator of v is the nearest common dominator-tree ancestor
+    // of its predecessors; tin / tout number the tree in preorder, so the
+    // descendants of v are the preorder range [tin(v), tout(v)).
+    std::vector<int32_t> idom(n, -1), dtin(n), dtout(n);
+    {
+        std::vector<int32_t> ti(n);
+        for (int32_t i = 0; i < n; i++) ti[topo[i]] = i;
+        for (int32_t v : topo) {
+            int32_t cur = -2;                       // -2: no predecessor seen yet
+            for (int32_t e = pred_ptr[v]; e < pred_ptr[v + 1]; e++) {
+                int32_t a = pred[e];
+                if (cur == -2) { cur = a; continue; }
+                int32_t b = cur;
+                while (a != b && a >= 0 && b >= 0) {
+                    if (ti[a] > ti[b]) a = idom[a]; else b = idom[b];
+                }
+                cur = (a == b) ? a : -1;
+            }
+            idom[v] = cur == -2 ? -1 : cur;
+        }
+        std::vector<int32_t> cptr(n + 2, 0), cidx(n);
+        for (int32_t v = 0; v < n; v++) cptr[idom[v] + 2]++;
+        for (int32_t i = 0; i <= n; i++) cptr[i + 1] += cptr[i];
+        {
+            std::vector<int32_t> fill(cptr.begin(), cptr.end() - 1);
+            for (int32_t v = 0; v < n; v++) cidx[fill[idom[v] + 1]++] = v;
+        }
+        // iterative preorder from the virtual root (children slot 0)
+        int32_t t = 0;
+        std::vector<std::pair<int32_t, int32_t>> st;   // (node, next child index)
+        st.push_back({-1, cptr[0]});
+        while (!st.empty()) {
+            auto& top = st.back();
+            const int32_t u = top.first;
+            if (top.second < cptr[u + 2]) {
+                const int32_t c = cidx[top.second++];
+                dtin[c] = t++;
+                st.push_back({c, cptr[c + 1]});
+            } else {
+                if (u >= 0) dtout[u] = t;
+                st.pop_back();
+            }
+        }
     }
     // --- eligible tensors (reading P6) -------------------------------------
     std::vector<int32_t> r_of(n, -1);
@@ -293,6 +340,8 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     size_t o_s = add(succ.data(), succ.size() * 4);
     size_t o_pp = add(pred_ptr.data(), pred_ptr.size() * 4);
     size_t o_p = add(pred.data(), pred.size() * 4);
+    size_t o_dtin = add(dtin.data(), dtin.size() * 4);
+    size_t o_dtout = add(dtout.data(), dtout.size() * 4);
     g->blob_bytes = off;
     cudaError_t e = cudaMalloc(&g->blob, off);
     if (e != cudaSuccess) {
@@ -331,6 +380,11 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     dg.tcost = (const double*)(b + o_tcost);
     dg.rflag = (const uint8_t*)(b + o_rflag);
     dg.base_cost = base_cost;
+    dg.dtin = (const int32_t*)(b + o_dtin);
+    dg.dtout = (const int32_t*)(b + o_dtout);
+    dg.pred_ptr = (const int32_t*)(b + o_pp);
+    dg.pred = (const int32_t*)(b + o_p);
+    g->idom = idom;
     g->gen.succ_ptr = (const int32_t*)(b + o_sp);
     g->gen.succ = (const int32_t*)(b + o_s);
     g->gen.pred_ptr = (const int32_t*)(b + o_pp);
@@ -439,6 +493,7 @@ extern "C" int magis_graph_free(magis_graph* g) {
     if (g->gws) cudaFree(g->gws);
     if (g->blob2) cudaFree(g->blob2);
     if (g->ovf2) cudaFree(g->ovf2);
+    if (g->hs_ws) cudaFree(g->hs_ws);
     if (g->afg2) cudaFree(g->afg2);
     if (g->gen_scratch) cudaFree(g->gen_scratch);
     for (int i = 0; i < 2; i++) {
@@ -488,6 +543,46 @@ extern "C" int magis_eval_schedules(const magis_graph* g, int64_t K, const int32
         cudaGetLastError();
         return set_error(MAGIS_E_CUDA, std::string("eval launch: ") + cudaGetErrorString(e));
     }
+    return MAGIS_SUCCESS;
+}
+
+// NEXT-3: hot-spots and heat / score of selected candidates.
+extern "C" int magis_hotspots(magis_graph* g, int64_t K, const int32_t* d_perm, const uint8_t* d_dec,
+                              int32_t nsplit, uint8_t* d_status, int64_t* d_peak, uint8_t* d_hot,
+                              int64_t* d_heat, double* d_score, void* cuda_stream) {
+    clear_error();
+    if (!g) return set_error(MAGIS_E_INVAL, "graph is NULL");
+    if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
+    if (nsplit < 1) return set_error(MAGIS_E_INVAL, "nsplit < 1");
+    if (K == 0) return MAGIS_SUCCESS;
+    if (!d_perm || !d_status || !d_peak || !d_hot) return set_error(MAGIS_E_INVAL, "null device pointer");
+    if (g->dev.R > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R > 0");
+    DeviceGuard guard(g->device);
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device);
+    const int grid = std::max(1, sms) * 2;
+    const size_t need = hotspot_ws_per_cta(g->dev) * (size_t)grid;
+    if (g->hs_ws_bytes < need) {
+        if (g->hs_ws) { cudaDeviceSynchronize(); cudaFree(g->hs_ws); g->hs_ws = nullptr; g->hs_ws_bytes = 0; }
+        if (cudaMalloc(&g->hs_ws, need) != cudaSuccess) {
+            cudaGetLastError();
+            return set_error(MAGIS_E_NOMEM, "cudaMalloc hot-spot workspace failed");
+        }
+        g->hs_ws_bytes = need;
+    }
+    cudaError_t e = hotspot_launch(g->dev, grid, g->hs_ws, K, d_perm, d_dec, nsplit, d_status, d_peak, d_hot, d_heat,
+                                   d_score, (cudaStream_t)cuda_stream);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return set_error(MAGIS_E_CUDA, std::string("hotspot launch: ") + cudaGetErrorString(e));
+    }
+    return MAGIS_SUCCESS;
+}
+
+extern "C" int magis_graph_idom(const magis_graph* g, int32_t* idom) {
+    clear_error();
+    if (!g || !idom) return set_error(MAGIS_E_INVAL, "null argument");
+    for (size_t v = 0; v < g->idom.size(); v++) idom[v] = g->idom[v];
     return MAGIS_SUCCESS;
 }
 

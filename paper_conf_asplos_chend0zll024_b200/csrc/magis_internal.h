@@ -51,6 +51,10 @@ struct DevGraph {
     const double* tcost;       // [R] cost(t_r)
     const uint8_t* rflag;      // [R]
     double base_cost;          // sum of cost over original nodes
+    const int32_t* dtin;       // [n] dominator-tree preorder index (NEXT-3)
+    const int32_t* dtout;      // [n] end of the node's preorder range
+    const int32_t* pred_ptr;   // [n+1] predecessors in G (deduplicated)
+    const int32_t* pred;
 };
 
 // Variant-2 plan (magis_eval2.cu): graph as per-thread streams in shared
@@ -183,6 +187,11 @@ cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, v
                          int64_t* peak, double* lat, cudaStream_t stream);
 cudaError_t eval2_occupancy(const Plan2& pl, int* blocks_per_sm);
 
+size_t hotspot_ws_per_cta(const DevGraph& g);
+cudaError_t hotspot_launch(const DevGraph& g, int grid, void* ws, int64_t K, const int32_t* perm, const uint8_t* dec,
+                           int32_t nsplit, uint8_t* status, int64_t* peak, uint8_t* hot, int64_t* heat,
+                           double* score, cudaStream_t stream);
+
 cudaError_t eval_configure(const DevGraph& g, int device, EvalConfig* cfg);
 cudaError_t eval_launch(const DevGraph& g, const EvalConfig& cfg, void* gws, int64_t K,
                         const int32_t* perm, const uint8_t* dec, uint8_t* status,
@@ -220,6 +229,9 @@ struct magis_graph {
     size_t gws_bytes = 0;
     int64_t n_edges = 0;
     int64_t n_super_edges = 0;
+    std::vector<int32_t> idom;     // dominator tree of G (host copy)
+    void* hs_ws = nullptr;         // hot-spot query workspace (lazily allocated)
+    size_t hs_ws_bytes = 0;
     // host-buffer (end-to-end) path: lazily allocated staging
     cudaStream_t aux = nullptr;
     int64_t stage_K = 0;

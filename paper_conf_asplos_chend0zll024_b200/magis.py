@@ -24,7 +24,8 @@ ST_NOT_PERM, ST_EDGE, ST_BAD_DEC = 1, 2, 4
 EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magis_eval_schedules",
            "magis_eval_schedules_host", "magis_pareto_workspace_size", "magis_pareto_merge",
            "magis_last_error", "magis_abi_version", "magis_device_supported", "magis_generate_candidates",
-           "magis_base_create", "magis_base_info", "magis_base_free", "magis_eval_windows"]
+           "magis_base_create", "magis_base_info", "magis_base_free", "magis_eval_windows", "magis_hotspots",
+           "magis_graph_idom"]
 
 
 class MagisError(RuntimeError):
@@ -97,6 +98,10 @@ def lib() -> ctypes.CDLL:
     L.magis_base_free.restype = ctypes.c_int
     L.magis_eval_windows.argtypes = [P, i64, P, P, P, i32, P, P, P, P]
     L.magis_eval_windows.restype = ctypes.c_int
+    L.magis_hotspots.argtypes = [P, i64, P, P, i32, P, P, P, P, P, P]
+    L.magis_hotspots.restype = ctypes.c_int
+    L.magis_graph_idom.argtypes = [P, P]
+    L.magis_graph_idom.restype = ctypes.c_int
     _lib = L
     return L
 
@@ -207,6 +212,35 @@ class Graph:
         _check(self._L.magis_generate_candidates(self._h, ctypes.byref(spec), int(id0), int(K), _tptr(perm),
                                                  _tptr(dec), _stream_ptr(stream)))
         return perm, dec
+
+    def hotspots(self, perm, dec=None, nsplit: int = 2, heat: bool = True, score: bool = True, stream=None):
+        """Memory hot-spots and heat / score (magis_hotspots, NEXT-3) of the
+        candidates in perm (cuda int32 [K, n_total]) / dec (cuda uint8 [K, R]).
+        Returns (status [K], peak [K], hot uint8 [K, n], heat int64 [K, n] or
+        None, score float64 [K, n] or None) device tensors."""
+        import torch
+        K = int(perm.shape[0])
+        assert perm.dtype == torch.int32 and perm.is_cuda and perm.is_contiguous()
+        assert perm.shape[1] == self.n_total
+        if self.R:
+            assert dec is not None and dec.dtype == torch.uint8 and dec.is_contiguous()
+            assert dec.shape[0] == K and dec.shape[1] == self.R
+        dev = perm.device
+        st = torch.empty(K, dtype=torch.uint8, device=dev)
+        pk = torch.empty(K, dtype=torch.int64, device=dev)
+        hot = torch.empty((K, self.n), dtype=torch.uint8, device=dev)
+        ht = torch.empty((K, self.n), dtype=torch.int64, device=dev) if heat else None
+        sc = torch.empty((K, self.n), dtype=torch.float64, device=dev) if score else None
+        _check(self._L.magis_hotspots(self._h, K, _tptr(perm), _tptr(dec) if self.R else None, int(nsplit),
+                                      _tptr(st), _tptr(pk), _tptr(hot), _tptr(ht) if heat else None,
+                                      _tptr(sc) if score else None, _stream_ptr(stream)))
+        return st, pk, hot, ht, sc
+
+    def idom(self) -> np.ndarray:
+        """Immediate dominators of the original graph (-1: virtual root)."""
+        out = np.empty(max(self.n, 1), np.int32)
+        _check(self._L.magis_graph_idom(self._h, _np_ptr(out)))
+        return out[:self.n]
 
     def eval_schedules_host(self, perm: np.ndarray, dec: Optional[np.ndarray] = None, out=None,
                             stream=None):
