@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU-baseline wall time")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-int32", action="store_true", help="e2e with int32 host schedules instead of uint16")
     ap.add_argument("--windows", action="store_true",
                     help="local-move candidates scored by windowed delta evaluation (NEXT-1); default config c5, K=1M")
     return ap.parse_args()
@@ -311,20 +312,26 @@ def main():
         hlt = np.empty(K, np.float64)
         out_pinned = (torch.empty(K, dtype=torch.uint8).pin_memory(), torch.empty(K, dtype=torch.int64).pin_memory(),
                       torch.empty(K, dtype=torch.float64).pin_memory())
-        g.eval_schedules_host(Ph_t, Dh_t, out=out_pinned)     # warm (allocates staging once)
+        # schedules cross PCIe in the compact uint16 wire format when the
+        # super-graph has < 65536 nodes (magis_eval_schedules_host_u16)
+        u16 = NT <= 65535 and not args.e2e_int32
+        Ph_w = torch.from_numpy(Ph.astype(np.uint16)).pin_memory() if u16 else Ph_t
+        g.eval_schedules_host(Ph_w, Dh_t, out=out_pinned)     # warm (allocates staging once)
         if world > 1:
             dist.barrier()
         n_e2e = max(1, min(args.steps, 5))
         t0 = time.perf_counter()
         for _ in range(n_e2e):
-            g.eval_schedules_host(Ph_t, Dh_t, out=out_pinned)
+            g.eval_schedules_host(Ph_w, Dh_t, out=out_pinned)
         e2e_s = (time.perf_counter() - t0) / n_e2e
         te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        api = ("magis_eval_schedules_host_u16 (uint16 schedules" if u16 else
+               "magis_eval_schedules_host (int32 schedules")
         e2e = {"value": round(world * K / te.item(), 1), "unit": UNIT,
-               "h2d_bytes_per_step": int(K * NT * 4 + K * R), "d2h_bytes_per_step": int(K * 17),
-               "api": "magis_eval_schedules_host (pinned host buffers, chunked double-buffered copies)",
+               "h2d_bytes_per_step": int(K * NT * (2 if u16 else 4) + K * R), "d2h_bytes_per_step": int(K * 17),
+               "api": api + ", pinned host buffers, chunked double-buffered copies)",
                "s_per_step": round(te.item(), 5)}
         ok_same = bool((out_pinned[1].numpy() == pk.cpu().numpy()).all())
         e2e["matches_device_path"] = ok_same

@@ -167,6 +167,17 @@ int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_t* h_perm,
                               double* h_latency, void* cuda_stream);
 
 /*
+ * As magis_eval_schedules_host with the schedules in the compact wire format:
+ * h_perm [K x n_total] uint16 host memory (n_total <= 65535).  Half the
+ * host->device bytes; the library widens each chunk on the device before
+ * evaluating it.  Errors as magis_eval_schedules_host, plus
+ * MAGIS_E_UNSUPPORTED if n_total > 65535.
+ */
+int magis_eval_schedules_host_u16(magis_graph* g, int64_t K, const uint16_t* h_perm,
+                                  const uint8_t* h_dec, uint8_t* h_status, int64_t* h_peak,
+                                  double* h_latency, void* cuda_stream);
+
+/*
  * Seeded candidate generation on the device.  Candidate k
  * (global id id0 + i) depends only on (spec->seed, k), so ranks generate
  * their shards independently.  The recipe stands in for MAGIS's rule

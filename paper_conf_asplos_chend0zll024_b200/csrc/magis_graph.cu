@@ -587,10 +587,16 @@ extern "C" int magis_graph_idom(const magis_graph* g, int32_t* idom) {
 }
 
 // End-to-end host path: chunked, double-buffered H2D -> eval -> D2H.
-extern "C" int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_t* h_perm,
-                                         const uint8_t* h_dec, uint8_t* h_status,
-                                         int64_t* h_peak, double* h_latency,
-                                         void* cuda_stream) {
+namespace {
+
+__global__ void widen_u16(const uint16_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dst[i] = (int32_t)src[i];
+}
+
+// pb = bytes per perm element on the host (4: int32, 2: uint16, widened on the device)
+int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8_t* h_dec, uint8_t* h_status,
+              int64_t* h_peak, double* h_latency, void* cuda_stream) {
     clear_error();
     if (!g) return set_error(MAGIS_E_INVAL, "graph is NULL");
     if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
@@ -599,19 +605,21 @@ extern "C" int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_
         return set_error(MAGIS_E_INVAL, "null host pointer");
     const int32_t R = g->dev.R, NT = g->dev.NT;
     if (R > 0 && !h_dec) return set_error(MAGIS_E_INVAL, "h_dec is NULL but R > 0");
+    if (pb == 2 && NT > 65535) return set_error(MAGIS_E_UNSUPPORTED, "uint16 schedules need n_total <= 65535");
     DeviceGuard guard(g->device);
     cudaStream_t s0 = (cudaStream_t)cuda_stream;
-    // chunk of ~64 MiB of perms
+    // chunk of ~64 MiB of int32 perms
     int64_t chunk = std::max<int64_t>(1, (64ll << 20) / ((int64_t)NT * 4));
     chunk = std::min<int64_t>(chunk, K);
     const size_t perm_b = align_up((size_t)chunk * NT * 4, 256);
+    const size_t narrow_b = align_up((size_t)chunk * NT * 2, 256);
     const size_t dec_b = align_up((size_t)chunk * std::max(R, 1), 256);
     const size_t out_b = align_up((size_t)chunk * 17, 256);
     if (g->stage_K < chunk) {
         for (int i = 0; i < 2; i++) {
             if (g->stage[i]) cudaFree(g->stage[i]);
             g->stage[i] = nullptr;
-            CK(cudaMalloc(&g->stage[i], perm_b + dec_b + out_b + 256));
+            CK(cudaMalloc(&g->stage[i], perm_b + narrow_b + dec_b + out_b + 256));
             if (!g->ev_h2d[i]) CK(cudaEventCreateWithFlags(&g->ev_h2d[i], cudaEventDisableTiming));
             if (!g->ev_done[i]) CK(cudaEventCreateWithFlags(&g->ev_done[i], cudaEventDisableTiming));
         }
@@ -625,16 +633,24 @@ extern "C" int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_
         int64_t k0 = c * chunk, kc = std::min(chunk, K - k0);
         char* base = (char*)g->stage[b];
         int32_t* dp = (int32_t*)base;
-        uint8_t* dd = (uint8_t*)(base + perm_b);
-        int64_t* dpk = (int64_t*)(base + perm_b + dec_b);
-        double* dlt = (double*)(base + perm_b + dec_b + align_up((size_t)chunk * 8, 64));
-        uint8_t* dst = (uint8_t*)(base + perm_b + dec_b + 2 * align_up((size_t)chunk * 8, 64));
+        uint16_t* dn = (uint16_t*)(base + perm_b);
+        uint8_t* dd = (uint8_t*)(base + perm_b + narrow_b);
+        char* ob = base + perm_b + narrow_b + dec_b;
+        int64_t* dpk = (int64_t*)ob;
+        double* dlt = (double*)(ob + align_up((size_t)chunk * 8, 64));
+        uint8_t* dst = (uint8_t*)(ob + 2 * align_up((size_t)chunk * 8, 64));
         // buffer b is free once the D2H of chunk c-2 finished
         if (c >= 2) CK(cudaStreamWaitEvent(g->aux, g->ev_done[b], 0));
-        CK(cudaMemcpyAsync(dp, h_perm + k0 * NT, (size_t)kc * NT * 4, cudaMemcpyHostToDevice, g->aux));
+        const char* hp = (const char*)h_perm + (size_t)k0 * NT * pb;
+        CK(cudaMemcpyAsync(pb == 4 ? (void*)dp : (void*)dn, hp, (size_t)kc * NT * pb, cudaMemcpyHostToDevice, g->aux));
         if (R > 0) CK(cudaMemcpyAsync(dd, h_dec + k0 * R, (size_t)kc * R, cudaMemcpyHostToDevice, g->aux));
         CK(cudaEventRecord(g->ev_h2d[b], g->aux));
         CK(cudaStreamWaitEvent(s0, g->ev_h2d[b], 0));
+        if (pb == 2) {
+            const int64_t ne = kc * (int64_t)NT;
+            const int blocks = (int)std::min<int64_t>((ne + 255) / 256, 4096);
+            widen_u16<<<blocks, 256, 0, s0>>>(dn, dp, ne);
+        }
         cudaError_t e = dispatch_eval(g, kc, dp, R > 0 ? dd : nullptr, dst, dpk, dlt, s0);
         if (e != cudaSuccess) {
             cudaGetLastError();
@@ -647,6 +663,22 @@ extern "C" int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_
     }
     CK(cudaStreamSynchronize(s0));
     return MAGIS_SUCCESS;
+}
+
+}  // namespace
+
+extern "C" int magis_eval_schedules_host(magis_graph* g, int64_t K, const int32_t* h_perm,
+                                         const uint8_t* h_dec, uint8_t* h_status,
+                                         int64_t* h_peak, double* h_latency,
+                                         void* cuda_stream) {
+    return host_path(g, K, h_perm, 4, h_dec, h_status, h_peak, h_latency, cuda_stream);
+}
+
+extern "C" int magis_eval_schedules_host_u16(magis_graph* g, int64_t K, const uint16_t* h_perm,
+                                             const uint8_t* h_dec, uint8_t* h_status,
+                                             int64_t* h_peak, double* h_latency,
+                                             void* cuda_stream) {
+    return host_path(g, K, h_perm, 2, h_dec, h_status, h_peak, h_latency, cuda_stream);
 }
 
 extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* spec, uint64_t id0, int64_t K,

@@ -25,7 +25,7 @@ EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magi
            "magis_eval_schedules_host", "magis_pareto_workspace_size", "magis_pareto_merge",
            "magis_last_error", "magis_abi_version", "magis_device_supported", "magis_generate_candidates",
            "magis_base_create", "magis_base_info", "magis_base_free", "magis_eval_windows", "magis_hotspots",
-           "magis_graph_idom"]
+           "magis_graph_idom", "magis_eval_schedules_host_u16"]
 
 
 class MagisError(RuntimeError):
@@ -79,6 +79,8 @@ def lib() -> ctypes.CDLL:
     L.magis_eval_schedules.restype = ctypes.c_int
     L.magis_eval_schedules_host.argtypes = [P, i64, P, P, P, P, P, P]
     L.magis_eval_schedules_host.restype = ctypes.c_int
+    L.magis_eval_schedules_host_u16.argtypes = [P, i64, P, P, P, P, P, P]
+    L.magis_eval_schedules_host_u16.restype = ctypes.c_int
     L.magis_pareto_workspace_size.argtypes = [i64]
     L.magis_pareto_workspace_size.restype = i64
     L.magis_pareto_merge.argtypes = [i64, P, P, P, P, i64, i64, P, P, P, P, i64, d, P, P, i64, P]
@@ -244,14 +246,19 @@ class Graph:
 
     def eval_schedules_host(self, perm: np.ndarray, dec: Optional[np.ndarray] = None, out=None,
                             stream=None):
-        """End-to-end call with host buffers (pinned numpy views or torch CPU tensors)."""
+        """End-to-end call with host buffers (pinned numpy views or torch CPU
+        tensors).  uint16 schedules use the compact wire format
+        (magis_eval_schedules_host_u16), anything else is taken as int32."""
         import torch
 
         def as_np(x, dt):
             if isinstance(x, torch.Tensor):
                 return x.numpy()
             return np.ascontiguousarray(x, dt)
-        p = as_np(perm, np.int32)
+        p = as_np(perm, None)
+        u16 = p.dtype == np.uint16
+        if not u16:
+            p = np.ascontiguousarray(p, np.int32)
         K = p.shape[0]
         assert p.shape[1] == self.n_total
         dd = as_np(dec, np.uint8) if (self.R and dec is not None) else None
@@ -261,8 +268,8 @@ class Graph:
             lt = np.empty(K, np.float64)
         else:
             st, pk, lt = (as_np(o, None) for o in out)
-        _check(self._L.magis_eval_schedules_host(self._h, K, _np_ptr(p), _np_ptr(dd), _np_ptr(st),
-                                                 _np_ptr(pk), _np_ptr(lt), _stream_ptr(stream)))
+        fn = self._L.magis_eval_schedules_host_u16 if u16 else self._L.magis_eval_schedules_host
+        _check(fn(self._h, K, _np_ptr(p), _np_ptr(dd), _np_ptr(st), _np_ptr(pk), _np_ptr(lt), _stream_ptr(stream)))
         return st, pk, lt
 
 

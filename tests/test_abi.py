@@ -18,7 +18,7 @@ HEADER = os.path.join(ROOT, "include", "magis.h")
 def declared():
     src = open(HEADER).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
-    return sorted(set(re.findall(r"\b(magis_[a-z_]+)\s*\(", src)))
+    return sorted(set(re.findall(r"\b(magis_[a-z_0-9]+)\s*\(", src)))
 
 
 @pytest.fixture(scope="module")

@@ -223,6 +223,13 @@ def test_host_path_matches_device_path():
     host = g.eval_schedules_host(Pp, Dp)
     for a, b in zip(dev, host):
         np.testing.assert_array_equal(a, b)
+    # compact uint16 wire format (magis_eval_schedules_host_u16), pageable and pinned
+    host16 = g.eval_schedules_host(P.astype(np.uint16), D)
+    for a, b in zip(dev, host16):
+        np.testing.assert_array_equal(a, b)
+    host16p = g.eval_schedules_host(torch.from_numpy(P.astype(np.uint16)).pin_memory(), Dp)
+    for a, b in zip(dev, host16p):
+        np.testing.assert_array_equal(a, b)
 
 
 def test_k_zero_and_one_and_ragged(variant):
