@@ -318,6 +318,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const double* cost_s = (const double*)(sb + pl.off_cost);
     const uint2* ninfo = (const uint2*)(sb + pl.off_ninfo);
     const uint16_t* lul = (const uint16_t*)(sb + pl.off_lul);
+    const uint32_t* urow = (const uint32_t*)(sb + pl.off_urow);     // [R] U_r offset | |U_r| << 16
+    const uint16_t* ubs = (const uint16_t*)(sb + pl.off_ubs);       // [nU] late users, by r
+    const uint16_t* utr = (const uint16_t*)(sb + pl.off_utr);       // [R] t_r
     uint16_t* pos = (uint16_t*)(sm + pl.off_pos);
     uint16_t* last = (uint16_t*)(sm + pl.off_last);
     uint2* AF = MODE == 2 ? (uint2*)(afg + (size_t)blockIdx.x * pl.af_bytes)   // [P][Sl] (alloc, free)
@@ -411,7 +414,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const int cm = tid / TPC, tt = tid - cm * TPC;
     const int32_t lo = tt * L;
     const bool vec4 = (NT & 3) == 0;
-    constexpr int LR = LMAX <= 16 ? LMAX : 1;      // perm chunk kept in registers when short
+    // perm chunk kept in registers when short (32 steps only where the
+    // tables sit in shared memory and the register budget allows it)
+    constexpr int kRegL = MODE <= 1 ? 32 : 16;
+    constexpr int LR = LMAX <= kRegL ? LMAX : 1;
     int32_t pr[LR];
     // this thread's chunk of candidate cm of group grp_ (-1 past the end)
     auto load_chunk = [&](int64_t grp_) {
@@ -436,7 +442,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             if (j + 3 < LR) pr[j + 3] = v.w;
         }
     };
-    if constexpr (LMAX <= 16) {
+    if constexpr (LMAX <= kRegL) {
         if (ncta > 0) load_chunk(blockIdx.x);
     }
     for (int gi = 0; gi < ncta; gi++) {
@@ -467,7 +473,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         {
             int bad = 0;
             const bool vc = (vmask >> cm) & 1u;
-            if constexpr (LMAX <= 16) {
+            if constexpr (LMAX <= kRegL) {
 #pragma unroll
                 for (int j = 0; j < LMAX; j++) {
                     if (vc && j < L && lo + j < NT) {
@@ -518,39 +524,36 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         for (int q = tid; q < P * R; q += TM) {
             const int c = q / R, r = q - c * R;
             if (!((vmask >> c) & 1u)) continue;
-            const int32_t u0 = __ldg(g.U_ptr + r), u1 = __ldg(g.U_ptr + r + 1);
+            const uint32_t ur = urow[r];                       // (U offset, |U_r|) packed
+            const uint32_t u0 = ur & 0xffffu, u1 = u0 + (ur >> 16);
+            const uint8_t d = dec_s[c * R + r];
+            uint32_t* em = evm + c * nwm;
+            uint16_t* pc_ = pos + c;
 #pragma unroll
-            for (int cc = 0; cc < P; cc++) {
-                if (cc != c) continue;
-                const uint8_t d = dec_s[cc * R + r];
-                uint32_t* em = evm + cc * nwm;
-#pragma unroll
-                for (int o = 0; o < 3; o++) {
-                    const int32_t id = n + 3 * r + o;
-                    const uint32_t p = pos[id * P + cc];
-                    if (p == 0) {
-                        atomicOr(&cl.flags[cc], MAGIS_ST_NOT_PERM);
-                        continue;
-                    }
-                    const bool act = (o == 0) ? (d == 1) : (d == 2);
-                    const uint32_t st = p - 1;
-                    if (!act) {
-                        AF[cc * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
-                        pos[id * P + cc] = 0;
-                    } else if (o > 0) {
-                        atomicOr(em + (st >> 5), 1u << (st & 31));
-                    }
+            for (int o = 0; o < 3; o++) {
+                const int32_t id = n + 3 * r + o;
+                const uint32_t p = pc_[id * P];
+                if (p == 0) {
+                    atomicOr(&cl.flags[c], MAGIS_ST_NOT_PERM);
+                    continue;
                 }
-                if (d == 2) {
-                    const uint32_t pt_ = pos[__ldg(g.elig + r) * P + cc];
-                    if (pt_) atomicOr(em + ((pt_ - 1) >> 5), 1u << ((pt_ - 1) & 31));
+                const bool act = (o == 0) ? (d == 1) : (d == 2);
+                const uint32_t st = p - 1;
+                if (!act) {
+                    AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
+                    pc_[id * P] = 0;
+                } else if (o > 0) {
+                    atomicOr(em + (st >> 5), 1u << (st & 31));
                 }
-                for (int32_t j = u0; j < u1; j++) {
-                    const int32_t b = __ldg(g.U_idx + j);
-                    const uint32_t pb = pos[b * P + cc];
-                    pos[(NT + j) * P + cc] = (d == 0) ? (uint16_t)pb : (uint16_t)0;
-                    if (d == 2 && pb) atomicOr(em + ((pb - 1) >> 5), 1u << ((pb - 1) & 31));
-                }
+            }
+            if (d == 2) {
+                const uint32_t pt_ = pc_[(uint32_t)utr[r] * P];
+                if (pt_) atomicOr(em + ((pt_ - 1) >> 5), 1u << ((pt_ - 1) & 31));
+            }
+            for (uint32_t j = u0; j < u1; j++) {
+                const uint32_t pb = pc_[(uint32_t)ubs[j] * P];
+                pc_[(NT + j) * P] = (d == 0) ? (uint16_t)pb : (uint16_t)0;
+                if (d == 2 && pb) atomicOr(em + ((pb - 1) >> 5), 1u << ((pb - 1) & 31));
             }
         }
         bar_sync(kBarMain, TM);
@@ -695,7 +698,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             double cs1 = 0.0;
             int o = wpre + evx;
             const int o0 = o;
-#pragma unroll
+            constexpr int kUnroll5 = LR > 1 ? LMAX : 8;     // full unroll only with the chunk in registers
+#pragma unroll kUnroll5
             for (int j = 0; j < LMAX; j++) {
                 if (j < nst) {
                     const uint2 af = AF[cm * Sl + j * S + tt];     // alloc / free of the step (units)
@@ -703,7 +707,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     m1 = max(m1, s1);
                     s1 -= af.y;
                     if (mysw) {
-                        const int32_t v = LMAX <= 16 ? pr[j % LR]
+                        const int32_t v = LMAX <= kRegL ? pr[j % LR]
                                                      : __ldg(perm + (grp * P + cm) * (int64_t)NT + lo + j);
                         if ((mbits >> j) & 1ull) {
                             kout[o] = ((unsigned long long)(lo + j) << 32) | (uint32_t)v;
@@ -732,7 +736,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             }
         }
         // the next group's chunk is loaded while this group finishes
-        if constexpr (LMAX <= 16) {
+        if constexpr (LMAX <= kRegL) {
             if (gi + 1 < ncta) load_chunk(grp + gridDim.x);
         }
         bar_sync(kBarMain, TM);

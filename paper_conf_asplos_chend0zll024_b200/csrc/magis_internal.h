@@ -79,6 +79,9 @@ struct Plan2 {
     uint32_t off_ninfo;      // [n] uint2: x = (r + 1 if node is t_r, else 0) | |{r : node in U_r}| << 16,
                              //            y = offset of that r list in lul
     uint32_t off_lul;        // u16 r lists (late-user -> tensors), see off_ninfo
+    uint32_t off_urow;       // [R] u32: offset of U_r in ubs | |U_r| << 16
+    uint32_t off_ubs;        // [nU] u16 late users, grouped by r
+    uint32_t off_utr;        // [R] u16 t_r
     uint32_t off_pos, off_last, off_af, off_dec, off_end;
     uint32_t off_evm;        // [P][NW] swap-event step marks (bit per step)
     uint32_t off_sdec;       // [2][P][Rw] decisions handed to the latency warp

@@ -186,6 +186,9 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
     p.off_rtab = (uint32_t)o;  o = a16(o + (size_t)std::max(R, 1) * 16);
     p.off_ninfo = (uint32_t)o; o = a16(o + (size_t)n * 8);
     p.off_lul = (uint32_t)o;   o = a16(o + (size_t)std::max(nU, 1) * 2);
+    p.off_urow = (uint32_t)o;  o = a16(o + (size_t)std::max(R, 1) * 4);
+    p.off_ubs = (uint32_t)o;   o = a16(o + (size_t)std::max(nU, 1) * 2);
+    p.off_utr = (uint32_t)o;   o = a16(o + (size_t)std::max(R, 1) * 2);
     p.static_bytes = (uint32_t)o;
     // graph tables in shared memory (staged) or read from the global image
     // (L1/L2; the row reads stay coalesced); per-step slots in shared memory or
@@ -247,6 +250,18 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
         for (int32_t r = 0; r < R; r++) ninfo[2 * sg.elig[r]] |= (uint32_t)(r + 1);
         put(p.off_ninfo, ninfo.data(), ninfo.size() * 4);
         put(p.off_lul, lul.data(), lul.size() * 2);
+        std::vector<uint32_t> urow(std::max(R, 1), 0);
+        std::vector<uint16_t> ubs(std::max(nU, 1), 0), utr(std::max(R, 1), 0);
+        for (int32_t r = 0; r < R; r++) {
+            const int32_t u0 = sg.U_ptr[r], cnt = sg.U_ptr[r + 1] - u0;
+            if (cnt > 0xffff) return false;
+            urow[r] = (uint32_t)u0 | ((uint32_t)cnt << 16);
+            utr[r] = (uint16_t)sg.elig[r];
+            for (int32_t j = u0; j < u0 + cnt; j++) ubs[j] = (uint16_t)sg.U_idx[j];
+        }
+        put(p.off_urow, urow.data(), (size_t)R * 4);
+        put(p.off_ubs, ubs.data(), (size_t)nU * 2);
+        put(p.off_utr, utr.data(), (size_t)R * 2);
     }
     return true;
 }
