@@ -165,12 +165,9 @@ __device__ __forceinline__ void bulk_stage(void* smem_dst, const void* gsrc, uin
 // the owning warp (woff, added by the latency warp), plus the decisions.
 struct SlotHdr {
     long long k[4];
-    long long peak[4];      // in size units
-    double ctot[4];         // sum of compute costs (swapping candidates)
     int status[4];
     int nev[4];
     int swp[4];             // candidate swaps some tensor
-    double woff[WM];        // exclusive compute-cost prefix of each warp within its team
 };
 
 struct Ctl {
@@ -285,9 +282,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     __shared__ uint64_t mbar;
     __shared__ SlotHdr hdr[2];
     __shared__ Ctl ctl[2];                     // per group parity (reset one group ahead)
-    __shared__ long long agg_s[WM];
-    __shared__ long long agg_m[WM];
-    __shared__ double agg_c[WM];
+    __shared__ long long agg_s[2][WM];         // per slot: warp aggregates of the scan,
+    __shared__ long long agg_m[2][WM];         //   folded by the latency warps
+    __shared__ double agg_c[2][WM];
+    __shared__ double lwoff[4][WM];            // per latency warp: cost prefix of each team warp
     __shared__ int wcnt[WM];                   // event steps per warp chunk
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -366,6 +364,28 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const int st = h.status[c];
                 const uint8_t* dd = sdec + (size_t)(slot * P + c) * Rw;
                 double lat = __longlong_as_double(0x7ff0000000000000ll);
+                long long pk = 0;
+                double ctot = 0.0;
+                if (!st) {
+                    // fold the team's WT warp aggregates: (sum, max-prefix) -> peak,
+                    // cost sums -> per-warp exclusive prefix and the total
+                    const int a = c * WT + (lane < WT ? lane : 0);
+                    long long ss = lane < WT ? agg_s[slot][a] : 0;
+                    long long mm = lane < WT ? agg_m[slot][a] : kNegInf;
+                    double cc = lane < WT ? agg_c[slot][a] : 0.0;
+                    const double c0 = cc;
+#pragma unroll
+                    for (int o = 1; o < WT; o <<= 1) {
+                        const long long ps = __shfl_up_sync(0xffffffffu, ss, o);
+                        const long long pm = __shfl_up_sync(0xffffffffu, mm, o);
+                        const double pc = __shfl_up_sync(0xffffffffu, cc, o);
+                        if (lane >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
+                    }
+                    if (lane < WT) lwoff[c][lane] = cc - c0;
+                    pk = __shfl_sync(0xffffffffu, mm, WT - 1);
+                    ctot = __shfl_sync(0xffffffffu, cc, WT - 1);
+                    __syncwarp();
+                }
                 if (st) {
                 } else if (!h.swp[c]) {
                     double bl = 0.0;                 // no swap: base cost + re-computations
@@ -375,32 +395,29 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     for (int o = 16; o > 0; o >>= 1) bl += __shfl_xor_sync(0xffffffffu, bl, o);
                     lat = g.base_cost + bl;
                 } else {
-                    const double* woff = h.woff + c * WT;
+                    const double* woff = lwoff[c];
                     const int ne = h.nev[c];
                     if (ne <= cap) {
                         const size_t b0 = (size_t)(slot * P + c) * cap;
-                        lat = candidate_latency(evk_s + b0, evc_s + b0, evi_s + b0, ne, woff, dd, endb, wt, h.ctot[c],
+                        lat = candidate_latency(evk_s + b0, evc_s + b0, evi_s + b0, ne, woff, dd, endb, wt, ctot,
                                                 lane);
                     } else {
                         char* ob = ovf + ((size_t)blockIdx.x * 8 + slot * 4 + c) * pl.ovf_stride;
                         const size_t me = (size_t)pl.max_events;
                         lat = candidate_latency((unsigned long long*)ob, (double*)(ob + me * 8),
-                                                (unsigned long long*)(ob + me * 16), ne, woff, dd, endb, wt, h.ctot[c],
+                                                (unsigned long long*)(ob + me * 16), ne, woff, dd, endb, wt, ctot,
                                                 lane);
                     }
                 }
                 if (lane == 0) {
                     out_status[k] = (uint8_t)st;
-                    out_peak[k] = st ? -1 : h.peak[c] * pl.unit;
+                    out_peak[k] = st ? -1 : pk * pl.unit;
                     out_lat[k] = lat;
                 }
             }
             __syncwarp();
             PROF_MARK(15);
-            if (gi + 2 < ncta) {
-                __threadfence_block();
-                bar_arrive(kBarEmpty + slot, TM + TL);
-            }
+            if (gi + 2 < ncta) bar_arrive(kBarEmpty + slot, TM + TL);
         }
         if (prof)
 #pragma unroll
@@ -462,10 +479,15 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 if (d == 2) swm |= 1u << c;
                 if ((d > 2) | ((d == 1) & !(__ldg(g.rflag + r) & kRHasInput))) badm |= 1u << c;
             }
-            if (swm) atomicOr(&cl.swm, (int)swm);
+            // one shared atomic per warp
+            swm = __reduce_or_sync(0xffffffffu, swm);
+            badm = __reduce_or_sync(0xffffffffu, badm);
+            if (lane == 0) {
+                if (swm) atomicOr(&cl.swm, (int)swm);
 #pragma unroll
-            for (int c = 0; c < P; c++)
-                if ((badm >> c) & 1u) atomicOr(&cl.flags[c], MAGIS_ST_BAD_DEC);
+                for (int c = 0; c < P; c++)
+                    if ((badm >> c) & 1u) atomicOr(&cl.flags[c], MAGIS_ST_BAD_DEC);
+            }
         }
         // ---- phase 1: inverse permutation (pos stored +1); this thread's
         //      chunk of its team's candidate is in registers (loaded during the
@@ -729,7 +751,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     const double pc = __shfl_up_sync(0xffffffffu, cc, o2);
                     if (lane >= o2) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
                 }
-                if (lane == 31) { agg_s[warp] = ss; agg_m[warp] = mm; agg_c[warp] = cc; }
+                if (lane == 31) { agg_s[slot][warp] = ss; agg_m[slot][warp] = mm; agg_c[slot][warp] = cc; }
                 // add the lane's exclusive cost prefix within the warp to its events
                 const double pre = cc - cs1;
                 for (int e = o0; e < o; e++) cout_[e] += pre;
@@ -741,37 +763,16 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         bar_sync(kBarMain, TM);
         PROF_MARK(5);
-        // ---- phase 6: fold the team aggregates, hand-off to the latency warp ------
-        if (warp == 0) {
-            long long ss = lane < WM ? agg_s[lane] : 0;
-            long long mm = lane < WM ? agg_m[lane] : kNegInf;
-            double cc = lane < WM ? agg_c[lane] : 0.0;
-            const double c0 = cc;
-#pragma unroll
-            for (int o = 1; o < WT; o <<= 1) {
-                const long long ps = __shfl_up_sync(0xffffffffu, ss, o, WT);
-                const long long pm = __shfl_up_sync(0xffffffffu, mm, o, WT);
-                const double pc = __shfl_up_sync(0xffffffffu, cc, o, WT);
-                if ((lane % WT) >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
-            }
-            if (lane < WM) h.woff[lane] = cc - c0;
-            // team totals sit in lane c * WT + WT - 1
-            const int src = (lane < P ? lane : 0) * WT + WT - 1;
-            const long long pk = __shfl_sync(0xffffffffu, mm, src);
-            const double ct = __shfl_sync(0xffffffffu, cc, src);
+        // ---- phase 6: hand-off to the latency warps (they fold the aggregates) ----
+        if (tid < P) {
+            const int c = tid;
             int ne = 0;
 #pragma unroll
-            for (int w = 0; w < WT; w++) ne += wcnt[(lane < P ? lane : 0) * WT + w];
-            if (lane < P) {
-                const int c = lane;
-                const bool ok = (okm >> c) & 1u;
-                h.k[c] = ((vmask >> c) & 1u) ? grp * P + c : LLONG_MAX;
-                h.status[c] = (int)((stm >> (4 * c)) & 15u);
-                h.peak[c] = ok ? pk : 0;
-                h.ctot[c] = ok ? ct : 0.0;
-                h.swp[c] = (int)((swm >> c) & 1u);
-                h.nev[c] = ne;
-            }
+            for (int w = 0; w < WT; w++) ne += wcnt[c * WT + w];
+            h.k[c] = ((vmask >> c) & 1u) ? grp * P + c : LLONG_MAX;
+            h.status[c] = (int)((stm >> (4 * c)) & 15u);
+            h.swp[c] = (int)((swm >> c) & 1u);
+            h.nev[c] = ne;
         }
         if (R > 0) {
             // decisions of the group -> the slot (rows padded to 16 bytes)
@@ -788,7 +789,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 dst[i] = x;
             }
         }
-        __threadfence_block();
+        // bar.arrive orders this thread's prior shared / global writes for the
+        // threads that sync on the barrier (no membar: it would also wait for
+        // the next group's perm loads already in flight)
         bar_arrive(kBarFull + slot, TM + TL);
         PROF_MARK(6);
         // clear pos and the event marks for the next group
