@@ -17,6 +17,11 @@ Parity status per function:
   * swap latency (queues) ........ parity unpinned by the paper (reading P7);
                                    pinned only by hand-computed toys T1
   * pareto / best ................ pinned (definition, brute-force dominance)
+  * GraphHash (Alg. 3 l.3-6) ..... pinned (SplitMix64 published outputs for
+                                   mix64; WL unfolding-tree equivalence by
+                                   brute force; relabelling / schedule
+                                   invariance; materialised Fig. 8 graphs)
+  * hash filter (Alg. 3 l.10-12) . pinned (O(K^2) first-occurrence definition)
 """
 from __future__ import annotations
 
@@ -66,6 +71,13 @@ def _load():
     lib.orc_best_mem.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_int64]
     lib.orc_best_lat.restype = ctypes.c_int64
     lib.orc_best_lat.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_double]
+    lib.orc_mix64.restype = ctypes.c_uint64
+    lib.orc_mix64.argtypes = [ctypes.c_uint64]
+    lib.orc_hash_words.restype = ctypes.c_uint64
+    lib.orc_hash_words.argtypes = [P, ctypes.c_int64]
+    lib.orc_graph_hash.restype = ctypes.c_int
+    lib.orc_graph_hash.argtypes = [P, P, P, P, P]
+    lib.orc_graph_hash_batch.argtypes = [P, P, ctypes.c_int64, P, P, P]
     _lib = lib
     return lib
 
@@ -174,6 +186,61 @@ class OracleGraph:
         st = self._lib.orc_hotspots(self._h, _ptr(perm), _ptr(dec), int(nsplit), _ptr(hot), _ptr(heat),
                                     _ptr(score), _ptr(pk))
         return int(st), int(pk[0]), hot[:self.n], heat[:self.n], score[:self.n]
+
+    def graph_hash(self, label, dec=None):
+        """GraphHash of one candidate's transformed graph (Alg. 3 lines 3-6,
+        P:1693-1700; readings G1-G4) -> (status, hash, x[n_total]); x_v = 0
+        for inactive nodes."""
+        label = np.ascontiguousarray(label, dtype=np.uint64)
+        assert label.shape == (self.n,)
+        if dec is None or self.R == 0:
+            dec = np.zeros(max(self.R, 1), dtype=np.uint8)
+        dec = np.ascontiguousarray(dec, dtype=np.uint8)
+        x = np.zeros(max(self.n_total, 1), np.uint64)
+        h = np.zeros(1, np.uint64)
+        st = self._lib.orc_graph_hash(self._h, _ptr(label), _ptr(dec), _ptr(x), _ptr(h))
+        return int(st), int(h[0]), x[:self.n_total]
+
+    def graph_hash_batch(self, label, decs):
+        """decs: (K, R) uint8 -> (status u8[K], hash u64[K])."""
+        label = np.ascontiguousarray(label, dtype=np.uint64)
+        decs = np.ascontiguousarray(decs, dtype=np.uint8)
+        K = decs.shape[0]
+        if self.R == 0:
+            decs = np.zeros((K, 1), dtype=np.uint8)
+        st = np.zeros(K, np.uint8)
+        hs = np.zeros(K, np.uint64)
+        self._lib.orc_graph_hash_batch(self._h, _ptr(label), K, _ptr(decs), _ptr(st), _ptr(hs))
+        return st, hs
+
+
+def mix64(z: int) -> int:
+    """The SplitMix64 output function (reading G1)."""
+    return int(_load().orc_mix64(ctypes.c_uint64(z & 0xFFFFFFFFFFFFFFFF)))
+
+
+def hash_words(words) -> int:
+    """hash() of Alg. 3 over the concatenation of 64-bit words (reading G1)."""
+    w = np.ascontiguousarray(words, dtype=np.uint64)
+    return int(_load().orc_hash_words(_ptr(w), int(w.shape[0])))
+
+
+def hash_filter(hashes, status, seen=None):
+    """Alg. 3 lines 10-12 over a batch in candidate-id order: candidate k is
+    new iff it is valid, its hash is not in X (``seen``) and no earlier valid
+    candidate of the batch has the same hash; X then takes every valid hash.
+    Returns (new u8[K], X)."""
+    X = set() if seen is None else set(seen)
+    new = np.zeros(len(hashes), np.uint8)
+    for k, (h, s) in enumerate(zip(hashes, status)):
+        if s:
+            continue
+        h = int(h)
+        if h in X:
+            continue
+        X.add(h)
+        new[k] = 1
+    return new, X
 
 
 def pareto(peak, lat, status, ids=None):

@@ -142,45 +142,19 @@ static int64_t node_bytes(const orc_graph *g, int32_t v)
 }
 
 /*
- * Evaluate one candidate.
- *   perm[NT]  : the schedule over super-graph ids (step -> node)
- *   dec[R]    : 0 keep, 1 re-materialize, 2 swap (may be NULL when R == 0)
- * Outputs: status bits (bit0 not a permutation, bit1 edge violated,
- * bit2 bad decision), peak bytes (-1 if invalid), latency (+inf if invalid),
- * first compacted step attaining the peak (-1 if invalid).
+ * Active set and transformed edge list of one candidate (Fig. 8,
+ * P:1328-1346; readings P5, P6): original nodes are always active; clone_r
+ * iff dec[r] = 1; store_r and load_r iff dec[r] = 2.  Re-mat moves the late
+ * users U_r to the clone A', which reads the original copies of pre(t_r);
+ * swap adds t_r -> Store -> Load and moves U_r to the Load.  active[NT] is
+ * zeroed by the caller; *tsrc / *tdst are malloc'ed here.
  */
-static void eval_impl(const orc_graph *g, const int32_t *perm, const uint8_t *dec,
-                      uint8_t *status_out, int64_t *peak_out, double *lat_out,
-                      int64_t *argmax_out, uint8_t *hot_out)
+static void transformed_graph(const orc_graph *g, const uint8_t *dec, uint8_t *active,
+                              int32_t **tsrc_out, int32_t **tdst_out, int64_t *nte_out)
 {
-    const int32_t n = g->n, R = g->R, NT = g->NT;
-    uint8_t status = 0;
-    uint8_t *seen = NULL, *active = NULL;
-    int32_t *pos = NULL, *step = NULL, *ord = NULL, *last = NULL;
-    int32_t *tsrc = NULL, *tdst = NULL;
+    const int32_t n = g->n, R = g->R;
     int64_t nte = 0, cap_te, i, k;
-    int32_t nact = 0;
-    int64_t peak = -1, argmax = -1;
-    double latency = INFINITY;
-
-    /* 1. permutation and decision check (P:402-405; reading P12) */
-    seen = (uint8_t *)calloc(NT ? NT : 1, 1);
-    for (i = 0; i < NT; i++) {
-        int32_t p = perm[i];
-        if (p < 0 || p >= NT || seen[p]) { status |= 1; continue; }
-        seen[p] = 1;
-    }
-    for (i = 0; i < R; i++) {
-        uint8_t d = dec[i];
-        if (d > 2) status |= 4;
-        /* re-materialization needs A's inputs (P:1333-1336): a tensor with no
-         * inputs cannot be re-computed (DESIGN.md reading R-noinput). */
-        if (d == 1 && !g->has_input[g->elig[i]]) status |= 4;
-    }
-    if (status) goto done;
-
-    /* 2. active set and transformed graph (Fig. 8, P:1333-1346) */
-    active = (uint8_t *)calloc(NT ? NT : 1, 1);
+    int32_t *tsrc, *tdst;
     for (i = 0; i < n; i++) active[i] = 1;
     for (i = 0; i < R; i++) {
         if (dec[i] == 1) active[n + 3 * i] = 1;
@@ -217,6 +191,50 @@ static void eval_impl(const orc_graph *g, const int32_t *perm, const uint8_t *de
             tsrc[nte] = n + 3 * (int32_t)i + 1; tdst[nte] = n + 3 * (int32_t)i + 2; nte++;
         }
     }
+    *tsrc_out = tsrc; *tdst_out = tdst; *nte_out = nte;
+}
+
+/*
+ * Evaluate one candidate.
+ *   perm[NT]  : the schedule over super-graph ids (step -> node)
+ *   dec[R]    : 0 keep, 1 re-materialize, 2 swap (may be NULL when R == 0)
+ * Outputs: status bits (bit0 not a permutation, bit1 edge violated,
+ * bit2 bad decision), peak bytes (-1 if invalid), latency (+inf if invalid),
+ * first compacted step attaining the peak (-1 if invalid).
+ */
+static void eval_impl(const orc_graph *g, const int32_t *perm, const uint8_t *dec,
+                      uint8_t *status_out, int64_t *peak_out, double *lat_out,
+                      int64_t *argmax_out, uint8_t *hot_out)
+{
+    const int32_t n = g->n, R = g->R, NT = g->NT;
+    uint8_t status = 0;
+    uint8_t *seen = NULL, *active = NULL;
+    int32_t *pos = NULL, *step = NULL, *ord = NULL, *last = NULL;
+    int32_t *tsrc = NULL, *tdst = NULL;
+    int64_t nte = 0, i, k;
+    int32_t nact = 0;
+    int64_t peak = -1, argmax = -1;
+    double latency = INFINITY;
+
+    /* 1. permutation and decision check (P:402-405; reading P12) */
+    seen = (uint8_t *)calloc(NT ? NT : 1, 1);
+    for (i = 0; i < NT; i++) {
+        int32_t p = perm[i];
+        if (p < 0 || p >= NT || seen[p]) { status |= 1; continue; }
+        seen[p] = 1;
+    }
+    for (i = 0; i < R; i++) {
+        uint8_t d = dec[i];
+        if (d > 2) status |= 4;
+        /* re-materialization needs A's inputs (P:1333-1336): a tensor with no
+         * inputs cannot be re-computed (DESIGN.md reading R-noinput). */
+        if (d == 1 && !g->has_input[g->elig[i]]) status |= 4;
+    }
+    if (status) goto done;
+
+    /* 2. active set and transformed graph (Fig. 8, P:1333-1346) */
+    active = (uint8_t *)calloc(NT ? NT : 1, 1);
+    transformed_graph(g, dec, active, &tsrc, &tdst, &nte);
 
     /* 3. validity: every dependency must be respected */
     pos = (int32_t *)malloc(sizeof(int32_t) * NT);
@@ -552,4 +570,110 @@ int64_t orc_best_lat(int64_t n, const int64_t *peak, const double *lat,
         if (id[i] < id[b]) b = i;
     }
     return b;
+}
+
+/* ------------------------------------------------------------------------
+ * GraphHash (Alg. 3 lines 3-6; the Weisfeiler-Lehman idea and
+ * "(+) means bytes concatenation").  Readings G1-G4:
+ *
+ *   hash(b), b a byte string of 8m bytes read as little-endian 64-bit words
+ *   w_0..w_{m-1}:   h = GAMMA * (m + 1);  h = mix64(h ^ w_i) for i = 0..m-1
+ *   mix64 = the SplitMix64 output function, GAMMA = 0x9E3779B97F4A7C15   (G1)
+ *
+ *   line 5:  x_v = hash( hash(label_v) (+) x_{u_1} (+) ... (+) x_{u_k} )
+ *            u_1..u_k = pre(v) in the transformed graph, in ascending order
+ *            of x_u (pre(v) is a set; G2)
+ *   line 6:  GraphHash(G) = hash( sum_v x_v mod 2^64 )
+ *
+ * label_v: the caller's 64-bit label of original op v; a clone A' carries
+ * label(t_r) (same op, same inputs; G3); Store_r / Load_r carry
+ * the tags 0x45524F5453 ("STORE") / 0x44414F4C ("LOAD") (G3).  The graph of
+ * a candidate is its transformed graph (Fig. 8) over the active nodes; the
+ * schedule does not enter (G4).  Invalid decisions: status bit 2, hash 0.
+ * ------------------------------------------------------------------------ */
+#define ORC_GAMMA 0x9E3779B97F4A7C15ull
+#define ORC_TAG_STORE 0x45524F5453ull
+#define ORC_TAG_LOAD 0x44414F4Cull
+
+uint64_t orc_mix64(uint64_t z)
+{
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+uint64_t orc_hash_words(const uint64_t *w, int64_t m)
+{
+    uint64_t h = ORC_GAMMA * (uint64_t)(m + 1);
+    int64_t i;
+    for (i = 0; i < m; i++) h = orc_mix64(h ^ w[i]);
+    return h;
+}
+
+static int cmp_u64(const void *a, const void *b)
+{
+    const uint64_t x = *(const uint64_t *)a, y = *(const uint64_t *)b;
+    return (x > y) - (x < y);
+}
+
+/* x_out[NT] (0 for inactive nodes) may be NULL.  Returns the status bits. */
+int orc_graph_hash(const orc_graph *g, const uint64_t *label, const uint8_t *dec,
+                   uint64_t *x_out, uint64_t *hash_out)
+{
+    const int32_t n = g->n, R = g->R, NT = g->NT;
+    uint8_t *active;
+    int32_t *tsrc, *tdst, *indeg, *queue;
+    int64_t nte, i, k;
+    int32_t qh = 0, qt = 0;
+    uint64_t *x, *buf, sum = 0;
+    int status = 0;
+
+    for (i = 0; i < R; i++) {
+        if (dec[i] > 2) status |= 4;
+        if (dec[i] == 1 && !g->has_input[g->elig[i]]) status |= 4;   /* reading R-noinput */
+    }
+    if (status) {
+        if (x_out) for (i = 0; i < NT; i++) x_out[i] = 0;
+        *hash_out = 0;
+        return status;
+    }
+    active = (uint8_t *)calloc(NT ? NT : 1, 1);
+    transformed_graph(g, dec, active, &tsrc, &tdst, &nte);
+    x = (uint64_t *)calloc(NT ? NT : 1, sizeof(uint64_t));
+    buf = (uint64_t *)malloc(sizeof(uint64_t) * (nte + 1));
+    indeg = (int32_t *)calloc(NT ? NT : 1, sizeof(int32_t));
+    queue = (int32_t *)malloc(sizeof(int32_t) * (NT ? NT : 1));
+    for (k = 0; k < nte; k++) indeg[tdst[k]]++;
+    for (i = 0; i < NT; i++) if (active[i] && indeg[i] == 0) queue[qt++] = (int32_t)i;
+    /* line 4: for v in topo-order(G) (Kahn) */
+    while (qh < qt) {
+        const int32_t v = queue[qh++];
+        uint64_t lab;
+        int64_t m = 0;
+        if (v < n) lab = label[v];
+        else {
+            const int32_t r = (v - n) / 3, kind = (v - n) % 3;
+            lab = kind == 0 ? label[g->elig[r]] : kind == 1 ? ORC_TAG_STORE : ORC_TAG_LOAD;
+        }
+        /* line 5: hash(v) (+) the x_u of pre(v), ascending */
+        buf[m++] = orc_hash_words(&lab, 1);
+        for (k = 0; k < nte; k++) if (tdst[k] == v) buf[m++] = x[tsrc[k]];
+        qsort(buf + 1, (size_t)(m - 1), sizeof(uint64_t), cmp_u64);
+        x[v] = orc_hash_words(buf, m);
+        sum += x[v];
+        for (k = 0; k < nte; k++) if (tsrc[k] == v && --indeg[tdst[k]] == 0) queue[qt++] = tdst[k];
+    }
+    /* line 6 */
+    *hash_out = orc_hash_words(&sum, 1);
+    if (x_out) for (i = 0; i < NT; i++) x_out[i] = x[i];
+    free(active); free(tsrc); free(tdst); free(x); free(buf); free(indeg); free(queue);
+    return 0;
+}
+
+void orc_graph_hash_batch(const orc_graph *g, const uint64_t *label, int64_t K, const uint8_t *decs,
+                          uint8_t *status, uint64_t *hash)
+{
+    int64_t k;
+    for (k = 0; k < K; k++)
+        status[k] = (uint8_t)orc_graph_hash(g, label, g->R ? decs + k * (int64_t)g->R : NULL, NULL, hash + k);
 }
