@@ -44,6 +44,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-int32", action="store_true", help="e2e with int32 host schedules instead of uint16")
+    ap.add_argument("--ghash", action="store_true",
+                    help="batched GraphHash + duplicate filter of the K candidates' graphs (NEXT-2)")
     ap.add_argument("--windows", action="store_true",
                     help="local-move candidates scored by windowed delta evaluation (NEXT-1); default config c5, K=1M")
     return ap.parse_args()
@@ -208,6 +210,8 @@ def main():
         if pool is not None:
             pool.close()
         return run_windows(args, wl, cfg, rank, world, local)
+    if args.ghash:
+        return run_ghash(args, wl, cfg, K, workload, pool, ncores, rank, world, local)
 
     import torch
     import torch.distributed as dist
@@ -460,6 +464,169 @@ def run_windows(args, wl, cfg, rank, world, local):
                              "kernel_ms_avg": round(kern, 4)},
                 "cpu_baseline": None, "e2e": None, "clocks": clk.summary(), "gpu_launches": args.steps * 7,
                 "setup": {"window_gen_s": round(gen_s, 3)}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def _oracle_hash_chunk(args):
+    decs, labels = args
+    import oracle
+    size, cost, iso, src, dst, elig, U, B, lam = _WL
+    g = oracle.OracleGraph(size, cost, iso, src, dst, elig, U, B, lam)
+    t = time.perf_counter()
+    st, hs = g.graph_hash_batch(labels, decs)
+    return st, hs, time.perf_counter() - t
+
+
+def ghash_words(wl, D):
+    """Words absorbed by hash() per candidate (algorithmic work of Alg. 3
+    line 5-6): per active node 1 + |pre(v)|, plus 1 for line 6."""
+    indeg = np.bincount(np.unique(wl.src.astype(np.int64) * wl.n + wl.dst) % wl.n, minlength=wl.n)
+    w0 = int((1 + indeg).sum()) + 1
+    if wl.R == 0:
+        return float(w0)
+    extra_remat = 1 + indeg[wl.elig]                  # clone: 1 + |pre(t_r)|
+    Dv = D[:, :wl.R]
+    per = w0 + (Dv == 1).astype(np.int64) @ extra_remat + 4 * (Dv == 2).sum(axis=1)   # Store 2 + Load 2
+    return float(per.mean())
+
+
+def run_ghash(args, wl, cfg, K, workload, pool, ncores, rank, world, local):
+    """NEXT-2: one step = magis_graph_hash over the K candidates' decision
+    vectors (the transformed graphs) + the hash-set filter (Alg. 3 lines
+    10-12) into a set cleared at the start of the step."""
+    import torch
+    import torch.distributed as dist
+    from magis_inputs import CandidateGenerator, CandidateSpec
+    from magis_inputs.labels import node_labels
+    from paper_conf_asplos_chend0zll024_b200 import Graph, GraphHasher, HashSet
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    labels = node_labels(wl)
+    _, Dh = CandidateGenerator(wl, CandidateSpec(seed=args.seed)).generate(rank * K, K)
+    Dh = np.ascontiguousarray(Dh[:, :max(wl.R, 1)])
+    Dh_t = torch.from_numpy(Dh).pin_memory()
+    D = Dh_t.to(dev)
+    g = Graph.from_workload(wl, device=local)
+    hz = GraphHasher(g, labels)
+    hs = HashSet(max(2 * K * world, 1024), device=local)
+    from paper_conf_asplos_chend0zll024_b200.distributed import global_filter
+    st = torch.empty(K, dtype=torch.uint8, device=dev)
+    hv = torch.empty(K, dtype=torch.int64, device=dev)
+    new = torch.empty(K, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step(evp=None):
+        hs.clear(stream=stream)
+        if evp:
+            evp[0].record(stream)
+        hz.hash(D if wl.R else K, status=st, out=hv, stream=stream)
+        if evp:
+            evp[1].record(stream)
+        if world > 1:      # the seen-set X is global: all-gather (hash, status), filter in id order
+            new.copy_(global_filter(hv, st, K, lambda hb, sb: hs.filter(hb, sb, stream=stream)))
+        else:
+            hs.filter(hv, st, out=new, stream=stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clk = ClockSampler(local)
+    with clk:
+        start.record(stream)
+        for i in range(args.steps):
+            step(evs[i])
+        end.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t = torch.tensor([start.elapsed_time(end), statistics.mean(a.elapsed_time(b) for a, b in evs)],
+                     dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms, kern = t.tolist()
+    ms_per_step = ms / args.steps
+    value = world * K / (ms_per_step / 1e3)
+    n_new = int(new.sum().item())
+    # roofline: ALU-pipe bound (DESIGN.md §6 GraphHash): one absorbed word =
+    # h ^ w + mix64 = 14 ALU-pipe + 6 FMA-pipe SASS ops; ALU pipe 16 lanes/clk/SMSP
+    words = ghash_words(wl, Dh)
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    clk_mhz = (clk.summary() or {}).get("sm_mhz") or 1965.0
+    peak_words = sms * 4 * 16 * clk_mhz * 1e6 / 14.0
+    achieved = K * words / (kern / 1e3)
+    # e2e: decisions H2D from pinned memory, hash + filter, results D2H
+    hst = torch.empty(K, dtype=torch.uint8).pin_memory()
+    hnew = torch.empty(K, dtype=torch.uint8).pin_memory()
+    hhash = torch.empty(K, dtype=torch.int64).pin_memory()
+    Dd = torch.empty_like(D)
+
+    def e2e_step():
+        Dd.copy_(Dh_t, non_blocking=True)
+        hs.clear(stream=stream)
+        hz.hash(Dd if wl.R else K, status=st, out=hv, stream=stream)
+        hs.filter(hv, st, out=new, stream=stream)
+        hst.copy_(st, non_blocking=True)
+        hhash.copy_(hv, non_blocking=True)
+        hnew.copy_(new, non_blocking=True)
+        torch.cuda.synchronize()
+    e2e_step()
+    n_e2e = max(1, min(args.steps, 5))
+    t0 = time.perf_counter()
+    for _ in range(n_e2e):
+        e2e_step()
+    e2e_s = (time.perf_counter() - t0) / n_e2e
+    te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e = {"value": round(world * K / te.item(), 1), "unit": UNIT, "h2d_bytes_per_step": int(Dh.nbytes),
+           "d2h_bytes_per_step": int(K * 10), "api": "GraphHasher.hash + HashSet.filter (magis_graph_hash, "
+           "magis_hashset_filter) with pinned host decisions / results", "s_per_step": round(te.item(), 5)}
+    cpu = None
+    if pool is not None:
+        hh = hv.cpu().numpy().view(np.uint64)
+        sth = st.cpu().numpy()
+        probe = 64
+        S = probe
+        parts = np.array_split(np.arange(probe), ncores)
+        t0 = time.perf_counter()
+        pool.map(_oracle_hash_chunk, [(Dh[p], labels) for p in parts if len(p)])
+        rate = probe / max(time.perf_counter() - t0, 1e-6)
+        S = int(min(K, max(probe, rate * args.cpu_seconds)))
+        parts = np.array_split(np.arange(S), ncores * 4)
+        t0 = time.perf_counter()
+        res = pool.map(_oracle_hash_chunk, [(Dh[p], labels) for p in parts if len(p)])
+        wall = time.perf_counter() - t0
+        rs = np.concatenate([r[0] for r in res])
+        rh = np.concatenate([r[1] for r in res])
+        cpu = {"value": round(S / wall, 1), "unit": UNIT, "cores": ncores, "kind": "oracle",
+               "sample": f"first {S} of the {K} candidates' graphs hashed (single-thread C oracle per process, "
+                         f"{ncores} processes), {wall:.1f} s",
+               "parity_on_sample": bool((rs == sth[:S]).all() and (rh == hh[:S]).all())}
+        pool.close()
+    if rank == 0:
+        line = {"metric": "candidate graphs hashed + filtered/sec (GraphHash, Alg. 3 lines 3-6, 10-12)",
+                "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+                "config": {**workload, "workload": f"{cfg}: GraphHash of {K} candidate graphs (decisions of the "
+                           "bench candidates) + duplicate filter (NEXT-2)", "parallelism": f"candidate-dp{world}",
+                           "new_graphs": n_new, "words_per_candidate": round(words, 1), "ghash": hz.info,
+                           "l2": "decisions stream once (K x R bytes); value slots L2-resident"},
+                "roofline": {"bound": "alu", "achieved": round(achieved / 1e9, 2), "peak": round(peak_words / 1e9, 1),
+                             "unit": "Gword/s", "frac": round(achieved / peak_words, 4), "traffic": None,
+                             "peak_source": "derived: SMs x 4 SMSP x 16 ALU lanes/clk (B300_MICROARCH rt_SMSP=2) x "
+                                            "SM clock / 14 ALU-pipe ops per absorbed word",
+                             "kernel": "magis::ghash_kernel", "kernel_ms_avg": round(kern, 4),
+                             "kernel_share_of_step": round(kern / ms_per_step, 4)},
+                "cpu_baseline": cpu, "e2e": e2e, "clocks": clk.summary(), "gpu_launches": args.steps * 3}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

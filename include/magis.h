@@ -313,6 +313,69 @@ int magis_pareto_merge(int64_t n, const int64_t* d_peak, const double* d_lat,
                        double lat_limit, int64_t* d_best, void* d_workspace,
                        int64_t workspace_bytes, void* cuda_stream);
 
+/*
+ * Batched GraphHash (Alg. 3 lines 3-6, and
+ * the Weisfeiler-Lehman test of P:1776-1778; readings G1-G4 in DESIGN.md).
+ * The graph of candidate k is its transformed graph (the Fig. 8 rules of
+ * dec[k] applied to G; the schedule does not enter, G4).  For
+ * every active node v, in topological order,
+ *     x_v = hash( hash(label_v) (+) x_{u_1} (+) ... (+) x_{u_d} )      (line 5)
+ * where u_1..u_d = pre(v) sorted by ascending x (G2) and (+) concatenates
+ * 64-bit words; GraphHash = hash( sum_v x_v mod 2^64 ) (line 6).
+ * hash(w_0..w_{m-1}) = fold h = mix64(h ^ w_i) from h = 0x9E3779B97F4A7C15 *
+ * (m + 1), mix64 = the SplitMix64 output function (G1).  A clone carries
+ * label(t_r); Store / Load carry 0x45524F5453 / 0x44414F4C (G3).
+ *
+ * magis_ghash_create: h_label [n_nodes] uint64 host memory (copied; the
+ *   caller's op signature, e.g. type + attributes + shape), builds the node
+ *   order, value slots and tables on the graph's device (synchronous).
+ *   *out is library-owned and tied to g (free it before g).
+ *   Errors: MAGIS_E_INVAL, MAGIS_E_NOMEM, MAGIS_E_CUDA.
+ * magis_graph_hash: d_dec [K x R] uint8 device memory (NULL if R == 0);
+ *   d_status [K] uint8 out (MAGIS_ST_BAD_DEC or 0); d_hash [K] uint64 out
+ *   (0 if status != 0).  Asynchronous on the stream, no allocation; the
+ *   scratch belongs to *h, so calls on one h are serialised by the caller.
+ *   Errors: MAGIS_E_INVAL (K < 0, null pointer), MAGIS_E_CUDA.
+ * magis_ghash_info: shared / global value slots per warp, the number of
+ *   values kept in global slots, persistent grid (any pointer may be NULL).
+ */
+typedef struct magis_ghash magis_ghash;   /* opaque, library-owned */
+
+int magis_ghash_create(const magis_graph* g, const uint64_t* h_label, magis_ghash** out);
+int magis_ghash_free(magis_ghash* h);
+int magis_graph_hash(magis_ghash* h, int64_t K, const uint8_t* d_dec, uint8_t* d_status, uint64_t* d_hash,
+                     void* cuda_stream);
+int magis_ghash_info(const magis_ghash* h, int32_t* shared_slots, int32_t* global_slots, int64_t* global_nodes,
+                     int32_t* grid);
+
+/*
+ * The duplicate filter of Alg. 3 lines 10-12 over a batch: a
+ * device hash set X of graph hashes.  magis_hashset_filter processes the
+ * batch as if in candidate-id order: d_new[k] = 1 iff d_status[k] == 0 (or
+ * d_status is NULL), d_hash[k] is not in X and no smaller k' of the batch
+ * with status 0 has the same hash; then every valid hash joins X.  All hash
+ * values (0 included) are ordinary keys.
+ * capacity: keys the set can hold (rounded up to a power of two, <= 2^40).
+ *   Open addressing: keep the load below ~0.7.  If the set is full an insert
+ *   is dropped, counted in n_overflow, and that candidate is reported new
+ *   (never a false duplicate).
+ * d_hash [K] uint64, d_status [K] uint8 or NULL, d_new [K] uint8 out: device
+ *   memory.  Asynchronous on the stream; calls on one set are serialised by
+ *   the caller (one stream).  K < 2^40; at most 2^24 - 2 filter calls between
+ *   clears (MAGIS_E_CAPACITY after that).
+ * magis_hashset_stats synchronises and returns |X| and dropped inserts.
+ * Errors: MAGIS_E_INVAL, MAGIS_E_NOMEM, MAGIS_E_CUDA, MAGIS_E_UNSUPPORTED
+ *   (no sm_100 device), MAGIS_E_CAPACITY.
+ */
+typedef struct magis_hashset magis_hashset;   /* opaque, library-owned */
+
+int magis_hashset_create(int device, int64_t capacity, magis_hashset** out);
+int magis_hashset_free(magis_hashset* s);
+int magis_hashset_clear(magis_hashset* s, void* cuda_stream);
+int magis_hashset_filter(magis_hashset* s, int64_t K, const uint64_t* d_hash, const uint8_t* d_status,
+                         uint8_t* d_new, void* cuda_stream);
+int magis_hashset_stats(const magis_hashset* s, int64_t* n_keys, int64_t* n_overflow);
+
 /* Thread-local message for the last nonzero return on this thread. */
 const char* magis_last_error(void);
 

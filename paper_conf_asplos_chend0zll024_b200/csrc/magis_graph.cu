@@ -385,6 +385,14 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     dg.pred_ptr = (const int32_t*)(b + o_pp);
     dg.pred = (const int32_t*)(b + o_p);
     g->idom = idom;
+    // host copies for plans built after load (GraphHash, NEXT-2)
+    g->h_pred_ptr = pred_ptr;
+    g->h_pred = pred;
+    g->h_topo = topo;
+    g->h_elig = elig;
+    g->h_Uptr = U_ptr;
+    g->h_Uidx = U_idx;
+    g->h_rflag = rflag;
     g->gen.succ_ptr = (const int32_t*)(b + o_sp);
     g->gen.succ = (const int32_t*)(b + o_s);
     g->gen.pred_ptr = (const int32_t*)(b + o_pp);

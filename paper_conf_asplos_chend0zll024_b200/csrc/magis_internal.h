@@ -233,6 +233,9 @@ struct magis_graph {
     int64_t n_edges = 0;
     int64_t n_super_edges = 0;
     std::vector<int32_t> idom;     // dominator tree of G (host copy)
+    // host copies of the load-time tables (plans built later: GraphHash)
+    std::vector<int32_t> h_pred_ptr, h_pred, h_topo, h_elig, h_Uptr, h_Uidx;
+    std::vector<uint8_t> h_rflag;
     void* hs_ws = nullptr;         // hot-spot query workspace (lazily allocated)
     size_t hs_ws_bytes = 0;
     // host-buffer (end-to-end) path: lazily allocated staging

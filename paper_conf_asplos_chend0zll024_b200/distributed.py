@@ -46,3 +46,28 @@ def global_front(front: Dict[str, torch.Tensor], cap: int, mem_limit: int = -1,
     merge = merge or (lambda peak, lat, ids, cap, M, L: magis.pareto_merge(
         peak, lat, None, ids=ids, cap=cap, mem_limit=M, lat_limit=L))
     return merge(g["front_peak"], g["front_lat"], g["front_id"], cap, mem_limit, lat_limit)
+
+
+def global_filter(hashes: torch.Tensor, status: torch.Tensor, kmax: int, filt: Callable,
+                  group=None) -> torch.Tensor:
+    """Alg. 3 lines 10-12 across ranks (NEXT-2): each rank hashed its own
+    contiguous shard of candidates; the (hash, status) pairs are all-gathered
+    in rank order -- which is global candidate-id order -- padded to ``kmax``
+    per rank with status 0xFF (ignored), and every rank runs the same filter
+    over the gathered list, so every rank's seen-set X stays identical.
+    ``filt(hashes, status) -> is_new`` is the caller's set (HashSet.filter on
+    the device; a host stand-in in the CPU tests).  Returns this rank's slice
+    of the new-flags."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    k = hashes.numel()
+    h = torch.zeros(kmax, dtype=torch.int64, device=hashes.device)
+    s = torch.full((kmax,), 0xFF, dtype=torch.uint8, device=status.device)
+    h[:k] = hashes
+    s[:k] = status
+    hb = torch.empty(world * kmax, dtype=torch.int64, device=h.device)
+    sb = torch.empty(world * kmax, dtype=torch.uint8, device=s.device)
+    dist.all_gather_into_tensor(hb, h, group=group)
+    dist.all_gather_into_tensor(sb, s, group=group)
+    new = filt(hb, sb)
+    return new[rank * kmax: rank * kmax + k]

@@ -25,7 +25,9 @@ EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magi
            "magis_eval_schedules_host", "magis_pareto_workspace_size", "magis_pareto_merge",
            "magis_last_error", "magis_abi_version", "magis_device_supported", "magis_generate_candidates",
            "magis_base_create", "magis_base_info", "magis_base_free", "magis_eval_windows", "magis_hotspots",
-           "magis_graph_idom", "magis_eval_schedules_host_u16"]
+           "magis_graph_idom", "magis_eval_schedules_host_u16", "magis_ghash_create", "magis_ghash_free",
+           "magis_graph_hash", "magis_ghash_info", "magis_hashset_create", "magis_hashset_free",
+           "magis_hashset_clear", "magis_hashset_filter", "magis_hashset_stats"]
 
 
 class MagisError(RuntimeError):
@@ -104,6 +106,25 @@ def lib() -> ctypes.CDLL:
     L.magis_hotspots.restype = ctypes.c_int
     L.magis_graph_idom.argtypes = [P, P]
     L.magis_graph_idom.restype = ctypes.c_int
+    L.magis_ghash_create.argtypes = [P, P, ctypes.POINTER(P)]
+    L.magis_ghash_create.restype = ctypes.c_int
+    L.magis_ghash_free.argtypes = [P]
+    L.magis_ghash_free.restype = ctypes.c_int
+    L.magis_graph_hash.argtypes = [P, i64, P, P, P, P]
+    L.magis_graph_hash.restype = ctypes.c_int
+    L.magis_ghash_info.argtypes = [P, ctypes.POINTER(i32), ctypes.POINTER(i32), ctypes.POINTER(i64),
+                                   ctypes.POINTER(i32)]
+    L.magis_ghash_info.restype = ctypes.c_int
+    L.magis_hashset_create.argtypes = [ctypes.c_int, i64, ctypes.POINTER(P)]
+    L.magis_hashset_create.restype = ctypes.c_int
+    L.magis_hashset_free.argtypes = [P]
+    L.magis_hashset_free.restype = ctypes.c_int
+    L.magis_hashset_clear.argtypes = [P, P]
+    L.magis_hashset_clear.restype = ctypes.c_int
+    L.magis_hashset_filter.argtypes = [P, i64, P, P, P, P]
+    L.magis_hashset_filter.restype = ctypes.c_int
+    L.magis_hashset_stats.argtypes = [P, ctypes.POINTER(i64), ctypes.POINTER(i64)]
+    L.magis_hashset_stats.restype = ctypes.c_int
     _lib = L
     return L
 
@@ -271,6 +292,92 @@ class Graph:
         fn = self._L.magis_eval_schedules_host_u16 if u16 else self._L.magis_eval_schedules_host
         _check(fn(self._h, K, _np_ptr(p), _np_ptr(dd), _np_ptr(st), _np_ptr(pk), _np_ptr(lt), _stream_ptr(stream)))
         return st, pk, lt
+
+
+class GraphHasher:
+    """Batched GraphHash of candidate graphs (magis_ghash_create /
+    magis_graph_hash; Alg. 3 lines 3-6).  labels: uint64 [n] op labels."""
+
+    def __init__(self, graph: "Graph", labels):
+        self._L = graph._L
+        self.graph = graph
+        lab = np.ascontiguousarray(labels, np.uint64)
+        assert lab.shape == (graph.n,)
+        h = ctypes.c_void_p()
+        _check(self._L.magis_ghash_create(graph._h, _np_ptr(lab), ctypes.byref(h)))
+        self._h = h
+        ns, gs, gn, gr = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int64(), ctypes.c_int32()
+        _check(self._L.magis_ghash_info(h, ctypes.byref(ns), ctypes.byref(gs), ctypes.byref(gn), ctypes.byref(gr)))
+        self.info = {"shared_slots": ns.value, "global_slots": gs.value, "global_nodes": gn.value,
+                     "grid": gr.value}
+
+    def hash(self, dec, status=None, out=None, stream=None):
+        """dec: cuda uint8 [K, R] (R == 0: a [K, 1] tensor or an int K).
+        Returns (status uint8 [K], hash int64 [K] holding the uint64 bits)."""
+        import torch
+        if isinstance(dec, int):
+            K, dev, dp = dec, torch.device("cuda", self.graph.device), None
+        else:
+            K, dev = int(dec.shape[0]), dec.device
+            assert dec.dtype == torch.uint8 and dec.is_contiguous()
+            if self.graph.R:
+                assert dec.shape[1] == self.graph.R
+            dp = _tptr(dec) if self.graph.R else None
+        status = torch.empty(K, dtype=torch.uint8, device=dev) if status is None else status
+        out = torch.empty(K, dtype=torch.int64, device=dev) if out is None else out
+        _check(self._L.magis_graph_hash(self._h, K, dp, _tptr(status), _tptr(out), _stream_ptr(stream)))
+        return status, out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._L.magis_ghash_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class HashSet:
+    """The seen-graph set X of Alg. 3 (lines 10-12) on the device."""
+
+    def __init__(self, capacity: int, device: int = 0):
+        self._L = lib()
+        h = ctypes.c_void_p()
+        _check(self._L.magis_hashset_create(int(device), int(capacity), ctypes.byref(h)))
+        self._h = h
+        self.device = device
+
+    def filter(self, hashes, status=None, out=None, stream=None):
+        """hashes: cuda int64 [K] (uint64 bits); status: cuda uint8 [K] or None.
+        Returns is_new uint8 [K] (first valid occurrence not already in X)."""
+        import torch
+        K = int(hashes.shape[0])
+        out = torch.empty(K, dtype=torch.uint8, device=hashes.device) if out is None else out
+        _check(self._L.magis_hashset_filter(self._h, K, _tptr(hashes), _tptr(status), _tptr(out),
+                                            _stream_ptr(stream)))
+        return out
+
+    def clear(self, stream=None):
+        _check(self._L.magis_hashset_clear(self._h, _stream_ptr(stream)))
+
+    def stats(self):
+        n, o = ctypes.c_int64(), ctypes.c_int64()
+        _check(self._L.magis_hashset_stats(self._h, ctypes.byref(n), ctypes.byref(o)))
+        return n.value, o.value
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._L.magis_hashset_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 class Base:

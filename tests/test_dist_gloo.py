@@ -102,3 +102,57 @@ def test_shard_ranges_cover_exactly():
             r = [pdist.shard_range(K, i, world) for i in range(world)]
             assert r[0][0] == 0 and r[-1][1] == K
             assert all(r[i][1] == r[i + 1][0] for i in range(world - 1))
+
+
+def _filter_worker(rank, world, port, K, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        rng = np.random.default_rng(9)
+        X = set()
+
+        def filt(hb, sb):
+            nonlocal X
+            new, X = oracle.hash_filter(hb.numpy().view(np.uint64), sb.numpy(), X)
+            return torch.from_numpy(new)
+        out = []
+        for b in range(3):
+            hv = rng.integers(0, 300, K).astype(np.uint64)
+            st = ((rng.random(K) < 0.1) * 4).astype(np.uint8)
+            lo, hi = pdist.shard_range(K, rank, world)
+            kmax = max(pdist.shard_range(K, r, world)[1] - pdist.shard_range(K, r, world)[0] for r in range(world))
+            new = pdist.global_filter(torch.from_numpy(hv[lo:hi].view(np.int64)), torch.from_numpy(st[lo:hi]),
+                                      kmax, filt)
+            out.append((lo, new.numpy().tolist()))
+        q.put((rank, out, sorted(X)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_hash_filter_matches_single_rank():
+    """NEXT-2 across ranks: the gathered filter equals one filter over all
+    candidates in id order, batch after batch, and every rank keeps the same X."""
+    world, K = 2, 1001
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = free_port()
+    procs = [ctx.Process(target=_filter_worker, args=(r, world, port, K, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    rng = np.random.default_rng(9)
+    X = set()
+    exp = []
+    for b in range(3):
+        hv = rng.integers(0, 300, K).astype(np.uint64)
+        st = ((rng.random(K) < 0.1) * 4).astype(np.uint8)
+        new, X = oracle.hash_filter(hv, st, X)
+        exp.append(new)
+    for rank, out, Xr in res:
+        assert Xr == sorted(X)
+        for b, (lo, new) in enumerate(out):
+            assert new == exp[b][lo:lo + len(new)].tolist()
