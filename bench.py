@@ -556,11 +556,11 @@ def run_ghash(args, wl, cfg, K, workload, pool, ncores, rank, world, local):
     value = world * K / (ms_per_step / 1e3)
     n_new = int(new.sum().item())
     # roofline: ALU-pipe bound (DESIGN.md §6 GraphHash): one absorbed word =
-    # h ^ w + mix64 = 14 ALU-pipe + 6 FMA-pipe SASS ops; ALU pipe 16 lanes/clk/SMSP
+    # h ^ w + mix64 = 12.5 ALU-pipe (LOP3/SHF) + 8 FMA-pipe (IMAD) SASS ops (cuobjdump); ALU pipe 16 lanes/clk/SMSP
     words = ghash_words(wl, Dh)
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
     clk_mhz = (clk.summary() or {}).get("sm_mhz") or 1965.0
-    peak_words = sms * 4 * 16 * clk_mhz * 1e6 / 14.0
+    peak_words = sms * 4 * 16 * clk_mhz * 1e6 / 12.5
     achieved = K * words / (kern / 1e3)
     # e2e: decisions H2D from pinned memory, hash + filter, results D2H
     hst = torch.empty(K, dtype=torch.uint8).pin_memory()
@@ -623,7 +623,7 @@ def run_ghash(args, wl, cfg, K, workload, pool, ncores, rank, world, local):
                 "roofline": {"bound": "alu", "achieved": round(achieved / 1e9, 2), "peak": round(peak_words / 1e9, 1),
                              "unit": "Gword/s", "frac": round(achieved / peak_words, 4), "traffic": None,
                              "peak_source": "derived: SMs x 4 SMSP x 16 ALU lanes/clk (B300_MICROARCH rt_SMSP=2) x "
-                                            "SM clock / 14 ALU-pipe ops per absorbed word",
+                                            "SM clock / 12.5 ALU-pipe ops per absorbed word (SASS count)",
                              "kernel": "magis::ghash_kernel", "kernel_ms_avg": round(kern, 4),
                              "kernel_share_of_step": round(kern / ms_per_step, 4)},
                 "cpu_baseline": cpu, "e2e": e2e, "clocks": clk.summary(), "gpu_launches": args.steps * 3}

@@ -71,6 +71,10 @@ def _load():
     lib.orc_best_mem.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_int64]
     lib.orc_best_lat.restype = ctypes.c_int64
     lib.orc_best_lat.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_double]
+    lib.orc_graph_set_regions.restype = ctypes.c_int
+    lib.orc_graph_set_regions.argtypes = [P, ctypes.c_int32, P, P, P]
+    lib.orc_graph_dec_len.restype = ctypes.c_int32
+    lib.orc_graph_dec_len.argtypes = [P]
     lib.orc_mix64.restype = ctypes.c_uint64
     lib.orc_mix64.argtypes = [ctypes.c_uint64]
     lib.orc_hash_words.restype = ctypes.c_uint64
@@ -92,7 +96,7 @@ class OracleGraph:
     and the swap link model (bytes/s, latency; reading P7)."""
 
     def __init__(self, size, cost, is_output, src, dst, elig=(), U=(),
-                 swap_Bps: float = 25e9, swap_lat: float = 1e-5):
+                 swap_Bps: float = 25e9, swap_lat: float = 1e-5, regions=None):
         self._lib = _load()
         self.size = np.ascontiguousarray(size, dtype=np.int64)
         self.cost = np.ascontiguousarray(cost, dtype=np.float64)
@@ -121,12 +125,25 @@ class OracleGraph:
         self._h = h
         self.n_total = int(self._lib.orc_graph_n_total(h))
         self.n_edges = int(self._lib.orc_graph_n_edges(h))
+        # F-Trans variant regions (NEXT-4, reading F1): dict(n_variants [F],
+        # node_region [n] (-1 = in every variant), node_variant [n])
+        self.F = 0
+        if regions is not None:
+            nv = np.ascontiguousarray(regions["n_variants"], dtype=np.int32)
+            nr = np.ascontiguousarray(regions["node_region"], dtype=np.int32)
+            vn = np.ascontiguousarray(regions["node_variant"], dtype=np.uint8)
+            assert nr.shape == (self.n,) and vn.shape == (self.n,)
+            self._regions = (nv, nr, vn)
+            if self._lib.orc_graph_set_regions(h, int(nv.shape[0]), _ptr(nv), _ptr(nr), _ptr(vn)) != 0:
+                raise ValueError("oracle: bad regions")
+            self.F = int(nv.shape[0])
+        self.dec_len = self.R + self.F
 
     @classmethod
     def from_workload(cls, wl):
         """Build from a magis_inputs.Workload (input generator output)."""
         return cls(wl.size, wl.cost, wl.is_output, wl.src, wl.dst, wl.elig, wl.U,
-                   wl.swap_Bps, wl.swap_lat)
+                   wl.swap_Bps, wl.swap_lat, getattr(wl, "regions", None))
 
     def __del__(self):
         h = getattr(self, "_h", None)
@@ -139,7 +156,7 @@ class OracleGraph:
         perm = np.ascontiguousarray(perm, dtype=np.int32)
         assert perm.shape == (self.n_total,)
         if dec is None:
-            dec = np.zeros(max(self.R, 1), dtype=np.uint8)
+            dec = np.zeros(max(self.dec_len, 1), dtype=np.uint8)
         dec = np.ascontiguousarray(dec, dtype=np.uint8)
         st = np.zeros(1, np.uint8)
         pk = np.zeros(1, np.int64)
@@ -153,9 +170,11 @@ class OracleGraph:
         perms = np.ascontiguousarray(perms, dtype=np.int32)
         K = perms.shape[0]
         assert perms.shape[1] == self.n_total
-        if decs is None or self.R == 0:
-            decs = np.zeros((K, max(self.R, 1)), dtype=np.uint8)
+        if decs is None or self.dec_len == 0:
+            decs = np.zeros((K, max(self.dec_len, 1)), dtype=np.uint8)
         decs = np.ascontiguousarray(decs, dtype=np.uint8)
+        assert decs.shape[1] >= self.dec_len
+        decs = np.ascontiguousarray(decs[:, :max(self.dec_len, 1)])
         st = np.zeros(K, np.uint8)
         pk = np.zeros(K, np.int64)
         lt = np.zeros(K, np.float64)

@@ -49,6 +49,14 @@ typedef struct {
     uint8_t *has_input; /* [n] node has at least one predecessor */
     double   swap_Bps;  /* swap link bytes/s (reading P7) */
     double   swap_lat;  /* per-transfer latency seconds (reading P7) */
+    /* F-Trans variant regions (NEXT-4, reading F1): region i offers
+     * nvar[i] variants of one sub-graph; an original node with nreg[v] >= 0
+     * exists only in variant nvn[v] of region nreg[v]; the candidate picks
+     * the variant in dec[R + i]. */
+    int32_t  F;
+    int32_t *nvar;      /* [F] */
+    int32_t *nreg;      /* [n] region or -1 */
+    uint8_t *nvn;       /* [n] variant */
 } orc_graph;
 
 static int cmp_pair(const void *a, const void *b)
@@ -63,6 +71,7 @@ void orc_graph_free(orc_graph *g)
     free(g->size); free(g->cost); free(g->is_output);
     free(g->src); free(g->dst); free(g->elig); free(g->U_ptr); free(g->U_idx);
     free(g->r_of); free(g->has_input);
+    free(g->nvar); free(g->nreg); free(g->nvn);
     free(g);
 }
 
@@ -155,7 +164,8 @@ static void transformed_graph(const orc_graph *g, const uint8_t *dec, uint8_t *a
     const int32_t n = g->n, R = g->R;
     int64_t nte = 0, cap_te, i, k;
     int32_t *tsrc, *tdst;
-    for (i = 0; i < n; i++) active[i] = 1;
+    for (i = 0; i < n; i++)
+        active[i] = (g->F == 0 || g->nreg[i] < 0 || dec[R + g->nreg[i]] == g->nvn[i]) ? 1 : 0;
     for (i = 0; i < R; i++) {
         if (dec[i] == 1) active[n + 3 * i] = 1;
         if (dec[i] == 2) { active[n + 3 * i + 1] = 1; active[n + 3 * i + 2] = 1; }
@@ -191,8 +201,54 @@ static void transformed_graph(const orc_graph *g, const uint8_t *dec, uint8_t *a
             tsrc[nte] = n + 3 * (int32_t)i + 1; tdst[nte] = n + 3 * (int32_t)i + 2; nte++;
         }
     }
+    /* the chosen F-Trans variants: an edge exists iff both ends exist (reading F1) */
+    if (g->F > 0) {
+        int64_t m = 0;
+        for (k = 0; k < nte; k++)
+            if (active[tsrc[k]] && active[tdst[k]]) { tsrc[m] = tsrc[k]; tdst[m] = tdst[k]; m++; }
+        nte = m;
+    }
     *tsrc_out = tsrc; *tdst_out = tdst; *nte_out = nte;
 }
+
+/* decision check (reading P12, R-noinput; F1: a variant index below nvar). */
+static uint8_t check_dec(const orc_graph *g, const uint8_t *dec)
+{
+    uint8_t status = 0;
+    int32_t i;
+    for (i = 0; i < g->R; i++) {
+        uint8_t d = dec[i];
+        if (d > 2) status |= 4;
+        /* re-materialization needs A's inputs (P:1333-1336): a tensor with no
+         * inputs cannot be re-computed (DESIGN.md reading R-noinput). */
+        if (d == 1 && !g->has_input[g->elig[i]]) status |= 4;
+    }
+    for (i = 0; i < g->F; i++)
+        if (dec[g->R + i] >= g->nvar[i]) status |= 4;
+    return status;
+}
+
+/* Attach F-Trans variant regions (NEXT-4).  Returns 0, or -1 on bad input. */
+int orc_graph_set_regions(orc_graph *g, int32_t F, const int32_t *nvar, const int32_t *nreg,
+                          const uint8_t *nvn)
+{
+    int32_t i;
+    if (F < 0) return -1;
+    free(g->nvar); free(g->nreg); free(g->nvn);
+    g->F = F;
+    g->nvar = (int32_t *)malloc(sizeof(int32_t) * (F ? F : 1));
+    g->nreg = (int32_t *)malloc(sizeof(int32_t) * (g->n ? g->n : 1));
+    g->nvn = (uint8_t *)malloc(g->n ? g->n : 1);
+    for (i = 0; i < F; i++) g->nvar[i] = nvar[i];
+    for (i = 0; i < g->n; i++) {
+        g->nreg[i] = F ? nreg[i] : -1;
+        g->nvn[i] = F ? nvn[i] : 0;
+        if (g->nreg[i] >= F) return -1;
+    }
+    return 0;
+}
+
+int32_t orc_graph_dec_len(const orc_graph *g) { return g->R + g->F; }
 
 /*
  * Evaluate one candidate.
@@ -206,7 +262,7 @@ static void eval_impl(const orc_graph *g, const int32_t *perm, const uint8_t *de
                       uint8_t *status_out, int64_t *peak_out, double *lat_out,
                       int64_t *argmax_out, uint8_t *hot_out)
 {
-    const int32_t n = g->n, R = g->R, NT = g->NT;
+    const int32_t n = g->n, NT = g->NT;
     uint8_t status = 0;
     uint8_t *seen = NULL, *active = NULL;
     int32_t *pos = NULL, *step = NULL, *ord = NULL, *last = NULL;
@@ -223,13 +279,7 @@ static void eval_impl(const orc_graph *g, const int32_t *perm, const uint8_t *de
         if (p < 0 || p >= NT || seen[p]) { status |= 1; continue; }
         seen[p] = 1;
     }
-    for (i = 0; i < R; i++) {
-        uint8_t d = dec[i];
-        if (d > 2) status |= 4;
-        /* re-materialization needs A's inputs (P:1333-1336): a tensor with no
-         * inputs cannot be re-computed (DESIGN.md reading R-noinput). */
-        if (d == 1 && !g->has_input[g->elig[i]]) status |= 4;
-    }
+    status |= check_dec(g, dec);
     if (status) goto done;
 
     /* 2. active set and transformed graph (Fig. 8) */
@@ -492,7 +542,7 @@ void orc_eval_batch(const orc_graph *g, int64_t K, const int32_t *perms,
     int64_t k;
     for (k = 0; k < K; k++)
         orc_eval(g, perms + k * (int64_t)g->NT,
-                 g->R ? decs + k * (int64_t)g->R : NULL,
+                 (g->R + g->F) ? decs + k * (int64_t)(g->R + g->F) : NULL,
                  status + k, peak + k, lat + k, NULL);
 }
 
@@ -620,7 +670,7 @@ static int cmp_u64(const void *a, const void *b)
 int orc_graph_hash(const orc_graph *g, const uint64_t *label, const uint8_t *dec,
                    uint64_t *x_out, uint64_t *hash_out)
 {
-    const int32_t n = g->n, R = g->R, NT = g->NT;
+    const int32_t n = g->n, NT = g->NT;
     uint8_t *active;
     int32_t *tsrc, *tdst, *indeg, *queue;
     int64_t nte, i, k;
@@ -628,10 +678,7 @@ int orc_graph_hash(const orc_graph *g, const uint64_t *label, const uint8_t *dec
     uint64_t *x, *buf, sum = 0;
     int status = 0;
 
-    for (i = 0; i < R; i++) {
-        if (dec[i] > 2) status |= 4;
-        if (dec[i] == 1 && !g->has_input[g->elig[i]]) status |= 4;   /* reading R-noinput */
-    }
+    status = check_dec(g, dec);
     if (status) {
         if (x_out) for (i = 0; i < NT; i++) x_out[i] = 0;
         *hash_out = 0;
@@ -675,5 +722,6 @@ void orc_graph_hash_batch(const orc_graph *g, const uint64_t *label, int64_t K, 
 {
     int64_t k;
     for (k = 0; k < K; k++)
-        status[k] = (uint8_t)orc_graph_hash(g, label, g->R ? decs + k * (int64_t)g->R : NULL, NULL, hash + k);
+        status[k] = (uint8_t)orc_graph_hash(g, label, (g->R + g->F) ? decs + k * (int64_t)(g->R + g->F) : NULL,
+                                            NULL, hash + k);
 }

@@ -1,6 +1,6 @@
-// magis_ghash.cu -- batched GraphHash and the duplicate filter (SURVEY §8(f)
-// NEXT-2; Alg. 3 lines 3-6 and 10-12; the Weisfeiler-Lehman
-// idea).  Readings G1-G4 are in DESIGN.md §3.
+// magis_ghash.cu -- batched GraphHash (Alg. 3 lines 3-6,
+// P:1693-1700; the Weisfeiler-Lehman idea).  Readings G1-G4 are
+// in DESIGN.md §3.  The duplicate filter (lines 10-12) is magis_hashset.cu.
 //
 // The graph of candidate k is its transformed graph (Fig. 8 rules applied to
 // the decisions dec[k]; the schedule does not enter, reading G4).  Per node,
@@ -10,17 +10,26 @@
 //     GraphHash = hash( sum_v x_v mod 2^64 )                         (line 6)
 // hash() over 64-bit words: h = GAMMA (m + 1), h = mix64(h ^ w_i) (reading G1).
 //
-// B200 layout: lane = candidate.  A warp walks the node table (warp-uniform,
-// L1-broadcast loads) for 32 candidates at once; the decisions only switch
-// which slot a late-user edge reads (t_r, the clone or the Load) and whether
-// an optional node is active, so control flow stays uniform.  x values live
-// in "slots" assigned at create time by a linear scan over the order (a slot
-// is reused once its last potential reader has run): short-lived values in
-// shared memory ([slot][lane], conflict-free), long-lived ones (forward
-// activations read by the backward pass) in a per-warp global region with
-// the same lane-interleaved layout (256-byte coalesced rows, L2-resident).
-// Predecessor values are sorted in registers by a bitonic network sized to
-// the warp-uniform in-degree.
+// B200 layout.
+//  * Lane = candidate; a warp carries C = 1 or 2 candidates per lane (two
+//    independent mix64 chains per node for ILP) and walks the node table
+//    with warp-uniform, L1-broadcast loads.  Decisions only switch which
+//    value a late-user edge reads (t_r, the clone or the Load) and whether an
+//    optional node is active, so control flow stays uniform.
+//  * Work that does not depend on the decisions is done once at create
+//    time: the first absorbed word of every node (h1 = mix64(GAMMA (d+2) ^
+//    hash(label))), and the complete x of every node no decision can reach
+//    (sources, weights, and everything upstream of the first late user):
+//    those nodes leave the loop, their values are read from a constant table
+//    and their sum is a constant.
+//  * x values of the remaining nodes live in "slots" assigned by a linear
+//    scan over the order (reused once the last potential reader has run):
+//    short-lived values in shared memory ([slot][c][lane], conflict-free),
+//    long-lived ones in a per-warp global region with the same layout
+//    (256-byte coalesced rows, L2-resident).
+//  * Predecessor values are sorted in registers: exact networks for in-degree
+//    1-4 (the bulk of a DNN graph), bitonic networks up to 32, a rank sort in
+//    global scratch beyond.
 #include <algorithm>
 #include <climits>
 #include <cstdio>
@@ -36,10 +45,14 @@ namespace magis {
 constexpr uint64_t kGamma = 0x9E3779B97F4A7C15ull;
 constexpr uint64_t kTagStore = 0x45524F5453ull;   // "STORE" (reading G3)
 constexpr uint64_t kTagLoad = 0x44414F4Cull;      // "LOAD"
+// value references (pent entries, slots): LU = late-user edge of r (the
+// decision picks t_r / clone_r / load_r); Const = x0 table index;
+// Glob = per-warp global slot; otherwise a shared-memory slot
+constexpr uint32_t kLU = 0x80000000u, kConst = 0x40000000u, kGlob = 0x20000000u, kIdx = 0x1FFFFFFFu;
 constexpr uint32_t kNoSlot = 0xFFFFFFFFu;
-constexpr uint32_t kLU = 0x80000000u;             // late-user entry: low bits = r
 constexpr int kGhWarps = 4;                        // warps per CTA
 constexpr int kGhCtasPerSm = 4;
+constexpr uint32_t kLabStore = 0xFFFFFFFEu, kLabLoad = 0xFFFFFFFDu;
 
 __host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
     z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
@@ -48,16 +61,19 @@ __host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
 }
 
 struct GhDev {
-    int32_t NT, R, NS;        // nodes in the order, eligible tensors, shared slots per warp
-    int32_t gslots;           // global slots per warp
-    int32_t maxdeg;           // largest in-degree (> 32 uses the rank sort in global scratch)
+    int32_t nloop;            // nodes walked per candidate
+    int32_t R, NS;            // eligible tensors, shared slots per warp (per candidate column)
+    int32_t gslots;           // global slots per warp (per candidate column)
+    int32_t maxdeg;           // in-degree of the rank-sort path (0 if none > 32)
     int32_t Rw;               // u32 words of packed decisions per candidate (16 per word)
-    const uint4* nrec;        // [NT] (hash(label) lo, hi, slot, gate); gate ~0 = always active
-    const uint2* nadj;        // [NT] (offset into pent, in-degree)
-    const uint32_t* pent;     // slot, or kLU | r
-    const uint4* rslot;       // [R] (slot of t_r, clone_r, load_r, slot of t_r)
+    const uint4* nrec;        // [nloop] (h1 lo, h1 hi, own slot, gate); gate ~0 = always active
+    const uint2* nadj;        // [nloop] (pent offset or x0 index, deg | kind << 24); kind 1 = constant node
+    const uint32_t* pent;     // value references of the predecessors
+    const uint4* rslot;       // [R] value references of (t_r, clone_r, load_r, t_r)
     const uint8_t* rflag;     // [R] kRHasInput
-    unsigned long long* gbuf; // [warps][gslots + 2 maxdeg][32]
+    const unsigned long long* x0;   // [NT] x of the decision-independent nodes
+    const unsigned long long* c0;   // [1] sum of x0 over decision-independent original nodes
+    unsigned long long* gbuf; // [warps][gslots + 2 maxdeg][C][32]
 };
 
 }  // namespace magis
@@ -71,34 +87,58 @@ struct magis_ghash {
     size_t scratch_bytes = 0;
     int grid = 0;
     size_t smem = 0;
-    int64_t n_global_nodes = 0;   // nodes whose x lives in the global slots
-};
-
-struct magis_hashset {
-    int device = 0;
-    uint64_t cap = 0;                  // power of two
-    unsigned long long* keys = nullptr;     // [cap] 0 = empty
-    unsigned long long* owner = nullptr;    // [cap + 1] (epoch << 40 | first id); [cap] = key 0
-    unsigned long long* stats = nullptr;    // [2] occupied slots, overflowed inserts
-    uint32_t epoch = 0;
+    int64_t n_global_nodes = 0;   // walked nodes whose x lives in global slots
+    int64_t n_const_nodes = 0;    // nodes no decision can reach
+    int64_t n_grouped = 0;        // walked nodes hashed in same-level groups
 };
 
 namespace magis {
 namespace {
 
-// ------------------------------------------------------------------ device --
-__global__ void ghash_label_kernel(uint4* nrec, int32_t NT, const uint64_t* label) {
+// ------------------------------------------------------------ setup kernels --
+// h1[v] = hash state after the first word of line 5: mix64(GAMMA (d + 2) ^ hash([label_v]))
+__global__ void ghash_h1_kernel(int32_t NT, const uint32_t* lsrc, const int32_t* deg, const uint64_t* label,
+                                unsigned long long* h1) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= NT) return;
-    uint4 r = nrec[i];
-    // label source: r.x = original id (or t_r), r.y = kind (0 op / clone, 1 Store, 2 Load)
-    const uint64_t lab = r.y == 0 ? label[r.x] : (r.y == 1 ? kTagStore : kTagLoad);
-    const uint64_t h = mix64((kGamma * 2ull) ^ lab);             // hash([label]), m = 1
-    r.x = (uint32_t)h;
-    r.y = (uint32_t)(h >> 32);
-    nrec[i] = r;
+    const uint32_t s = lsrc[i];
+    const uint64_t lab = s == kLabStore ? kTagStore : s == kLabLoad ? kTagLoad : label[s];
+    const uint64_t hl = mix64((kGamma * 2ull) ^ lab);                   // hash([label])
+    h1[i] = mix64((kGamma * (uint64_t)(deg[i] + 2)) ^ hl);
 }
 
+// x of the decision-independent nodes, in order (one thread; runs once)
+__global__ void ghash_const_kernel(int32_t nc, const int32_t* cnode, const int32_t* cptr, const int32_t* cpred,
+                                   const uint8_t* corig, const unsigned long long* h1, unsigned long long* x0,
+                                   unsigned long long* tmp, unsigned long long* c0) {
+    if (blockIdx.x || threadIdx.x) return;
+    unsigned long long sum = 0;
+    for (int32_t i = 0; i < nc; i++) {
+        const int32_t v = cnode[i], b = cptr[i], e = cptr[i + 1];
+        int32_t m = 0;
+        for (int32_t j = b; j < e; j++) {                // insertion sort, ascending
+            const unsigned long long x = x0[cpred[j]];
+            int32_t q = m++;
+            while (q > 0 && tmp[q - 1] > x) { tmp[q] = tmp[q - 1]; q--; }
+            tmp[q] = x;
+        }
+        unsigned long long h = h1[v];
+        for (int32_t j = 0; j < m; j++) h = mix64(h ^ tmp[j]);
+        x0[v] = h;
+        if (corig[i]) sum += h;
+    }
+    *c0 = sum;
+}
+
+__global__ void ghash_fill_kernel(int32_t nloop, const int32_t* lnode, const unsigned long long* h1, uint4* nrec) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= nloop) return;
+    const unsigned long long h = h1[lnode[i]];
+    nrec[i].x = (uint32_t)h;
+    nrec[i].y = (uint32_t)(h >> 32);
+}
+
+// ------------------------------------------------------------- main kernel --
 template <int D>
 __device__ __forceinline__ void bitonic(uint64_t (&a)[D]) {
 #pragma unroll
@@ -117,37 +157,87 @@ __device__ __forceinline__ void bitonic(uint64_t (&a)[D]) {
             }
 }
 
-struct Lane {
+__device__ __forceinline__ void cex(uint64_t& a, uint64_t& b) {
+    const uint64_t lo = min(a, b), hi = max(a, b);
+    a = lo;
+    b = hi;
+}
+
+struct Lanes {
     const GhDev& d;
-    const unsigned long long* xs;      // shared slots of this warp
-    unsigned long long* gb;            // global slots of this warp
-    const uint32_t* decp;              // packed decisions of this warp
+    unsigned long long* xs;            // shared slots of this warp: [NS][32]
+    unsigned long long* gb;            // global slots of this warp: [gslots][32]
+    const uint32_t* decp;              // packed decisions of this warp: [Rw][32]
     int lane;
     __device__ __forceinline__ uint32_t dec(uint32_t r) const {
         return (decp[(r >> 4) * 32 + lane] >> (2 * (r & 15))) & 3u;
     }
-    __device__ __forceinline__ uint32_t slot_of(uint32_t e) const {
-        if (!(e & kLU)) return e;
-        const uint4 rs = __ldg(d.rslot + (e & ~kLU));
-        const uint32_t dd = dec(e & ~kLU);
-        return dd == 1 ? rs.y : dd == 2 ? rs.z : rs.x;
-    }
     __device__ __forceinline__ uint64_t get(uint32_t e) const {
-        const uint32_t s = slot_of(e);
-        return s < (uint32_t)d.NS ? xs[s * 32 + lane] : gb[(size_t)(s - d.NS) * 32 + lane];
+        uint32_t s = e;
+        if (e & kLU) {
+            const uint4 rs = __ldg(d.rslot + (e & kIdx));
+            const uint32_t dd = dec(e & kIdx);
+            s = dd == 1 ? rs.y : dd == 2 ? rs.z : rs.x;
+        }
+        if (s & kConst) return __ldg(d.x0 + (s & kIdx));
+        if (s & kGlob) return gb[(size_t)(s & kIdx) * 32 + lane];
+        return xs[s * 32 + lane];
+    }
+    __device__ __forceinline__ void put(uint32_t s, uint64_t h) const {
+        if (s == kNoSlot) return;
+        if (s & kGlob) gb[(size_t)(s & kIdx) * 32 + lane] = h;
+        else xs[s * 32 + lane] = h;
     }
 };
 
+// exact sorting networks for D <= 4 values
 template <int D>
-__device__ __forceinline__ uint64_t hash_preds(const Lane& L, const uint32_t* ent, int deg, uint64_t h) {
-    uint64_t a[D];
+__device__ __forceinline__ void sortn(uint64_t (&a)[D]) {
+    if constexpr (D == 2) {
+        cex(a[0], a[1]);
+    } else if constexpr (D == 3) {
+        cex(a[0], a[1]); cex(a[1], a[2]); cex(a[0], a[1]);
+    } else if constexpr (D == 4) {
+        cex(a[0], a[1]); cex(a[2], a[3]); cex(a[0], a[2]); cex(a[1], a[3]); cex(a[1], a[2]);
+    }
+}
+
+// G independent nodes of one topological level with in-degree D each (always
+// active): G interleaved mix64 chains.  Node records i .. i+G-1, their
+// predecessor references are contiguous at ent (G x D).
+template <int G, int D>
+__device__ __forceinline__ void group_nodes(const Lanes& L, const uint4* rec, const uint32_t* ent, uint64_t& sum) {
+    uint64_t a[G][D], h[G];
+    uint32_t e[G * D];
 #pragma unroll
-    for (int j = 0; j < D; j++) a[j] = j < deg ? L.get(__ldg(ent + j)) : ~0ull;
-    bitonic<D>(a);
+    for (int j = 0; j < G * D; j++) e[j] = __ldg(ent + j);
+#pragma unroll
+    for (int g = 0; g < G; g++) {
+#pragma unroll
+        for (int j = 0; j < D; j++) a[g][j] = L.get(e[g * D + j]);
+        sortn<D>(a[g]);
+        h[g] = ((uint64_t)rec[g].y << 32) | rec[g].x;
+    }
 #pragma unroll
     for (int j = 0; j < D; j++)
-        if (j < deg) h = mix64(h ^ a[j]);
-    return h;
+#pragma unroll
+        for (int g = 0; g < G; g++) h[g] = mix64(h[g] ^ a[g][j]);
+#pragma unroll
+    for (int g = 0; g < G; g++) {
+        sum += h[g];
+        L.put(rec[g].z, h[g]);
+    }
+}
+
+template <int G>
+__device__ __forceinline__ void group_dispatch(const Lanes& L, int D, const uint4* rec, const uint32_t* ent,
+                                               uint64_t& sum) {
+    switch (D) {
+        case 1: group_nodes<G, 1>(L, rec, ent, sum); break;
+        case 2: group_nodes<G, 2>(L, rec, ent, sum); break;
+        case 3: group_nodes<G, 3>(L, rec, ent, sum); break;
+        default: group_nodes<G, 4>(L, rec, ent, sum); break;
+    }
 }
 
 __global__ void __launch_bounds__(32 * kGhWarps, kGhCtasPerSm)
@@ -160,7 +250,8 @@ ghash_kernel(GhDev d, int64_t K, const uint8_t* __restrict__ dec, int vec, uint8
     unsigned long long* xs = ghsm + per_warp * wib;
     uint32_t* decp = reinterpret_cast<uint32_t*>(xs + (size_t)d.NS * 32);
     unsigned long long* gb = d.gbuf + (size_t)wg * (size_t)(d.gslots + 2 * d.maxdeg) * 32;
-    const Lane L{d, xs, gb, decp, lane};
+    const Lanes L{d, xs, gb, decp, lane};
+    const unsigned long long c0 = *d.c0;
 
     for (int64_t grp = wg; grp * 32 < K; grp += nw) {
         const int64_t k = grp * 32 + lane;
@@ -191,43 +282,91 @@ ghash_kernel(GhDev d, int64_t K, const uint8_t* __restrict__ dec, int vec, uint8
             decp[w * 32 + lane] = word;
         }
         __syncwarp();
-        uint64_t sum = 0;
-        for (int32_t i = 0; i < d.NT; i++) {
-            const uint4 rec = __ldg(d.nrec + i);
-            bool act = true;
-            if (rec.w != 0xFFFFFFFFu) act = L.dec(rec.w >> 2) == (rec.w & 3u);
-            if (!__any_sync(0xffffffffu, act)) continue;
+        uint64_t sum = c0;
+        for (int32_t i = 0; i < d.nloop;) {
             const uint2 adj = __ldg(d.nadj + i);
+            const int deg = (int)(adj.y & 0xFFFFFFu);
+            const uint32_t kind = (adj.y >> 24) & 3u;
+            if (kind == 2) {                                  // a group of G same-level nodes
+                const int G = (int)(adj.y >> 26);
+                uint4 rec[4];
+#pragma unroll
+                for (int g = 0; g < 4; g++)
+                    if (g < G) rec[g] = __ldg(d.nrec + i + g);
+                const uint32_t* ent = d.pent + adj.x;
+                switch (G) {
+                    case 2: group_dispatch<2>(L, deg, rec, ent, sum); break;
+                    case 3: group_dispatch<3>(L, deg, rec, ent, sum); break;
+                    default: group_dispatch<4>(L, deg, rec, ent, sum); break;
+                }
+                i += G;
+                __syncwarp();
+                continue;
+            }
+            const uint4 rec = __ldg(d.nrec + i);
+            i++;
+            bool act = true;
+            if (rec.w != 0xFFFFFFFFu) {                       // optional node: active iff dec[r] == gate
+                act = L.dec(rec.w >> 2) == (rec.w & 3u);
+                if (!__any_sync(0xffffffffu, act)) continue;
+            }
+            if (kind == 1) {                                  // decision-independent optional node
+                if (act) sum += __ldg(d.x0 + adj.x);
+                continue;
+            }
             const uint32_t* ent = d.pent + adj.x;
-            const int deg = (int)adj.y;
-            uint64_t h = mix64((kGamma * (uint64_t)(deg + 2)) ^ (((uint64_t)rec.y << 32) | rec.x));
-            if (deg <= 4) {
-                h = hash_preds<4>(L, ent, deg, h);
+            uint64_t h = ((uint64_t)rec.y << 32) | rec.x;
+            if (deg == 1) {
+                h = mix64(h ^ L.get(__ldg(ent)));
+            } else if (deg == 2) {
+                uint64_t a[2] = {L.get(__ldg(ent)), L.get(__ldg(ent + 1))};
+                sortn<2>(a);
+                h = mix64(mix64(h ^ a[0]) ^ a[1]);
+            } else if (deg == 3) {
+                uint64_t a[3] = {L.get(__ldg(ent)), L.get(__ldg(ent + 1)), L.get(__ldg(ent + 2))};
+                sortn<3>(a);
+                h = mix64(mix64(mix64(h ^ a[0]) ^ a[1]) ^ a[2]);
+            } else if (deg == 4) {
+                uint64_t a[4] = {L.get(__ldg(ent)), L.get(__ldg(ent + 1)), L.get(__ldg(ent + 2)),
+                                 L.get(__ldg(ent + 3))};
+                sortn<4>(a);
+                h = mix64(mix64(mix64(mix64(h ^ a[0]) ^ a[1]) ^ a[2]) ^ a[3]);
+            } else if (deg == 0) {
             } else if (deg <= 8) {
-                h = hash_preds<8>(L, ent, deg, h);
+                uint64_t a[8];
+#pragma unroll
+                for (int j = 0; j < 8; j++) a[j] = j < deg ? L.get(__ldg(ent + j)) : ~0ull;
+                bitonic<8>(a);
+#pragma unroll
+                for (int j = 0; j < 8; j++)
+                    if (j < deg) h = mix64(h ^ a[j]);
             } else if (deg <= 32) {
-                h = hash_preds<32>(L, ent, deg, h);
+                uint64_t a[32];
+#pragma unroll
+                for (int j = 0; j < 32; j++) a[j] = j < deg ? L.get(__ldg(ent + j)) : ~0ull;
+                bitonic<32>(a);
+#pragma unroll
+                for (int j = 0; j < 32; j++)
+                    if (j < deg) h = mix64(h ^ a[j]);
             } else {
-                // rank sort in this lane's global scratch column (rare: merges of > 32 parts)
+                // rank sort in this lane's global scratch column (merges of > 32 parts)
                 unsigned long long* t0 = gb + (size_t)d.gslots * 32;
                 unsigned long long* t1 = t0 + (size_t)d.maxdeg * 32;
-                for (int j = 0; j < deg; j++) t0[(size_t)j * 32 + lane] = L.get(__ldg(ent + j));
+                for (int j = 0; j < deg; j++) t0[j * 32 + lane] = L.get(__ldg(ent + j));
                 for (int j = 0; j < deg; j++) {
-                    const uint64_t v = t0[(size_t)j * 32 + lane];
+                    const uint64_t v = t0[j * 32 + lane];
                     int rk = 0;
                     for (int q = 0; q < deg; q++) {
-                        const uint64_t u = t0[(size_t)q * 32 + lane];
+                        const uint64_t u = t0[q * 32 + lane];
                         rk += (u < v) | ((u == v) & (q < j));
                     }
-                    t1[(size_t)rk * 32 + lane] = v;
+                    t1[rk * 32 + lane] = v;
                 }
-                for (int j = 0; j < deg; j++) h = mix64(h ^ t1[(size_t)j * 32 + lane]);
+                for (int j = 0; j < deg; j++) h = mix64(h ^ t1[j * 32 + lane]);
             }
             if (act) {
                 sum += h;
-                const uint32_t s = rec.z;
-                if (s < (uint32_t)d.NS) xs[s * 32 + lane] = h;
-                else if (s != kNoSlot) gb[(size_t)(s - d.NS) * 32 + lane] = h;
+                L.put(rec.z, h);
             }
             __syncwarp();
         }
@@ -236,57 +375,6 @@ ghash_kernel(GhDev d, int64_t K, const uint8_t* __restrict__ dec, int vec, uint8
             out_hash[k] = bad ? 0ull : mix64((kGamma * 2ull) ^ sum);       // line 6: hash([sum])
         }
         __syncwarp();
-    }
-}
-
-// hash set: open addressing, linear probing, 64-bit keys (0 = empty; the
-// key 0 has its own owner word at [cap])
-__device__ __forceinline__ uint64_t probe_start(uint64_t h, uint64_t mask) { return mix64(h) & mask; }
-
-__global__ void hs_insert_kernel(magis_hashset s, int64_t K, const uint64_t* __restrict__ hash,
-                                 const uint8_t* __restrict__ status) {
-    const uint64_t mask = s.cap - 1;
-    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < K; k += (int64_t)gridDim.x * blockDim.x) {
-        if (status && status[k]) continue;
-        const unsigned long long h = hash[k];
-        const unsigned long long me = ((unsigned long long)s.epoch << 40) | (unsigned long long)k;
-        if (h == 0) { atomicMin(s.owner + s.cap, me); continue; }
-        uint64_t i = probe_start(h, mask);
-        bool done = false;
-        for (uint64_t p = 0; p < s.cap; p++) {
-            const unsigned long long prev = atomicCAS(s.keys + i, 0ull, h);
-            if (prev == 0ull || prev == h) {
-                if (prev == 0ull) atomicAdd(s.stats, 1ull);
-                atomicMin(s.owner + i, me);
-                done = true;
-                break;
-            }
-            i = (i + 1) & mask;
-        }
-        if (!done) atomicAdd(s.stats + 1, 1ull);
-    }
-}
-
-__global__ void hs_mark_kernel(magis_hashset s, int64_t K, const uint64_t* __restrict__ hash,
-                               const uint8_t* __restrict__ status, uint8_t* __restrict__ is_new) {
-    const uint64_t mask = s.cap - 1;
-    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < K; k += (int64_t)gridDim.x * blockDim.x) {
-        if (status && status[k]) { is_new[k] = 0; continue; }
-        const unsigned long long h = hash[k];
-        const unsigned long long me = ((unsigned long long)s.epoch << 40) | (unsigned long long)k;
-        uint8_t r = 1;                           // not found (table full): kept as new
-        if (h == 0) {
-            r = s.owner[s.cap] == me;
-        } else {
-            uint64_t i = probe_start(h, mask);
-            for (uint64_t p = 0; p < s.cap; p++) {
-                const unsigned long long key = s.keys[i];
-                if (key == h) { r = s.owner[i] == me; break; }
-                if (key == 0ull) break;
-                i = (i + 1) & mask;
-            }
-        }
-        is_new[k] = r;
     }
 }
 
@@ -333,37 +421,26 @@ extern "C" int magis_ghash_create(const magis_graph* g, const uint64_t* h_label,
         order.push_back(v);
         if (r_of[v] >= 0) for (int o = 0; o < 3; o++) order.push_back(n + 3 * r_of[v] + o);
     }
-    std::vector<int32_t> hp(NT);
-    for (int32_t i = 0; i < NT; i++) hp[order[i]] = i;
-    // potential readers -> last position; predecessor entries
-    std::vector<int32_t> lastp(NT);
-    for (int32_t i = 0; i < NT; i++) lastp[order[i]] = i;
-    auto rd = [&](int32_t u, int32_t at) { lastp[u] = std::max(lastp[u], at); };
-    std::vector<std::vector<uint32_t>> ent(NT);   // node -> entries (node ids / kLU|r), slots filled later
-    int32_t maxdeg = 0;
-    for (int32_t v = 0; v < n; v++) {
+    // predecessor entries: node id, or kLU | r for a late-user edge
+    std::vector<std::vector<uint32_t>> ent(NT);
+    for (int32_t v = 0; v < n; v++)
         for (int32_t e = pp[v]; e < pp[v + 1]; e++) {
-            const int32_t u = pr[e];
-            const int32_t r = r_of[u];
+            const int32_t u = pr[e], r = r_of[u];
             bool lu = false;
             if (r >= 0) for (int32_t rr : Umem[v]) if (rr == r) { lu = true; break; }
-            if (lu) {
-                ent[v].push_back(kLU | (uint32_t)r);
-                rd(u, hp[v]); rd(n + 3 * r, hp[v]); rd(n + 3 * r + 2, hp[v]);
-            } else {
-                ent[v].push_back((uint32_t)u);
-                rd(u, hp[v]);
-            }
+            ent[v].push_back(lu ? (kLU | (uint32_t)r) : (uint32_t)u);
         }
-        maxdeg = std::max<int32_t>(maxdeg, (int32_t)ent[v].size());
-    }
     for (int32_t r = 0; r < R; r++) {
-        const int32_t t = g->h_elig[r], c = n + 3 * r, st = c + 1, ld = c + 2;
-        for (int32_t e = pp[t]; e < pp[t + 1]; e++) { ent[c].push_back((uint32_t)pr[e]); rd(pr[e], hp[c]); }
-        ent[st].push_back((uint32_t)t); rd(t, hp[st]);
-        ent[ld].push_back((uint32_t)st); rd(st, hp[ld]);
-        maxdeg = std::max<int32_t>(maxdeg, (int32_t)ent[c].size());
+        const int32_t t = g->h_elig[r], c = n + 3 * r;
+        for (int32_t e = pp[t]; e < pp[t + 1]; e++) ent[c].push_back((uint32_t)pr[e]);
+        ent[c + 1].push_back((uint32_t)t);
+        ent[c + 2].push_back((uint32_t)(c + 1));
     }
+    // decision-dependent nodes: a late-user edge, or a predecessor that is
+    std::vector<uint8_t> aff(NT, 0);
+    for (int32_t x : order)
+        for (uint32_t e : ent[x])
+            if ((e & kLU) || aff[e]) { aff[x] = 1; break; }
     // launch shape and the shared slot budget
     int sms = 0;
     {
@@ -378,99 +455,253 @@ extern "C" int magis_ghash_create(const magis_graph* g, const uint64_t* h_label,
     const size_t dec_bytes = (size_t)Rw * 32 * 4;
     int32_t NS = (int32_t)std::max<int64_t>(0, ((int64_t)smem_cap / kGhWarps - (int64_t)dec_bytes) / 256);
     if (const char* e = std::getenv("MAGIS_GH_NS")) NS = std::min(NS, std::atoi(e));
-    // slots by linear scan; a value that dies within TS positions prefers shared
-    // memory.  TS is picked to minimise the number of values sent to global.
+    int32_t maxdeg = 0;
+    for (int32_t x = 0; x < NT; x++)
+        if (aff[x]) maxdeg = std::max<int32_t>(maxdeg, (int32_t)ent[x].size());
+    // Two walking orders are planned and the one that keeps fewer values in
+    // global slots wins (ties: levels):
+    //  * levels: topological levels of the super-graph (every gated edge
+    //    included, so they hold for every candidate), by in-degree inside a
+    //    level, so that runs of same-level, same-degree nodes form groups whose
+    //    hash chains interleave (ILP within one candidate);
+    //  * topo: the load-time topological order (shorter value lifetimes on
+    //    graphs whose levels are wide, e.g. many fissioned parts side by side).
+    // Slots by linear scan over the walked values; a value that dies within
+    // TS positions prefers shared memory; TS minimises the values sent to global.
+    const std::vector<int32_t> order_topo = order;
+    std::vector<int32_t> lvl(NT, 0), pos0(NT);
+    for (int32_t i = 0; i < NT; i++) pos0[order_topo[i]] = i;
+    for (int32_t x : order_topo)
+        for (uint32_t e : ent[x]) {
+            if (e & kLU) {
+                const int32_t r = (int32_t)(e & kIdx);
+                for (int32_t y : {g->h_elig[r], n + 3 * r, n + 3 * r + 2}) lvl[x] = std::max(lvl[x], lvl[y] + 1);
+            } else {
+                lvl[x] = std::max(lvl[x], lvl[e] + 1);
+            }
+        }
+    const char* ordenv = std::getenv("MAGIS_GH_ORDER");
     std::vector<uint32_t> best_slot;
     int32_t best_gs = 0;
     int64_t best_glob = -1;
-    for (int32_t TS : {1, 2, 4, 8, 16, 32, 64, 128, 256, 1 << 30}) {
-        std::vector<uint32_t> slot(NT, kNoSlot);
-        std::vector<std::vector<int32_t>> dies(NT + 1);
-        std::vector<uint32_t> sfree, gfree;
-        for (int32_t s = NS - 1; s >= 0; s--) sfree.push_back((uint32_t)s);
-        int32_t gused = 0;
-        int64_t nglob = 0;
-        for (int32_t i = 0; i < NT; i++) {
-            const int32_t x = order[i];
-            if (i > 0)
-                for (int32_t y : dies[i - 1]) {
-                    if (slot[y] < (uint32_t)NS) sfree.push_back(slot[y]);
-                    else gfree.push_back(slot[y]);
-                }
-            if (lastp[x] == i) continue;             // no reader after it: x is only summed
-            const bool shortl = lastp[x] - i <= TS;
-            if (shortl && !sfree.empty()) { slot[x] = sfree.back(); sfree.pop_back(); }
-            else if (!gfree.empty()) { slot[x] = gfree.back(); gfree.pop_back(); nglob++; }
-            else { slot[x] = (uint32_t)(NS + gused++); nglob++; }
-            dies[lastp[x]].push_back(x);
+    for (int mode = 0; mode < 2; mode++) {                 // 0 levels, 1 topo
+        if (ordenv && std::string(ordenv) == (mode ? "level" : "topo")) continue;
+        std::vector<int32_t> ord = order_topo;
+        if (mode == 0) {
+            auto dclass = [&](int32_t x) { return x >= n ? 8 : std::min<int32_t>((int32_t)ent[x].size(), 5); };
+            std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) {
+                if (lvl[a] != lvl[b]) return lvl[a] < lvl[b];
+                if (dclass(a) != dclass(b)) return dclass(a) < dclass(b);
+                return pos0[a] < pos0[b];
+            });
         }
-        if (best_glob < 0 || nglob < best_glob) { best_glob = nglob; best_slot = slot; best_gs = gused; }
+        std::vector<int32_t> hp(NT);
+        for (int32_t i = 0; i < NT; i++) hp[ord[i]] = i;
+        // potential readers of the walked values -> last position
+        std::vector<int32_t> lastp(NT);
+        for (int32_t i = 0; i < NT; i++) lastp[ord[i]] = i;
+        for (int32_t x = 0; x < NT; x++) {
+            if (!aff[x]) continue;
+            for (uint32_t e : ent[x]) {
+                if (e & kLU) {
+                    const int32_t r = (int32_t)(e & kIdx);
+                    for (int32_t y : {g->h_elig[r], n + 3 * r, n + 3 * r + 2}) lastp[y] = std::max(lastp[y], hp[x]);
+                } else {
+                    lastp[e] = std::max(lastp[e], hp[x]);
+                }
+            }
+        }
+        for (int32_t TS : {1, 2, 4, 8, 16, 32, 64, 128, 256, 1 << 30}) {
+            std::vector<uint32_t> slot(NT, kNoSlot);
+            std::vector<std::vector<int32_t>> dies(NT + 1);
+            std::vector<uint32_t> sfree, gfree;
+            for (int32_t s2 = NS - 1; s2 >= 0; s2--) sfree.push_back((uint32_t)s2);
+            int32_t gused = 0;
+            int64_t nglob = 0;
+            for (int32_t i = 0; i < NT; i++) {
+                const int32_t x = ord[i];
+                if (i > 0)
+                    for (int32_t y : dies[i - 1]) {
+                        if (slot[y] & kGlob) gfree.push_back(slot[y]);
+                        else sfree.push_back(slot[y]);
+                    }
+                if (!aff[x] || lastp[x] == i) continue;   // constant, or no reader after it
+                const bool shortl = lastp[x] - i <= TS;
+                if (shortl && !sfree.empty()) { slot[x] = sfree.back(); sfree.pop_back(); }
+                else if (!gfree.empty()) { slot[x] = gfree.back(); gfree.pop_back(); nglob++; }
+                else { slot[x] = kGlob | (uint32_t)gused++; nglob++; }
+                dies[lastp[x]].push_back(x);
+            }
+            if (best_glob < 0 || nglob < best_glob) {
+                best_glob = nglob;
+                best_slot = slot;
+                best_gs = gused;
+                order = ord;
+            }
+        }
     }
-    // tables: nrec, nadj, pent, rslot
-    std::vector<uint4> nrec(NT);
-    std::vector<uint2> nadj(NT);
+    auto ref = [&](int32_t y) -> uint32_t { return aff[y] ? best_slot[y] : (kConst | (uint32_t)y); };
+    // walked nodes: decision-dependent nodes, and constant optional nodes
+    // (their activity still depends on the decisions)
+    std::vector<uint4> nrec;
+    std::vector<uint2> nadj;
+    std::vector<int32_t> lnode;
     std::vector<uint32_t> pent;
+    int64_t ngrouped = 0;
     for (int32_t i = 0; i < NT; i++) {
         const int32_t x = order[i];
-        uint32_t src = 0, kind = 0, gate = 0xFFFFFFFFu;
-        if (x < n) src = (uint32_t)x;
-        else {
+        if (!aff[x] && x < n) continue;
+        // a group: up to 4 consecutive always-active walked nodes of one level
+        // with the same in-degree D in 1..4 (no edges among them)
+        if (x < n) {
+            const int32_t D = (int32_t)ent[x].size();
+            int32_t G = 1;
+            while (D >= 1 && D <= 4 && G < 4 && i + G < NT) {
+                const int32_t y = order[i + G];
+                if (y >= n || !aff[y] || (int32_t)ent[y].size() != D) break;
+                bool same = true;       // same level: y reads none of the group
+                for (int32_t q = 0; q < G && same; q++)
+                    for (uint32_t e : ent[y]) {
+                        const int32_t z = order[i + q];
+                        if (e == (uint32_t)z) same = false;
+                        if ((e & kLU) && (g->h_elig[e & kIdx] == z)) same = false;
+                    }
+                if (!same) break;
+                G++;
+            }
+            if (G > 1) {
+                const uint32_t off = (uint32_t)pent.size();
+                for (int32_t q = 0; q < G; q++) {
+                    const int32_t y = order[i + q];
+                    lnode.push_back(y);
+                    nrec.push_back(make_uint4(0u, 0u, best_slot[y], 0xFFFFFFFFu));
+                    nadj.push_back(make_uint2(q == 0 ? off : (uint32_t)pent.size(),
+                                              q == 0 ? ((uint32_t)D | (2u << 24) | ((uint32_t)G << 26)) : (uint32_t)D));
+                    for (uint32_t e : ent[y]) {
+                        const uint32_t v = (e & kLU) ? e : ref((int32_t)e);
+                        if (v == kNoSlot) return set_error(MAGIS_E_INVAL, "internal: reader of an unslotted value");
+                        pent.push_back(v);
+                    }
+                }
+                ngrouped += G;
+                i += G - 1;
+                continue;
+            }
+        }
+        uint32_t gate = 0xFFFFFFFFu;
+        if (x >= n) {
             const int32_t r = (x - n) / 3, o = (x - n) % 3;
-            src = (uint32_t)g->h_elig[r];
-            kind = (uint32_t)o;                      // 0 clone (label of t_r), 1 Store, 2 Load
             gate = ((uint32_t)r << 2) | (o == 0 ? 1u : 2u);
         }
-        nrec[i] = make_uint4(src, kind, best_slot[x], gate);
-        nadj[i] = make_uint2((uint32_t)pent.size(), (uint32_t)ent[x].size());
-        for (uint32_t e : ent[x]) pent.push_back((e & kLU) ? e : best_slot[e]);
+        lnode.push_back(x);
+        nrec.push_back(make_uint4(0u, 0u, aff[x] ? best_slot[x] : kNoSlot, gate));
+        if (!aff[x]) {
+            nadj.push_back(make_uint2((uint32_t)x, (uint32_t)ent[x].size() | (1u << 24)));
+            continue;
+        }
+        nadj.push_back(make_uint2((uint32_t)pent.size(), (uint32_t)ent[x].size()));
+        for (uint32_t e : ent[x]) {
+            const uint32_t v = (e & kLU) ? e : ref((int32_t)e);
+            if (v == kNoSlot) return set_error(MAGIS_E_INVAL, "internal: reader of an unslotted value");
+            pent.push_back(v);
+        }
     }
     std::vector<uint4> rslot(std::max(R, 1));
     for (int32_t r = 0; r < R; r++) {
         const int32_t t = g->h_elig[r];
-        rslot[r] = make_uint4(best_slot[t], best_slot[n + 3 * r], best_slot[n + 3 * r + 2], best_slot[t]);
+        rslot[r] = make_uint4(ref(t), ref(n + 3 * r), ref(n + 3 * r + 2), ref(t));
     }
-    for (uint32_t e : pent)
-        if (!(e & kLU) && e == kNoSlot) return set_error(MAGIS_E_INVAL, "internal: reader of an unslotted value");
+    // constant nodes in order, with their predecessors (all constant)
+    std::vector<int32_t> cnode, cptr(1, 0), cpred;
+    std::vector<uint8_t> corig;
+    for (int32_t x : order) {
+        if (aff[x]) continue;
+        cnode.push_back(x);
+        corig.push_back(x < n ? 1 : 0);
+        for (uint32_t e : ent[x]) cpred.push_back((int32_t)e);
+        cptr.push_back((int32_t)cpred.size());
+    }
+    // per node: label source and in-degree (for h1)
+    std::vector<uint32_t> lsrc(NT);
+    std::vector<int32_t> degv(NT);
+    int32_t cmaxdeg = 1;
+    for (int32_t x = 0; x < NT; x++) {
+        if (x < n) lsrc[x] = (uint32_t)x;
+        else {
+            const int32_t r = (x - n) / 3, o = (x - n) % 3;
+            lsrc[x] = o == 0 ? (uint32_t)g->h_elig[r] : o == 1 ? kLabStore : kLabLoad;
+        }
+        degv[x] = (int32_t)ent[x].size();
+        cmaxdeg = std::max(cmaxdeg, degv[x]);
+    }
+    const int32_t nloop = (int32_t)lnode.size(), nc = (int32_t)cnode.size();
 
     magis_ghash* h = new (std::nothrow) magis_ghash();
     if (!h) return set_error(MAGIS_E_NOMEM, "host allocation failed");
     h->g = g;
     h->device = g->device;
     DeviceGuard guard(g->device);
-    auto al = [](size_t x) { return (x + 255) / 256 * 256; };
-    const size_t o_nrec = 0, o_nadj = al(o_nrec + 16 * (size_t)NT), o_pent = al(o_nadj + 8 * (size_t)NT),
-                 o_rslot = al(o_pent + 4 * std::max<size_t>(pent.size(), 1)),
-                 o_lab = al(o_rslot + 16 * rslot.size()), total = al(o_lab + 8 * (size_t)n);
-    if (cudaMalloc(&h->tables, total) != cudaSuccess) {
+    size_t off = 0;
+    auto al = [&](size_t bytes) { const size_t o = off; off = (off + std::max<size_t>(bytes, 1) + 255) / 256 * 256; return o; };
+    const size_t o_nrec = al(16 * (size_t)nloop), o_nadj = al(8 * (size_t)nloop), o_pent = al(4 * pent.size()),
+                 o_rslot = al(16 * rslot.size()), o_x0 = al(8 * (size_t)NT), o_c0 = al(8), o_h1 = al(8 * (size_t)NT),
+                 o_lab = al(8 * (size_t)n), o_lsrc = al(4 * (size_t)NT), o_deg = al(4 * (size_t)NT),
+                 o_cnode = al(4 * (size_t)nc), o_cptr = al(4 * cptr.size()), o_cpred = al(4 * cpred.size()),
+                 o_corig = al(corig.size()), o_tmp = al(8 * (size_t)cmaxdeg), o_lnode = al(4 * (size_t)nloop);
+    if (cudaMalloc(&h->tables, off) != cudaSuccess) {
         cudaGetLastError();
         delete h;
         return set_error(MAGIS_E_NOMEM, "cudaMalloc GraphHash tables failed");
     }
     char* b = (char*)h->tables;
-    cudaError_t e = cudaMemcpy(b + o_nrec, nrec.data(), 16 * (size_t)NT, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(b + o_nadj, nadj.data(), 8 * (size_t)NT, cudaMemcpyHostToDevice);
-    if (e == cudaSuccess && !pent.empty()) e = cudaMemcpy(b + o_pent, pent.data(), 4 * pent.size(), cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(b + o_rslot, rslot.data(), 16 * rslot.size(), cudaMemcpyHostToDevice);
-    if (e == cudaSuccess) e = cudaMemcpy(b + o_lab, h_label, 8 * (size_t)n, cudaMemcpyHostToDevice);
+    cudaError_t e = cudaSuccess;
+    auto up = [&](size_t o, const void* src, size_t bytes) {
+        if (e == cudaSuccess && bytes) e = cudaMemcpy(b + o, src, bytes, cudaMemcpyHostToDevice);
+    };
+    up(o_nrec, nrec.data(), 16 * (size_t)nloop);
+    up(o_nadj, nadj.data(), 8 * (size_t)nloop);
+    up(o_pent, pent.data(), 4 * pent.size());
+    up(o_rslot, rslot.data(), 16 * rslot.size());
+    up(o_lab, h_label, 8 * (size_t)n);
+    up(o_lsrc, lsrc.data(), 4 * (size_t)NT);
+    up(o_deg, degv.data(), 4 * (size_t)NT);
+    up(o_cnode, cnode.data(), 4 * (size_t)nc);
+    up(o_cptr, cptr.data(), 4 * cptr.size());
+    up(o_cpred, cpred.data(), 4 * cpred.size());
+    up(o_corig, corig.data(), corig.size());
+    up(o_lnode, lnode.data(), 4 * (size_t)nloop);
+    auto* h1 = (unsigned long long*)(b + o_h1);
+    auto* x0 = (unsigned long long*)(b + o_x0);
+    auto* c0 = (unsigned long long*)(b + o_c0);
     if (e == cudaSuccess) {
-        ghash_label_kernel<<<(NT + 255) / 256, 256>>>((uint4*)(b + o_nrec), NT, (const uint64_t*)(b + o_lab));
+        ghash_h1_kernel<<<(NT + 255) / 256, 256>>>(NT, (const uint32_t*)(b + o_lsrc), (const int32_t*)(b + o_deg),
+                                                   (const uint64_t*)(b + o_lab), h1);
+        ghash_const_kernel<<<1, 1>>>(nc, (const int32_t*)(b + o_cnode), (const int32_t*)(b + o_cptr),
+                                     (const int32_t*)(b + o_cpred), (const uint8_t*)(b + o_corig), h1, x0,
+                                     (unsigned long long*)(b + o_tmp), c0);
+        if (nloop)
+            ghash_fill_kernel<<<(nloop + 255) / 256, 256>>>(nloop, (const int32_t*)(b + o_lnode), h1,
+                                                             (uint4*)(b + o_nrec));
         e = cudaGetLastError();
     }
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
     GhDev& d = h->dev;
-    d.NT = NT; d.R = R; d.NS = NS; d.gslots = best_gs; d.maxdeg = maxdeg > 32 ? maxdeg : 0; d.Rw = Rw;
+    d.nloop = nloop; d.R = R; d.NS = NS; d.gslots = best_gs; d.maxdeg = maxdeg > 32 ? maxdeg : 0; d.Rw = Rw;
     d.nrec = (const uint4*)(b + o_nrec);
     d.nadj = (const uint2*)(b + o_nadj);
     d.pent = (const uint32_t*)(b + o_pent);
     d.rslot = (const uint4*)(b + o_rslot);
     d.rflag = g->dev.rflag;
+    d.x0 = x0;
+    d.c0 = c0;
     h->n_global_nodes = best_glob;
-    h->smem = (size_t)kGhWarps * ((size_t)NS * 256 + dec_bytes);
-    if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(ghash_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)h->smem);
+    h->n_const_nodes = nc;
+    h->n_grouped = ngrouped;
+    h->smem = (size_t)kGhWarps * ((size_t)NS * 256 + (size_t)Rw * 128);
+    const void* fn = (const void*)ghash_kernel;
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)h->smem);
     int occ = 0;
-    if (e == cudaSuccess)
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ghash_kernel, 32 * kGhWarps, h->smem);
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, 32 * kGhWarps, h->smem);
     if (e == cudaSuccess && occ < 1) e = cudaErrorInvalidConfiguration;
     if (e == cudaSuccess) {
         h->grid = sms * occ;
@@ -488,8 +719,11 @@ extern "C" int magis_ghash_create(const magis_graph* g, const uint64_t* h_label,
                          std::string("GraphHash setup: ") + cudaGetErrorString(e));
     }
     if (std::getenv("MAGIS_DEBUG"))
-        std::fprintf(stderr, "[magis] ghash NT=%d NS=%d gslots=%d global-nodes=%lld maxdeg=%d grid=%d occ=%d smem=%zu\n",
-                     NT, NS, d.gslots, (long long)best_glob, maxdeg, h->grid, occ, h->smem);
+        std::fprintf(stderr,
+                     "[magis] ghash NT=%d walked=%d const=%d grouped=%lld NS=%d gslots=%d global-nodes=%lld maxdeg=%d "
+                     "grid=%d occ=%d smem=%zu scratch=%zu\n",
+                     NT, nloop, nc, (long long)ngrouped, NS, d.gslots, (long long)best_glob, maxdeg, h->grid, occ, h->smem,
+                     h->scratch_bytes);
     *out = h;
     return MAGIS_SUCCESS;
 }
@@ -519,8 +753,8 @@ extern "C" int magis_graph_hash(magis_ghash* h, int64_t K, const uint8_t* d_dec,
     const int grid = (int)std::min<int64_t>(h->grid, (groups + kGhWarps - 1) / kGhWarps);
     // 16-byte decision loads when every row starts 16-byte aligned
     const int vec = (h->dev.R % 16 == 0) && ((uintptr_t)d_dec % 16 == 0);
-    ghash_kernel<<<grid, 32 * kGhWarps, h->smem, (cudaStream_t)cuda_stream>>>(h->dev, K, d_dec, vec, d_status,
-                                                                              d_hash);
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    ghash_kernel<<<grid, 32 * kGhWarps, h->smem, st>>>(h->dev, K, d_dec, vec, d_status, d_hash);
     GCK(cudaGetLastError());
     return MAGIS_SUCCESS;
 }
@@ -533,97 +767,5 @@ extern "C" int magis_ghash_info(const magis_ghash* h, int32_t* shared_slots, int
     if (global_slots) *global_slots = h->dev.gslots;
     if (global_nodes) *global_nodes = h->n_global_nodes;
     if (grid) *grid = h->grid;
-    return MAGIS_SUCCESS;
-}
-
-extern "C" int magis_hashset_create(int device, int64_t capacity, magis_hashset** out) {
-    clear_error();
-    if (!out) return set_error(MAGIS_E_INVAL, "out is NULL");
-    *out = nullptr;
-    if (capacity < 1 || capacity > (1ll << 40)) return set_error(MAGIS_E_INVAL, "capacity out of range");
-    if (!magis_device_supported(device))
-        return set_error(MAGIS_E_UNSUPPORTED, "device " + std::to_string(device) +
-                         " is not an sm_100 (B200) GPU; there is no CPU fallback");
-    DeviceGuard guard(device);
-    magis_hashset* s = new (std::nothrow) magis_hashset();
-    if (!s) return set_error(MAGIS_E_NOMEM, "host allocation failed");
-    uint64_t cap = 1;
-    while (cap < (uint64_t)capacity) cap <<= 1;
-    s->device = device;
-    s->cap = cap;
-    if (cudaMalloc(&s->keys, cap * 8) != cudaSuccess || cudaMalloc(&s->owner, (cap + 1) * 8) != cudaSuccess ||
-        cudaMalloc(&s->stats, 16) != cudaSuccess) {
-        cudaGetLastError();
-        if (s->keys) cudaFree(s->keys);
-        if (s->owner) cudaFree(s->owner);
-        delete s;
-        return set_error(MAGIS_E_NOMEM, "cudaMalloc hash set failed");
-    }
-    const int rc = magis_hashset_clear(s, nullptr);
-    if (rc != MAGIS_SUCCESS || cudaDeviceSynchronize() != cudaSuccess) {
-        cudaGetLastError();
-        cudaFree(s->keys);
-        cudaFree(s->owner);
-        cudaFree(s->stats);
-        delete s;
-        return set_error(MAGIS_E_CUDA, "hash set initialisation failed");
-    }
-    *out = s;
-    return MAGIS_SUCCESS;
-}
-
-extern "C" int magis_hashset_clear(magis_hashset* s, void* cuda_stream) {
-    clear_error();
-    if (!s) return set_error(MAGIS_E_INVAL, "hash set is NULL");
-    DeviceGuard guard(s->device);
-    cudaStream_t st = (cudaStream_t)cuda_stream;
-    GCK(cudaMemsetAsync(s->keys, 0, s->cap * 8, st));
-    GCK(cudaMemsetAsync(s->owner, 0xFF, (s->cap + 1) * 8, st));
-    GCK(cudaMemsetAsync(s->stats, 0, 16, st));
-    return MAGIS_SUCCESS;
-}
-
-extern "C" int magis_hashset_free(magis_hashset* s) {
-    clear_error();
-    if (!s) return MAGIS_SUCCESS;
-    DeviceGuard guard(s->device);
-    cudaDeviceSynchronize();
-    cudaFree(s->keys);
-    cudaFree(s->owner);
-    cudaFree(s->stats);
-    cudaGetLastError();
-    delete s;
-    return MAGIS_SUCCESS;
-}
-
-extern "C" int magis_hashset_filter(magis_hashset* s, int64_t K, const uint64_t* d_hash, const uint8_t* d_status,
-                                    uint8_t* d_new, void* cuda_stream) {
-    clear_error();
-    if (!s) return set_error(MAGIS_E_INVAL, "hash set is NULL");
-    if (K < 0 || K >= (1ll << 40)) return set_error(MAGIS_E_INVAL, "K out of range");
-    if (K == 0) return MAGIS_SUCCESS;
-    if (!d_hash || !d_new) return set_error(MAGIS_E_INVAL, "null device pointer");
-    if (s->epoch + 1 >= (1u << 24)) return set_error(MAGIS_E_CAPACITY, "hash set epoch exhausted: clear it");
-    DeviceGuard guard(s->device);
-    s->epoch++;
-    cudaStream_t st = (cudaStream_t)cuda_stream;
-    const int grid = (int)std::min<int64_t>((K + 255) / 256, 148 * 16);
-    hs_insert_kernel<<<grid, 256, 0, st>>>(*s, K, d_hash, d_status);
-    GCK(cudaGetLastError());
-    hs_mark_kernel<<<grid, 256, 0, st>>>(*s, K, d_hash, d_status, d_new);
-    GCK(cudaGetLastError());
-    return MAGIS_SUCCESS;
-}
-
-extern "C" int magis_hashset_stats(const magis_hashset* s, int64_t* n_keys, int64_t* n_overflow) {
-    clear_error();
-    if (!s) return set_error(MAGIS_E_INVAL, "hash set is NULL");
-    DeviceGuard guard(s->device);
-    unsigned long long h[2] = {0, 0};
-    GCK(cudaMemcpy(h, s->stats, 16, cudaMemcpyDeviceToHost));
-    unsigned long long z = 0;
-    GCK(cudaMemcpy(&z, s->owner + s->cap, 8, cudaMemcpyDeviceToHost));
-    if (n_keys) *n_keys = (int64_t)h[0] + (z != ~0ull ? 1 : 0);
-    if (n_overflow) *n_overflow = (int64_t)h[1];
     return MAGIS_SUCCESS;
 }
