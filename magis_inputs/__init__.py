@@ -19,6 +19,10 @@ CONFIGS = {
     "c3": dict(desc="BERT-large training s512 b32 fp32, F-Trans n=4 on attention/FFN", K=262144, R_max=256),
     "c4": dict(desc="SD-v1-shaped UNet training b8 1024px bf16, F-Trans n=32 on attention", K=65536, R_max=512),
     "c5": dict(desc="GPT-Neo-1.3B-shaped decoder training s512 b32 bf16", K=1048576, R_max=128),
+    # NEXT-4: C3's BERT-large with every attention / FFN group as an F-Trans
+    # region offering n in {1, 2, 4} side by side (the candidate picks one)
+    "c3f": dict(desc="BERT-large training s512 b32 fp32, F-Trans variant regions n in {1,2,4} per attention/FFN",
+                K=65536, R_max=128),
 }
 
 
@@ -41,6 +45,10 @@ def build_workload(cfg: str, **kw) -> Workload:
         b = ftrans.apply(b, n)
     elif cfg == "c5":
         b = models.gpt_neo_1p3b(B=kw.get("batch", 32), S=kw.get("seq", 512), layers=kw.get("layers", 24))
+    elif cfg == "c3f":
+        b = models.bert_large(B=kw.get("batch", 32), S=kw.get("seq", 512), ftrans=4,
+                              layers=kw.get("layers", 24))
+        b = ftrans.apply_variants(b, kw.get("ns", (2, 4)))
     else:
         raise ValueError(cfg)
     wl = b.finish(meta={"config": cfg})

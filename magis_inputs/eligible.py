@@ -28,10 +28,21 @@ def select(wl: Workload, R_max: int, min_span: int = 8) -> Workload:
         cons[u].append(v)
         has_in[v] = True
     loss = wl.loss_node if wl.loss_node >= 0 else n // 2
+    # F-Trans variant graphs (NEXT-4): the Fig. 8 rules stay on the nodes that
+    # exist in every variant -- t, its inputs and its late users ungated
+    gated = (wl.regions["node_region"] >= 0) if wl.regions is not None else np.zeros(n, bool)
+    if gated.any():
+        pre_gated = np.zeros(n, bool)
+        for u, v in zip(wl.src.tolist(), wl.dst.tolist()):
+            if gated[u]:
+                pre_gated[v] = True
+        cons = [[v for v in cs if not gated[v]] for cs in cons]
     cand = []
     for t in range(n):
         c = sorted(set(cons[t]))
         if wl.kind[t] != "op" or wl.is_output[t] or not has_in[t] or len(c) < 2:
+            continue
+        if gated[t] or (gated.any() and pre_gated[t]):
             continue
         if c[-1] - c[0] < min_span or c[-1] <= loss:
             continue

@@ -52,6 +52,13 @@ class Workload:
     swap_lat: float = SWAP_LAT
     loss_node: int = -1
     meta: Dict = field(default_factory=dict)
+    # F-Trans variant regions (NEXT-4, reading F1): n_variants [F],
+    # node_region [n] (-1: present in every variant), node_variant [n]
+    regions: Optional[Dict] = None
+
+    @property
+    def F(self) -> int:
+        return 0 if self.regions is None else len(self.regions["n_variants"])
 
     @property
     def n(self) -> int:
@@ -99,10 +106,14 @@ class Builder:
         self.splitdim: List[int] = []           # +1 split along the tag's positive dim, -1 reduce, 0 none
         self.loss_node = -1
         self.shared: Dict[str, set] = {}       # F-Trans group -> activations read unsliced
+        self.cost_fix: List[Optional[float]] = []   # cost override (variant graphs), else the formula
+        self.region: List[int] = []            # F-Trans variant region of the node, -1 = always present
+        self.variant: List[int] = []           # variant of that region the node belongs to
+        self.n_variants: List[int] = []        # per region
 
     def node(self, name: str, nbytes: int, inputs: Sequence[int] = (), flops: float = 0.0,
              kind: str = "op", tensor: bool = False, tag: Optional[str] = None,
-             splitdim: int = 0) -> int:
+             splitdim: int = 0, cost: Optional[float] = None, region: int = -1, variant: int = 0) -> int:
         v = len(self.names)
         ins = list(dict.fromkeys(int(u) for u in inputs))
         for u in ins:
@@ -116,9 +127,14 @@ class Builder:
         self.inputs.append(ins)
         self.tag.append(tag)
         self.splitdim.append(int(splitdim))
+        self.cost_fix.append(cost)
+        self.region.append(int(region))
+        self.variant.append(int(variant))
         return v
 
     def cost_of(self, v: int) -> float:
+        if self.cost_fix and self.cost_fix[v] is not None:
+            return self.cost_fix[v]
         if self.kind[v] in ("input", "weight", "label"):
             return 0.0
         rw = self.size[v] + sum(self.size[u] for u in self.inputs[v])
@@ -149,6 +165,10 @@ class Builder:
         if elig is not None:
             wl.elig = np.asarray(elig, np.int32)
             wl.U = [list(map(int, u)) for u in U]
+        if self.n_variants:
+            wl.regions = {"n_variants": np.asarray(self.n_variants, np.int32),
+                          "node_region": np.asarray(self.region, np.int32),
+                          "node_variant": np.asarray(self.variant, np.uint8)}
         return wl
 
 

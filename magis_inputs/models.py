@@ -218,9 +218,9 @@ def transformer(name: str, layers: int, D: int, H: int, Fd: int, vocab: int, B: 
     return b
 
 
-def bert_large(B: int = 32, S: int = 512, ftrans: int = 4):
-    return transformer(f"bert_large_s{S}_b{B}_ft{ftrans}", 24, 1024, 16, 4096, 30522, B, S,
-                       4, pre_ln=False, ftrans=ftrans)
+def bert_large(B: int = 32, S: int = 512, ftrans: int = 4, layers: int = 24):
+    return transformer(f"bert_large_s{S}_b{B}_ft{ftrans}" + (f"_l{layers}" if layers != 24 else ""), layers,
+                       1024, 16, 4096, 30522, B, S, 4, pre_ln=False, ftrans=ftrans)
 
 
 def gpt_neo_1p3b(B: int = 32, S: int = 512, layers: int = 24):
