@@ -63,8 +63,8 @@ def _pool_init(arrays):
 def _oracle_chunk(args):
     perms, decs = args
     import oracle
-    size, cost, iso, src, dst, elig, U, B, lam = _WL
-    g = oracle.OracleGraph(size, cost, iso, src, dst, elig, U, B, lam)
+    size, cost, iso, src, dst, elig, U, B, lam, regions = _WL
+    g = oracle.OracleGraph(size, cost, iso, src, dst, elig, U, B, lam, regions)
     t = time.perf_counter()
     st, pk, lt = g.eval_batch(perms, decs)
     return st, pk, lt, time.perf_counter() - t
@@ -196,13 +196,18 @@ def main():
     wl = build_workload(cfg)
     if need_pool:
         import multiprocessing as mp
-        arrays = (wl.size, wl.cost, wl.is_output, wl.src, wl.dst, wl.elig, wl.U, wl.swap_Bps, wl.swap_lat)
+        arrays = (wl.size, wl.cost, wl.is_output, wl.src, wl.dst, wl.elig, wl.U, wl.swap_Bps, wl.swap_lat,
+                  wl.regions)
         pool = mp.get_context("fork").Pool(ncores, initializer=_pool_init, initargs=(arrays,))
 
     workload = {"workload": f"{cfg}: {CONFIGS[cfg]['desc']}", "graph": wl.name, "n_nodes": wl.n,
                 "n_edges": wl.n_edges, "R": wl.R, "n_total": wl.n_total, "K_per_rank": K,
                 "candidates": "75% random topo orders, 24% local moves (w<=64), 1% transposition; "
                               "P(remat)=P(swap)=5%", "seed": args.seed}
+    if wl.F:
+        workload["regions"] = wl.F
+        workload["candidates"] = ("99% random topo orders of the chosen variants, 1% transposition; "
+                                  "variant uniform per region; P(remat)=P(swap)=5%")
 
     if args.impl == "reference":
         return run_reference(args, wl, K, workload, pool, ncores, rank, world)
@@ -237,16 +242,19 @@ def main():
     load_s = time.perf_counter() - t0
     R, NT = g.R, g.n_total
     # device candidate generator (§8(a) a1), timed separately from evaluation
-    Pg, Dg = g.generate_candidates(rank * K, K, seed=args.seed)          # warm-up / scratch allocation
-    torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    g.generate_candidates(rank * K, K, seed=args.seed, perm=Pg, dec=Dg)
-    e1.record()
-    torch.cuda.synchronize()
-    gen_dev_ms = e0.elapsed_time(e1)
-    gen_match = bool(torch.equal(Pg, P) and (R == 0 or torch.equal(Dg[:, :R], D[:, :R])))
-    del Pg, Dg
+    # (the F-Trans variant graphs of NEXT-4 are generated on the host only)
+    gen_dev_ms, gen_match = None, None
+    if wl.F == 0:
+        Pg, Dg = g.generate_candidates(rank * K, K, seed=args.seed)          # warm-up / scratch allocation
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        g.generate_candidates(rank * K, K, seed=args.seed, perm=Pg, dec=Dg)
+        e1.record()
+        torch.cuda.synchronize()
+        gen_dev_ms = e0.elapsed_time(e1)
+        gen_match = bool(torch.equal(Pg, P) and (R == 0 or torch.equal(Dg[:, :R], D[:, :R])))
+        del Pg, Dg
     stream = torch.cuda.current_stream()
     st = torch.empty(K, dtype=torch.uint8, device=dev)
     pk = torch.empty(K, dtype=torch.int64, device=dev)
@@ -258,7 +266,7 @@ def main():
     def step(ev_pair=None):
         if ev_pair:
             ev_pair[0].record(stream)
-        g.eval_schedules(P, D if R else None, st, pk, lt, stream=stream)
+        g.eval_schedules(P, D if g.dec_len else None, st, pk, lt, stream=stream)
         if ev_pair:
             ev_pair[1].record(stream)
         fr = pareto_merge(pk, lt, st, id_base=rank * K, cap=args.cap, mem_limit=mem_limit,
@@ -296,7 +304,7 @@ def main():
     value = world * K / (ms_per_step / 1e3)
 
     # --- roofline of the dominant kernel (eval): algorithmic bytes per launch
-    bytes_per_cand = 4 * NT + R + 17
+    bytes_per_cand = 4 * NT + g.dec_len + 17
     alg_bytes = K * bytes_per_cand
     achieved = alg_bytes / (kern_avg / 1e3) / 1e9
     peak_gbs, peak_src = peaks()
@@ -334,7 +342,7 @@ def main():
         api = ("magis_eval_schedules_host_u16 (uint16 schedules" if u16 else
                "magis_eval_schedules_host (int32 schedules")
         e2e = {"value": round(world * K / te.item(), 1), "unit": UNIT,
-               "h2d_bytes_per_step": int(K * NT * (2 if u16 else 4) + K * R), "d2h_bytes_per_step": int(K * 17),
+               "h2d_bytes_per_step": int(K * NT * (2 if u16 else 4) + K * g.dec_len), "d2h_bytes_per_step": int(K * 17),
                "api": api + ", pinned host buffers, chunked double-buffered copies)",
                "s_per_step": round(te.item(), 5)}
         ok_same = bool((out_pinned[1].numpy() == pk.cpu().numpy()).all())
@@ -370,8 +378,8 @@ def main():
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk.summary(),
                 "gpu_launches": gpu_launches,
                 "setup": {"candidate_gen_s": round(gen_s, 3), "graph_load_s": round(load_s, 3),
-                          "device_gen_ms": round(gen_dev_ms, 3),
-                          "device_gen_cand_per_s": round(K / (gen_dev_ms / 1e3), 1),
+                          "device_gen_ms": round(gen_dev_ms, 3) if gen_dev_ms else None,
+                          "device_gen_cand_per_s": round(K / (gen_dev_ms / 1e3), 1) if gen_dev_ms else None,
                           "device_gen_matches_host": gen_match,
                           "eval_variant": g.info["variant"], "grid": g.info["grid"], "block": g.info["block"],
                           "smem_bytes": g.info["smem_bytes"]}}
@@ -472,8 +480,8 @@ def run_windows(args, wl, cfg, rank, world, local):
 def _oracle_hash_chunk(args):
     decs, labels = args
     import oracle
-    size, cost, iso, src, dst, elig, U, B, lam = _WL
-    g = oracle.OracleGraph(size, cost, iso, src, dst, elig, U, B, lam)
+    size, cost, iso, src, dst, elig, U, B, lam, regions = _WL
+    g = oracle.OracleGraph(size, cost, iso, src, dst, elig, U, B, lam, regions)
     t = time.perf_counter()
     st, hs = g.graph_hash_batch(labels, decs)
     return st, hs, time.perf_counter() - t

@@ -34,7 +34,7 @@ extern "C" {
 #pragma GCC visibility push(default)   /* the library builds with -fvisibility=hidden */
 #endif
 
-#define MAGIS_ABI_VERSION 1
+#define MAGIS_ABI_VERSION 2
 
 enum {
     MAGIS_SUCCESS = 0,
@@ -114,6 +114,7 @@ typedef struct magis_graph_info {
     int64_t table_bytes;       /* device bytes of the graph tables */
     double base_cost;          /* sum of cost(v) over original nodes */
     int32_t pack;              /* candidates scored together per CTA step (variant 2), else 1 */
+    int32_t n_regions;         /* F-Trans variant regions F (decision row = R + F bytes) */
 } magis_graph_info;
 
 /*
@@ -129,6 +130,43 @@ typedef struct magis_graph_info {
  */
 int magis_graph_load(const magis_graph_desc* desc, int device, magis_graph** out);
 
+/*
+ * F-Trans variant regions (§4.2-4.3, §5.1
+ * P:1295-1326; reading F1 in DESIGN.md).  An F-Trans f = (S, D, n) replaces
+ * the sub-graph S by n parts plus slices and merges (Fig. 5).  A region holds
+ * several such versions of one S side by side in the graph (variant 0 = S
+ * unsplit, variant j = one factor n_j): the caller materialises them as
+ * ordinary nodes and labels each with (region, variant).  A candidate picks
+ * one variant per region; a node of region i exists iff the candidate's
+ * choice for i equals its variant, an edge exists iff both ends exist, and
+ * nodes that do not exist are no-ops wherever the schedule puts them (they
+ * hold no memory and cost no time).  The decision row of a candidate becomes
+ * [R eligible decisions | F region variants] (uint8, R + F bytes).
+ *   n_regions     F >= 0.
+ *   n_variants    [F] 1..4.
+ *   node_region   [n_nodes] region of the node, or -1 (present in every variant).
+ *   node_variant  [n_nodes] variant of that region (< n_variants[region]).
+ * Constraints (MAGIS_E_INVAL otherwise): an edge joins nodes of at most one
+ * (region, variant) (regions do not touch; a consumer outside a region reads
+ * every variant's version of a region output); eligible tensors, their
+ * inputs and their late users are outside regions (the Fig. 8 rules act on
+ * the ops present in every variant).  A variant index >= n_variants in a
+ * candidate is MAGIS_ST_BAD_DEC.  Graphs with regions are scored by the
+ * general gated kernel (variant 0/1); magis_generate_candidates,
+ * magis_base_create, magis_hotspots and magis_ghash_create return
+ * MAGIS_E_UNSUPPORTED on them.  magis_graph_load(d, dev, out) is
+ * magis_graph_load_regions(d, NULL, dev, out).
+ */
+typedef struct magis_region_desc {
+    int32_t n_regions;
+    const int32_t* n_variants;
+    const int32_t* node_region;
+    const uint8_t* node_variant;
+} magis_region_desc;
+
+int magis_graph_load_regions(const magis_graph_desc* desc, const magis_region_desc* regions, int device,
+                             magis_graph** out);
+
 /* Release a graph (NULL is a no-op).  Synchronises the graph's device. */
 int magis_graph_free(magis_graph* g);
 
@@ -141,7 +179,8 @@ int magis_graph_info_get(const magis_graph* g, magis_graph_info* info);
  *   plus the latency model (sum of compute costs; with swaps, the three
  *   in-order queues compute / D2H / H2D of reading P7).
  * d_perm     [K x n_total] int32, row-major, device memory: step -> super id.
- * d_dec      [K x R] uint8 device memory, or NULL (all zero) when R == 0.
+ * d_dec      [K x (R + F)] uint8 device memory (F = n_regions, usually 0), or
+ *            NULL when R + F == 0.
  * d_status   [K] uint8  out: MAGIS_ST_* bits.
  * d_peak     [K] int64  out: M_peak in bytes (-1 if status != 0).
  * d_latency  [K] double out: seconds (+inf if status != 0).

@@ -37,6 +37,9 @@ def _load():
         lib.candgen.argtypes = [i32, i32, P, P, P, P, P, P, P, u64, i32, i32, i32, i32, i32, i32,
                                 u64, i64, P, P, i32]
         lib.candgen.restype = None
+        lib.candgen_regions.argtypes = [i32, i32, P, P, P, P, P, P, P, u64, i32, i32, i32, i32, i32, i32,
+                                        u64, i64, P, P, i32, i32, P, P, P]
+        lib.candgen_regions.restype = None
         lib.wingen.argtypes = [i32, i32, P, P, P, P, P, P, P, P, P, P, u64, i32, i32, u64, i64, P, P, P]
         lib.wingen.restype = None
         _lib = lib
@@ -84,22 +87,33 @@ class CandidateGenerator:
         self.elig = np.ascontiguousarray(wl.elig, np.int32)
 
     def generate(self, id0: int, K: int, nthreads: int | None = None, out=None):
-        """-> (perms int32 [K, n_total], decs uint8 [K, max(R,1)])."""
+        """-> (perms int32 [K, n_total], decs uint8 [K, max(R + F, 1)]); with
+        F-Trans variant regions (NEXT-4) the last F columns are the chosen
+        variants."""
         lib = _load()
         wl, sp = self.wl, self.spec
         NT = wl.n_total
+        F = wl.F
         if out is None:
             perms = np.empty((K, NT), np.int32)
-            decs = np.zeros((K, max(wl.R, 1)), np.uint8)
+            decs = np.zeros((K, max(wl.R + F, 1)), np.uint8)
         else:
             perms, decs = out
         if nthreads is None:
             nthreads = max(1, min(os.cpu_count() or 1, 64))
         p = lambda a: a.ctypes.data_as(ctypes.c_void_p)
-        lib.candgen(wl.n, wl.R, p(self.succ_ptr), p(self.succ_idx), p(self.pred_ptr), p(self.pred_idx),
-                    p(self.elig), p(self.U_ptr), p(self.U_idx), ctypes.c_uint64(sp.seed),
-                    sp.pct_random, sp.pct_local, sp.p_remat, sp.p_swap, sp.wmax, sp.slack,
-                    ctypes.c_uint64(id0), K, p(perms), p(decs), int(nthreads))
+        args = [wl.n, wl.R, p(self.succ_ptr), p(self.succ_idx), p(self.pred_ptr), p(self.pred_idx),
+                p(self.elig), p(self.U_ptr), p(self.U_idx), ctypes.c_uint64(sp.seed),
+                sp.pct_random, sp.pct_local, sp.p_remat, sp.p_swap, sp.wmax, sp.slack,
+                ctypes.c_uint64(id0), K, p(perms), p(decs), int(nthreads)]
+        if F:
+            rg = wl.regions
+            self._rk = (np.ascontiguousarray(rg["n_variants"], np.int32),
+                        np.ascontiguousarray(rg["node_region"], np.int32),
+                        np.ascontiguousarray(rg["node_variant"], np.uint8))
+            lib.candgen_regions(*args, F, *(p(a) for a in self._rk))
+        else:
+            lib.candgen(*args)
         return perms, decs
 
 

@@ -39,6 +39,7 @@
 #define S_WIN 4u
 #define S_SLK 5u
 #define S_TRN 6u
+#define S_VAR 7u
 
 static inline uint64_t mix64(uint64_t x)
 {
@@ -68,6 +69,13 @@ typedef struct {
     int32_t pct_random, pct_local;
     int32_t p_remat, p_swap;   /* per 10000 */
     int32_t wmax, slack;
+    /* F-Trans variant regions (NEXT-4): dec[R + i] = rnd(VAR, i) % nvar[i];
+     * only the ops of the chosen variants (and the ungated ones) are ordered;
+     * local moves (F2) become F1; absent ops follow the optional nodes. */
+    int32_t F;
+    const int32_t *nvar;       /* [F] */
+    const int32_t *nreg;       /* [n] region or -1 */
+    const uint8_t *nvn;        /* [n] variant */
 } gen_cfg;
 
 typedef struct {
@@ -77,6 +85,7 @@ typedef struct {
     int32_t *posb;
     int64_t *opt;    /* sort keys of active optional nodes */
     uint8_t *inwin;
+    uint8_t *act;    /* present original ops (regions), or NULL */
 } gen_ws;
 
 static void heap_push(uint64_t *h, int32_t *n, uint64_t x)
@@ -120,11 +129,11 @@ static void keyed_kahn(const gen_cfg *c, gen_ws *w, uint64_t k, int32_t lo, int3
     for (v = lo; v < hi; v++) {
         int32_t d = 0;
         for (e = c->pred_ptr[v]; e < c->pred_ptr[v + 1]; e++)
-            if (c->pred_idx[e] >= lo) d++;   /* preds < lo are already placed */
+            if (c->pred_idx[e] >= lo && (!w->act || w->act[c->pred_idx[e]])) d++;   /* preds < lo are placed */
         w->indeg[v] = d;
     }
     for (v = lo; v < hi; v++)
-        if (w->indeg[v] == 0)
+        if (w->indeg[v] == 0 && (!w->act || w->act[v]))
             heap_push(w->heap, &nh, ((rnd(c->seed, k, S_KEY, (uint64_t)v) >> 32) << 32) | (uint32_t)v);
     while (nh > 0) {
         uint64_t x = heap_pop(w->heap, &nh);
@@ -132,7 +141,7 @@ static void keyed_kahn(const gen_cfg *c, gen_ws *w, uint64_t k, int32_t lo, int3
         out[m++] = u;
         for (e = c->succ_ptr[u]; e < c->succ_ptr[u + 1]; e++) {
             int32_t s = c->succ_idx[e];
-            if (s >= hi) continue;
+            if (s >= hi || (w->act && !w->act[s])) continue;
             if (--w->indeg[s] == 0)
                 heap_push(w->heap, &nh, ((rnd(c->seed, k, S_KEY, (uint64_t)s) >> 32) << 32) | (uint32_t)s);
         }
@@ -155,7 +164,17 @@ static void gen_one(const gen_cfg *c, gen_ws *w, uint64_t k, int32_t *perm, uint
         dec[r] = d;
     }
 
-    if ((int32_t)fam < c->pct_random || (int32_t)fam >= c->pct_random + c->pct_local) {
+    int32_t nb = n;                         /* ops in the base order */
+    if (c->F > 0) {
+        for (i = 0; i < c->F; i++)
+            dec[R + i] = (uint8_t)(rnd(c->seed, k, S_VAR, (uint64_t)i) % (uint64_t)c->nvar[i]);
+        nb = 0;
+        for (i = 0; i < n; i++) {
+            w->act[i] = (uint8_t)(c->nreg[i] < 0 || dec[R + c->nreg[i]] == c->nvn[i]);
+            nb += w->act[i];
+        }
+    }
+    if (c->F > 0 || (int32_t)fam < c->pct_random || (int32_t)fam >= c->pct_random + c->pct_local) {
         keyed_kahn(c, w, k, 0, n, w->base);
     } else {
         int32_t len = 2 + (int32_t)(rnd(c->seed, k, S_WIN, 0) % (uint64_t)(c->wmax - 1));
@@ -165,7 +184,7 @@ static void gen_one(const gen_cfg *c, gen_ws *w, uint64_t k, int32_t *perm, uint
         for (i = 0; i < n; i++) w->base[i] = i;
         keyed_kahn(c, w, k, b, b + len, w->base + b);
     }
-    for (i = 0; i < n; i++) w->posb[w->base[i]] = i;
+    for (i = 0; i < nb; i++) w->posb[w->base[i]] = i;
 
     for (r = 0; r < R; r++) {
         int32_t t = c->elig[r], q = INT32_MAX, j, g;
@@ -188,7 +207,7 @@ static void gen_one(const gen_cfg *c, gen_ws *w, uint64_t k, int32_t *perm, uint
     }
     qsort(w->opt, (size_t)nopt, sizeof(int64_t), cmp_i64);
     oi = 0;
-    for (i = 0; i <= n; i++) {
+    for (i = 0; i <= nb; i++) {
         while (oi < nopt && (int32_t)(w->opt[oi] >> 32) == i) {
             int32_t rr = (int32_t)(w->opt[oi] & 0x3fffffff);
             int32_t pr = (int32_t)((w->opt[oi] >> 30) & 3);
@@ -198,8 +217,11 @@ static void gen_one(const gen_cfg *c, gen_ws *w, uint64_t k, int32_t *perm, uint
             perm[m++] = id;
             oi++;
         }
-        if (i < n) perm[m++] = w->base[i];
+        if (i < nb) perm[m++] = w->base[i];
     }
+    if (c->F > 0)                           /* ops of the variants not chosen: no-ops, ascending */
+        for (i = 0; i < n; i++)
+            if (!w->act[i]) perm[m++] = i;
     for (r = 0; r < R; r++) {
         if (dec[r] != 1) perm[m++] = n + 3 * r;
         if (dec[r] != 2) { perm[m++] = n + 3 * r + 1; perm[m++] = n + 3 * r + 2; }
@@ -233,12 +255,21 @@ static void *worker(void *arg)
     w.posb = (int32_t *)malloc(sizeof(int32_t) * (c->n + 1));
     w.opt = (int64_t *)malloc(sizeof(int64_t) * (2 * c->R + 1));
     w.inwin = NULL;
+    w.act = c->F > 0 ? (uint8_t *)malloc((size_t)c->n + 1) : NULL;
     for (k = j->k0; k < j->k1; k++)
         gen_one(c, &w, j->id0 + (uint64_t)k, j->perms + k * (int64_t)c->NT,
-                j->decs + k * (int64_t)(c->R ? c->R : 1));
-    free(w.indeg); free(w.heap); free(w.base); free(w.posb); free(w.opt);
+                j->decs + k * (int64_t)((c->R + c->F) ? c->R + c->F : 1));
+    free(w.indeg); free(w.heap); free(w.base); free(w.posb); free(w.opt); free(w.act);
     return NULL;
 }
+
+void candgen_regions(int32_t n, int32_t R, const int64_t *succ_ptr, const int32_t *succ_idx,
+                     const int64_t *pred_ptr, const int32_t *pred_idx, const int32_t *elig,
+                     const int64_t *U_ptr, const int32_t *U_idx, uint64_t seed,
+                     int32_t pct_random, int32_t pct_local, int32_t p_remat, int32_t p_swap,
+                     int32_t wmax, int32_t slack, uint64_t id0, int64_t K,
+                     int32_t *perms, uint8_t *decs, int32_t nthreads,
+                     int32_t F, const int32_t *nvar, const int32_t *nreg, const uint8_t *nvn);
 
 /* Generate candidates with global ids id0 .. id0+K-1 into perms (K x NT) and
  * decs (K x max(R,1)).  nthreads >= 1. */
@@ -249,6 +280,19 @@ void candgen(int32_t n, int32_t R, const int64_t *succ_ptr, const int32_t *succ_
              int32_t wmax, int32_t slack, uint64_t id0, int64_t K,
              int32_t *perms, uint8_t *decs, int32_t nthreads)
 {
+    candgen_regions(n, R, succ_ptr, succ_idx, pred_ptr, pred_idx, elig, U_ptr, U_idx, seed, pct_random,
+                    pct_local, p_remat, p_swap, wmax, slack, id0, K, perms, decs, nthreads, 0, NULL, NULL, NULL);
+}
+
+/* As candgen, over a graph with F-Trans variant regions: decs is K x (R + F). */
+void candgen_regions(int32_t n, int32_t R, const int64_t *succ_ptr, const int32_t *succ_idx,
+                     const int64_t *pred_ptr, const int32_t *pred_idx, const int32_t *elig,
+                     const int64_t *U_ptr, const int32_t *U_idx, uint64_t seed,
+                     int32_t pct_random, int32_t pct_local, int32_t p_remat, int32_t p_swap,
+                     int32_t wmax, int32_t slack, uint64_t id0, int64_t K,
+                     int32_t *perms, uint8_t *decs, int32_t nthreads,
+                     int32_t F, const int32_t *nvar, const int32_t *nreg, const uint8_t *nvn)
+{
     gen_cfg c;
     pthread_t th[256];
     job jobs[256];
@@ -258,6 +302,7 @@ void candgen(int32_t n, int32_t R, const int64_t *succ_ptr, const int32_t *succ_
     c.elig = elig; c.U_ptr = U_ptr; c.U_idx = U_idx; c.seed = seed;
     c.pct_random = pct_random; c.pct_local = pct_local; c.p_remat = p_remat; c.p_swap = p_swap;
     c.wmax = wmax < 2 ? 2 : wmax; c.slack = slack < 0 ? 0 : slack;
+    c.F = F; c.nvar = nvar; c.nreg = nreg; c.nvn = nvn;
     if (nthreads < 1) nthreads = 1;
     if (nthreads > 256) nthreads = 256;
     if (K < nthreads) nthreads = K > 0 ? (int32_t)K : 1;

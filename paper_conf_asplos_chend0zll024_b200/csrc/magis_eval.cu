@@ -31,7 +31,7 @@ constexpr int kWarps = kBlock / 32;
 
 static size_t al(size_t x) { return (x + 15) / 16 * 16; }
 
-StateLayout state_layout(int32_t NT, int32_t R, int32_t max_events) {
+StateLayout state_layout(int32_t NT, int32_t R, int32_t max_events, int32_t Rd) {
     StateLayout L{};
     size_t o = 0;
     L.pos = o;       o += al((size_t)NT * 4);
@@ -45,7 +45,7 @@ StateLayout state_layout(int32_t NT, int32_t R, int32_t max_events) {
     L.endT = o;      o += al((size_t)R * 8);
     L.endS = o;      o += al((size_t)R * 8);
     L.endL = o;      o += al((size_t)R * 8);
-    L.dec = o;       o += al((size_t)R);
+    L.dec = o;       o += al((size_t)Rd);
     L.total = o;
     return L;
 }
@@ -159,11 +159,15 @@ eval_kernel(DevGraph g, int64_t K, const int32_t* __restrict__ perm,
         // ---- P0: decisions, reset ------------------------------------------------
         if (tid == 0) { sc.status = 0; sc.nev = 0; }
         int bad_dec = 0, any_sw = 0;
-        for (int32_t r = tid; r < R; r += kBlock) {
-            uint8_t d = dec[k * (int64_t)R + r];
+        for (int32_t r = tid; r < g.Rd; r += kBlock) {
+            uint8_t d = dec[k * (int64_t)g.Rd + r];
             dec_s[r] = d;
-            bad_dec |= (d > 2) | ((d == 1) & !(g.rflag[r] & kRHasInput));
-            any_sw |= (d == 2);
+            if (r < R) {
+                bad_dec |= (d > 2) | ((d == 1) & !(g.rflag[r] & kRHasInput));
+                any_sw |= (d == 2);
+            } else {
+                bad_dec |= d >= __ldg(g.nvar + (r - R));   // reading F1: a variant of region r - R
+            }
         }
         for (int32_t v = tid; v < NT; v += kBlock) pos[v] = -1;
         bad_dec = __syncthreads_or(bad_dec);
@@ -248,6 +252,8 @@ eval_kernel(DevGraph g, int64_t K, const int32_t* __restrict__ perm,
             double cl = 0.0;
             for (int32_t r = tid; r < R; r += kBlock)
                 if (dec_s[r] == 1) cl += __ldg(g.tcost + r);
+            for (int32_t i = tid; i < g.F; i += kBlock)              // the chosen F-Trans variants
+                cl += __ldg(g.vcost + 4 * i + dec_s[R + i]);
             lat = g.base_cost + block_sum_d(cl, sc.red_d);
         } else {
             double ctot;
@@ -318,7 +324,7 @@ cudaError_t eval_configure(const DevGraph& g, int device, EvalConfig* cfg) {
     cudaDeviceProp prop;
     cudaError_t e = cudaGetDeviceProperties(&prop, device);
     if (e != cudaSuccess) return e;
-    StateLayout L = state_layout(g.NT, g.R, g.max_events);
+    StateLayout L = state_layout(g.NT, g.R, g.max_events, g.Rd);
     cfg->block = kBlock;
     cfg->state_bytes = (L.total + 255) / 256 * 256;
     const size_t smem_cap = (size_t)prop.sharedMemPerBlockOptin - sizeof(Scratch) - 1024;
@@ -344,7 +350,7 @@ cudaError_t eval_launch(const DevGraph& g, const EvalConfig& cfg, void* gws, int
                         const int32_t* perm, const uint8_t* dec, uint8_t* status,
                         int64_t* peak, double* lat, cudaStream_t stream) {
     if (K <= 0) return cudaSuccess;
-    StateLayout L = state_layout(g.NT, g.R, g.max_events);
+    StateLayout L = state_layout(g.NT, g.R, g.max_events, g.Rd);
     const int grid = (int)std::min<int64_t>(cfg.grid, K);
     if (cfg.variant == 0) {
         eval_kernel<false><<<grid, kBlock, cfg.smem, stream>>>(g, K, perm, dec, status, peak, lat,

@@ -404,6 +404,7 @@ extern "C" int magis_ghash_create(const magis_graph* g, const uint64_t* h_label,
     if (!out) return set_error(MAGIS_E_INVAL, "out is NULL");
     *out = nullptr;
     if (!g || !h_label) return set_error(MAGIS_E_INVAL, "null argument");
+    if (g->dev.F > 0) return set_error(MAGIS_E_UNSUPPORTED, "magis_ghash_create: not available on graphs with F-Trans regions");
     const int32_t n = g->dev.n, R = g->dev.R, NT = g->dev.NT;
     const auto& pp = g->h_pred_ptr;
     const auto& pr = g->h_pred;

@@ -96,12 +96,37 @@ cudaError_t dispatch_eval(const magis_graph* g, int64_t K, const int32_t* perm, 
 }  // namespace
 
 extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_graph** out) {
+    return magis_graph_load_regions(d, nullptr, device, out);
+}
+
+extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_region_desc* rd, int device,
+                                        magis_graph** out) {
     clear_error();
     if (!out) return set_error(MAGIS_E_INVAL, "out is NULL");
     *out = nullptr;
     if (!d) return set_error(MAGIS_E_INVAL, "desc is NULL");
     const int32_t n = d->n_nodes;
     const int32_t R = d->n_eligible;
+    // --- F-Trans variant regions (NEXT-4, reading F1) -------------------------
+    const int32_t F = rd ? rd->n_regions : 0;
+    if (F < 0) return set_error(MAGIS_E_INVAL, "n_regions < 0");
+    if (F > 0 && (!rd->n_variants || !rd->node_region || !rd->node_variant))
+        return set_error(MAGIS_E_INVAL, "null region array");
+    if ((int64_t)R + F > (1 << 23)) return set_error(MAGIS_E_UNSUPPORTED, "n_eligible + n_regions > 2^23");
+    std::vector<int32_t> nreg(n, -1);         // gate of an original node: -1 or (R + region) << 2 | variant
+    for (int32_t i = 0; i < F; i++)
+        if (rd->n_variants[i] < 1 || rd->n_variants[i] > 4)
+            return set_error(MAGIS_E_INVAL, "n_variants must be in 1..4 (region " + std::to_string(i) + ")");
+    if (F > 0)
+        for (int32_t v = 0; v < n; v++) {
+            const int32_t ri = rd->node_region[v];
+            if (ri < -1 || ri >= F) return set_error(MAGIS_E_INVAL, "node_region out of range at node " + std::to_string(v));
+            if (ri >= 0) {
+                if (rd->node_variant[v] >= rd->n_variants[ri])
+                    return set_error(MAGIS_E_INVAL, "node_variant out of range at node " + std::to_string(v));
+                nreg[v] = ((R + ri) << 2) | rd->node_variant[v];
+            }
+        }
     if (n < 1) return set_error(MAGIS_E_INVAL, "n_nodes < 1");
     if (R < 0) return set_error(MAGIS_E_INVAL, "n_eligible < 0");
     if (d->n_edges < 0) return set_error(MAGIS_E_INVAL, "n_edges < 0");
@@ -132,6 +157,8 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
         if (u < 0 || u >= n || v < 0 || v >= n)
             return set_error(MAGIS_E_INVAL, "edge id out of range at edge " + std::to_string(e));
         if (u == v) return set_error(MAGIS_E_INVAL, "self-loop at node " + std::to_string(u));
+        if (nreg[u] >= 0 && nreg[v] >= 0 && nreg[u] != nreg[v])
+            return set_error(MAGIS_E_INVAL, "edge between different F-Trans variants at edge " + std::to_string(e));
         keys.push_back(((uint64_t)(uint32_t)u << 32) | (uint32_t)v);
     }
     std::sort(keys.begin(), keys.end());
@@ -220,6 +247,10 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
         int32_t t = d->eligible_tensor[r];
         if (t < 0 || t >= n) return set_error(MAGIS_E_INVAL, "eligible id out of range");
         if (d->is_output[t]) return set_error(MAGIS_E_INVAL, "graph output marked eligible: " + std::to_string(t));
+        if (nreg[t] >= 0) return set_error(MAGIS_E_INVAL, "eligible tensor inside an F-Trans region: " + std::to_string(t));
+        for (int32_t e = pred_ptr[t]; e < pred_ptr[t + 1]; e++)
+            if (nreg[pred[e]] >= 0)
+                return set_error(MAGIS_E_INVAL, "eligible tensor reads an F-Trans region: " + std::to_string(t));
         if (r_of[t] >= 0) return set_error(MAGIS_E_INVAL, "duplicate eligible tensor " + std::to_string(t));
         r_of[t] = r;
         int64_t a = d->late_user_ptr[r], b = d->late_user_ptr[r + 1];
@@ -231,6 +262,7 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
         for (int32_t bb : us) {
             if (bb < 0 || bb >= n || !std::binary_search(succ.begin() + succ_ptr[t], succ.begin() + succ_ptr[t + 1], bb))
                 return set_error(MAGIS_E_INVAL, "U_r not a subset of cons(t_r) for r=" + std::to_string(r));
+            if (nreg[bb] >= 0) return set_error(MAGIS_E_INVAL, "late user inside an F-Trans region for r=" + std::to_string(r));
         }
     }
     const int32_t NT = n + 3 * R;
@@ -252,7 +284,7 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
             se.push_back({n + 3 * r, v, (r << 2) | 1});      // clone_r -> b (dec 1)
             se.push_back({n + 3 * r + 2, v, (r << 2) | 2});  // load_r -> b (dec 2)
         } else {
-            se.push_back({u, v, kAlways});
+            se.push_back({u, v, nreg[u] >= 0 ? nreg[u] : nreg[v]});   // kAlways (-1) outside regions
         }
     }
     for (int32_t r = 0; r < R; r++) {
@@ -281,11 +313,16 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     std::vector<int32_t> ngate(NT, kAlways);
     std::vector<uint8_t> nflag(NT, 0);
     double base_cost = 0.0;
+    std::vector<int32_t> nvar(std::max(F, 1), 1);
+    std::vector<double> vcost((size_t)4 * std::max(F, 1), 0.0);
+    for (int32_t i = 0; i < F; i++) nvar[i] = rd->n_variants[i];
     for (int32_t v = 0; v < n; v++) {
         size[v] = d->out_bytes[v];
         cost[v] = d->cost[v];
         nflag[v] = (uint8_t)((d->is_output[v] ? kFlagOutput : 0) | kFlagCompute);
-        base_cost += d->cost[v];
+        ngate[v] = nreg[v];
+        if (nreg[v] >= 0) vcost[(size_t)4 * ((nreg[v] >> 2) - R) + (nreg[v] & 3)] += d->cost[v];
+        else base_cost += d->cost[v];
     }
     std::vector<int32_t> elig(R), U_ptr(R + 1, 0), U_idx((size_t)nU);
     std::vector<double> xfer(R), tcost(R);
@@ -342,6 +379,8 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     size_t o_p = add(pred.data(), pred.size() * 4);
     size_t o_dtin = add(dtin.data(), dtin.size() * 4);
     size_t o_dtout = add(dtout.data(), dtout.size() * 4);
+    size_t o_nvar = add(nvar.data(), nvar.size() * 4);
+    size_t o_vcost = add(vcost.data(), vcost.size() * 8);
     g->blob_bytes = off;
     cudaError_t e = cudaMalloc(&g->blob, off);
     if (e != cudaSuccess) {
@@ -384,6 +423,10 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     dg.dtout = (const int32_t*)(b + o_dtout);
     dg.pred_ptr = (const int32_t*)(b + o_pp);
     dg.pred = (const int32_t*)(b + o_p);
+    dg.F = F;
+    dg.Rd = R + F;
+    dg.nvar = (const int32_t*)(b + o_nvar);
+    dg.vcost = (const double*)(b + o_vcost);
     g->idom = idom;
     // host copies for plans built after load (GraphHash, NEXT-2)
     g->h_pred_ptr = pred_ptr;
@@ -409,7 +452,7 @@ extern "C" int magis_graph_load(const magis_graph_desc* d, int device, magis_gra
     {
         const char* force = std::getenv("MAGIS_VARIANT");
         const char* pforce = std::getenv("MAGIS_P");
-        const bool allow2 = !(force && std::atoi(force) != 2);
+        const bool allow2 = !(force && std::atoi(force) != 2) && F == 0;   // variant 2 folds only Fig. 8 gates
         cudaDeviceProp prop;
         if (allow2 && cudaGetDeviceProperties(&prop, device) == cudaSuccess) {
             std::vector<double> rtab((size_t)2 * R);
@@ -531,6 +574,7 @@ extern "C" int magis_graph_info_get(const magis_graph* g, magis_graph_info* info
     info->table_bytes = (int64_t)g->blob_bytes;
     info->base_cost = g->dev.base_cost;
     info->pack = g->cfg.variant == 2 ? g->plan2.P : 1;
+    info->n_regions = g->dev.F;
     return MAGIS_SUCCESS;
 }
 
@@ -543,7 +587,7 @@ extern "C" int magis_eval_schedules(const magis_graph* g, int64_t K, const int32
     if (K == 0) return MAGIS_SUCCESS;
     if (!d_perm || !d_status || !d_peak || !d_latency)
         return set_error(MAGIS_E_INVAL, "null device pointer");
-    if (g->dev.R > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R > 0");
+    if (g->dev.Rd > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R + n_regions > 0");
     DeviceGuard guard(g->device);
     cudaError_t e = dispatch_eval(g, K, d_perm, d_dec, d_status, d_peak, d_latency,
                                   (cudaStream_t)cuda_stream);
@@ -559,12 +603,13 @@ extern "C" int magis_hotspots(magis_graph* g, int64_t K, const int32_t* d_perm, 
                               int32_t nsplit, uint8_t* d_status, int64_t* d_peak, uint8_t* d_hot,
                               int64_t* d_heat, double* d_score, void* cuda_stream) {
     clear_error();
+    if (g && g->dev.F > 0) return set_error(MAGIS_E_UNSUPPORTED, "magis_hotspots: not available on graphs with F-Trans regions");
     if (!g) return set_error(MAGIS_E_INVAL, "graph is NULL");
     if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
     if (nsplit < 1) return set_error(MAGIS_E_INVAL, "nsplit < 1");
     if (K == 0) return MAGIS_SUCCESS;
     if (!d_perm || !d_status || !d_peak || !d_hot) return set_error(MAGIS_E_INVAL, "null device pointer");
-    if (g->dev.R > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R > 0");
+    if (g->dev.Rd > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R + n_regions > 0");
     DeviceGuard guard(g->device);
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device);
@@ -611,8 +656,8 @@ int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8
     if (K == 0) return MAGIS_SUCCESS;
     if (!h_perm || !h_status || !h_peak || !h_latency)
         return set_error(MAGIS_E_INVAL, "null host pointer");
-    const int32_t R = g->dev.R, NT = g->dev.NT;
-    if (R > 0 && !h_dec) return set_error(MAGIS_E_INVAL, "h_dec is NULL but R > 0");
+    const int32_t R = g->dev.Rd, NT = g->dev.NT;          // decision row: R eligible + F regions
+    if (R > 0 && !h_dec) return set_error(MAGIS_E_INVAL, "h_dec is NULL but R + n_regions > 0");
     if (pb == 2 && NT > 65535) return set_error(MAGIS_E_UNSUPPORTED, "uint16 schedules need n_total <= 65535");
     DeviceGuard guard(g->device);
     cudaStream_t s0 = (cudaStream_t)cuda_stream;
@@ -692,6 +737,7 @@ extern "C" int magis_eval_schedules_host_u16(magis_graph* g, int64_t K, const ui
 extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* spec, uint64_t id0, int64_t K,
                                          int32_t* d_perm, uint8_t* d_dec, void* cuda_stream) {
     clear_error();
+    if (g && g->dev.F > 0) return set_error(MAGIS_E_UNSUPPORTED, "magis_generate_candidates: not available on graphs with F-Trans regions");
     if (!g || !spec) return set_error(MAGIS_E_INVAL, "null argument");
     if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
     if (K == 0) return MAGIS_SUCCESS;
@@ -720,10 +766,11 @@ extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* s
 extern "C" int magis_base_create(magis_graph* g, const int32_t* d_perm, const uint8_t* d_dec, magis_base** out,
                                  void* cuda_stream) {
     clear_error();
+    if (g && g->dev.F > 0) return set_error(MAGIS_E_UNSUPPORTED, "magis_base_create: not available on graphs with F-Trans regions");
     if (!out) return set_error(MAGIS_E_INVAL, "out is NULL");
     *out = nullptr;
     if (!g || !d_perm) return set_error(MAGIS_E_INVAL, "null argument");
-    if (g->dev.R > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R > 0");
+    if (g->dev.Rd > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R + n_regions > 0");
     DeviceGuard guard(g->device);
     magis_base* b = new (std::nothrow) magis_base();
     if (!b) return set_error(MAGIS_E_NOMEM, "host allocation failed");

@@ -55,6 +55,13 @@ struct DevGraph {
     const int32_t* dtout;      // [n] end of the node's preorder range
     const int32_t* pred_ptr;   // [n+1] predecessors in G (deduplicated)
     const int32_t* pred;
+    // F-Trans variant regions (NEXT-4, reading F1): a candidate's decision
+    // row is [R eligible decisions | F region variants]; gates of region
+    // nodes index dec[R + i]
+    int32_t F;                 // regions (0: none)
+    int32_t Rd;                // decision row length R + F
+    const int32_t* nvar;       // [F] variants per region (<= 4)
+    const double* vcost;       // [4F] sum of cost over the nodes of (region, variant)
 };
 
 // Variant-2 plan (magis_eval2.cu): graph as per-thread streams in shared
@@ -162,7 +169,7 @@ struct EvalConfig {
 struct StateLayout {
     size_t pos, last, A, Fr, C, evkey_in, evkey_out, evcb, endT, endS, endL, dec, total;
 };
-StateLayout state_layout(int32_t NT, int32_t R, int32_t max_events);
+StateLayout state_layout(int32_t NT, int32_t R, int32_t max_events, int32_t Rd);
 
 // Host-side inputs of the variant-2 planner (super-graph in CSR form).
 struct SuperGraphHost {

@@ -27,7 +27,7 @@ EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magi
            "magis_base_create", "magis_base_info", "magis_base_free", "magis_eval_windows", "magis_hotspots",
            "magis_graph_idom", "magis_eval_schedules_host_u16", "magis_ghash_create", "magis_ghash_free",
            "magis_graph_hash", "magis_ghash_info", "magis_hashset_create", "magis_hashset_free",
-           "magis_hashset_clear", "magis_hashset_filter", "magis_hashset_stats"]
+           "magis_hashset_clear", "magis_hashset_filter", "magis_hashset_stats", "magis_graph_load_regions"]
 
 
 class MagisError(RuntimeError):
@@ -56,7 +56,12 @@ class GraphInfo(ctypes.Structure):
                 ("n_edges", ctypes.c_int64), ("n_super_edges", ctypes.c_int64), ("device", ctypes.c_int32),
                 ("variant", ctypes.c_int32), ("grid", ctypes.c_int32), ("block", ctypes.c_int32),
                 ("smem_bytes", ctypes.c_int64), ("table_bytes", ctypes.c_int64), ("base_cost", ctypes.c_double),
-                ("pack", ctypes.c_int32)]
+                ("pack", ctypes.c_int32), ("n_regions", ctypes.c_int32)]
+
+
+class RegionDesc(ctypes.Structure):
+    _fields_ = [("n_regions", ctypes.c_int32), ("n_variants", ctypes.c_void_p), ("node_region", ctypes.c_void_p),
+                ("node_variant", ctypes.c_void_p)]
 
 
 _lib = None
@@ -73,6 +78,9 @@ def lib() -> ctypes.CDLL:
     P, i32, i64, d = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_double
     L.magis_graph_load.argtypes = [ctypes.POINTER(GraphDesc), ctypes.c_int, ctypes.POINTER(P)]
     L.magis_graph_load.restype = ctypes.c_int
+    L.magis_graph_load_regions.argtypes = [ctypes.POINTER(GraphDesc), ctypes.POINTER(RegionDesc), ctypes.c_int,
+                                           ctypes.POINTER(P)]
+    L.magis_graph_load_regions.restype = ctypes.c_int
     L.magis_graph_free.argtypes = [P]
     L.magis_graph_free.restype = ctypes.c_int
     L.magis_graph_info_get.argtypes = [P, ctypes.POINTER(GraphInfo)]
@@ -157,7 +165,7 @@ class Graph:
 
     def __init__(self, out_bytes, cost, is_output, edge_src, edge_dst, eligible: Sequence[int] = (),
                  late_users: Sequence[Sequence[int]] = (), swap_bytes_per_s: float = 25e9,
-                 swap_latency_s: float = 1e-5, device: int = 0):
+                 swap_latency_s: float = 1e-5, device: int = 0, regions=None):
         L = lib()
         self._L = L
         self._h = None
@@ -177,7 +185,16 @@ class Graph:
                       _np_ptr(ed), int(el.size), _np_ptr(el), ptr.ctypes.data_as(ctypes.c_void_p),
                       _np_ptr(idx), float(swap_bytes_per_s), float(swap_latency_s))
         h = ctypes.c_void_p()
-        _check(L.magis_graph_load(ctypes.byref(d), int(device), ctypes.byref(h)))
+        if regions is None:
+            _check(L.magis_graph_load(ctypes.byref(d), int(device), ctypes.byref(h)))
+        else:
+            # F-Trans variant regions (NEXT-4): dict(n_variants, node_region, node_variant)
+            nv = np.ascontiguousarray(regions["n_variants"], np.int32)
+            nr = np.ascontiguousarray(regions["node_region"], np.int32)
+            vn = np.ascontiguousarray(regions["node_variant"], np.uint8)
+            self._keep_regions = (nv, nr, vn)
+            rd = RegionDesc(int(nv.size), _np_ptr(nv), _np_ptr(nr), _np_ptr(vn))
+            _check(L.magis_graph_load_regions(ctypes.byref(d), ctypes.byref(rd), int(device), ctypes.byref(h)))
         self._h = h
         self.device = device
         info = GraphInfo()
@@ -186,11 +203,13 @@ class Graph:
         self.n_total = info.n_total
         self.R = info.n_eligible
         self.n = info.n_nodes
+        self.F = info.n_regions
+        self.dec_len = self.R + self.F          # decision row: R eligible + F region variants
 
     @classmethod
     def from_workload(cls, wl, device: int = 0) -> "Graph":
         return cls(wl.size, wl.cost, wl.is_output, wl.src, wl.dst, wl.elig, wl.U, wl.swap_Bps,
-                   wl.swap_lat, device)
+                   wl.swap_lat, device, getattr(wl, "regions", None))
 
     def close(self):
         if self._h:
@@ -204,20 +223,20 @@ class Graph:
             pass
 
     def eval_schedules(self, perm, dec=None, status=None, peak=None, latency=None, stream=None):
-        """perm: cuda int32 [K, n_total]; dec: cuda uint8 [K, R] (or None if R == 0).
+        """perm: cuda int32 [K, n_total]; dec: cuda uint8 [K, R + F] (or None if R + F == 0).
         Returns (status uint8 [K], peak int64 [K], latency float64 [K]) device tensors."""
         import torch
         K = int(perm.shape[0])
         assert perm.dtype == torch.int32 and perm.is_cuda and perm.is_contiguous()
         assert perm.shape[1] == self.n_total, (perm.shape, self.n_total)
-        if self.R:
+        if self.dec_len:
             assert dec is not None and dec.dtype == torch.uint8 and dec.is_contiguous()
-            assert dec.shape[0] == K and dec.shape[1] == self.R
+            assert dec.shape[0] == K and dec.shape[1] == self.dec_len
         dev = perm.device
         status = torch.empty(K, dtype=torch.uint8, device=dev) if status is None else status
         peak = torch.empty(K, dtype=torch.int64, device=dev) if peak is None else peak
         latency = torch.empty(K, dtype=torch.float64, device=dev) if latency is None else latency
-        _check(self._L.magis_eval_schedules(self._h, K, _tptr(perm), _tptr(dec) if self.R else None,
+        _check(self._L.magis_eval_schedules(self._h, K, _tptr(perm), _tptr(dec) if self.dec_len else None,
                                             _tptr(status), _tptr(peak), _tptr(latency),
                                             _stream_ptr(stream)))
         return status, peak, latency
@@ -282,7 +301,7 @@ class Graph:
             p = np.ascontiguousarray(p, np.int32)
         K = p.shape[0]
         assert p.shape[1] == self.n_total
-        dd = as_np(dec, np.uint8) if (self.R and dec is not None) else None
+        dd = as_np(dec, np.uint8) if (self.dec_len and dec is not None) else None
         if out is None:
             st = np.empty(K, np.uint8)
             pk = np.empty(K, np.int64)

@@ -47,7 +47,7 @@ def test_every_declared_symbol_is_exported(lib):
 
 
 def test_abi_version_and_no_device_here(lib):
-    assert lib.magis_abi_version() == 1
+    assert lib.magis_abi_version() == 2
     import torch
     if not torch.cuda.is_available():
         assert lib.magis_device_supported(0) == 0
@@ -120,3 +120,30 @@ def test_valid_graph_needs_b200(lib):
     assert lib.magis_graph_load(ctypes.byref(d), 0, ctypes.byref(h)) == -5   # no CPU fallback
     with pytest.raises(magis.MagisError):
         magis.Graph([1, 1, 1], [0.0] * 3, [0, 0, 1], [0, 1], [1, 2])
+
+
+@pytest.mark.parametrize("reg,elig,U,code", [
+    (dict(nv=[5], nr=[-1, 0, -1, -1], vn=[0, 0, 0, 0]), (), (), -1),       # n_variants > 4
+    (dict(nv=[2], nr=[-1, 0, -1, -1], vn=[0, 2, 0, 0]), (), (), -1),       # variant out of range
+    (dict(nv=[2], nr=[-1, 3, -1, -1], vn=[0, 0, 0, 0]), (), (), -1),       # region out of range
+    (dict(nv=[2], nr=[-1, 0, 0, -1], vn=[0, 0, 1, 0]), (), (), -1),        # edge between two variants
+    (dict(nv=[2], nr=[-1, 0, -1, -1], vn=[0, 0, 0, 0]), [1], [[2]], -1),   # eligible inside a region
+    (dict(nv=[2], nr=[-1, 0, -1, -1], vn=[0, 0, 0, 0]), [2], [[3]], -1),   # eligible reads a region
+    (dict(nv=[2], nr=[-1, -1, 0, -1], vn=[0, 0, 0, 0]), [1], [[2]], -1),   # late user inside a region
+    (dict(nv=[2], nr=[-1, 0, -1, -1], vn=[0, 0, 0, 0]), (), (), -5),       # valid: needs the B200
+])
+def test_region_validation_without_gpu(lib, reg, elig, U, code):
+    """F-Trans variant regions (NEXT-4, reading F1) are validated on the host."""
+    import torch
+    if torch.cuda.is_available() and code == -5:
+        pytest.skip("GPU present")
+    # chain 0 -> 1 -> 2 -> 3 plus 1 -> 3
+    d, keep = _desc(4, [4, 4, 4, 4], [0.0, 1.0, 1.0, 1.0], [0, 0, 0, 1], [0, 1, 2, 1], [1, 2, 3, 3], elig, U)
+    nv = np.asarray(reg["nv"], np.int32)
+    nr = np.asarray(reg["nr"], np.int32)
+    vn = np.asarray(reg["vn"], np.uint8)
+    rd = magis.RegionDesc(len(nv), nv.ctypes.data_as(ctypes.c_void_p), nr.ctypes.data_as(ctypes.c_void_p),
+                          vn.ctypes.data_as(ctypes.c_void_p))
+    h = ctypes.c_void_p()
+    rc = lib.magis_graph_load_regions(ctypes.byref(d), ctypes.byref(rd), 0, ctypes.byref(h))
+    assert rc == code, lib.magis_last_error()
