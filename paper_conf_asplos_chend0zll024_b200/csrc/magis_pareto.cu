@@ -28,7 +28,7 @@ constexpr int kPB = 512;           // threads per K1 / K3 block
 constexpr int kPer = kCH / kPB;    // 8 points per thread
 constexpr int kSmemChunk = kCH * 26;   // pk, lt, ix (8 B each) + ord (2 B)
 
-__device__ unsigned long long g_pareto_dummy[2];
+__device__ unsigned long long g_pareto_dummy[3];
 
 struct PWs {
     int64_t* spk;   // [C*CH] staircase peaks
@@ -38,7 +38,7 @@ struct PWs {
     int32_t* pref;  // [C*CH]
     int32_t* cnt;   // [C]
     int32_t* tot;   // [C]
-    unsigned long long* ctr;   // [2]: cntM, cntL
+    unsigned long long* ctr;   // [3]: cntM, cntL, front size
 };
 
 static size_t a256(size_t x) { return (x + 255) / 256 * 256; }
@@ -74,6 +74,7 @@ __device__ __forceinline__ bool key_less(long long pa, double la, long long ia, 
 __global__ void pareto_init(PWs w, int64_t* front_n, int64_t* best) {
     w.ctr[0] = 0;
     w.ctr[1] = 0;
+    w.ctr[2] = 0;
     *front_n = 0;
     if (best) { best[0] = -1; best[1] = -1; }
 }
@@ -267,7 +268,10 @@ pareto_count(PWs w, int64_t mem_limit, double lat_limit) {
         if (i < cnt) w.pref[base + i] = r;
         r += f[q];
     }
-    if (tid == 0) w.tot[c] = wcnt[kPB / 32];
+    if (tid == 0) {
+        w.tot[c] = wcnt[kPB / 32];
+        atomicAdd(&w.ctr[2], (unsigned long long)wcnt[kPB / 32]);
+    }
     for (int o = 16; o > 0; o >>= 1) {
         cm += __shfl_xor_sync(0xffffffffu, cm, o);
         cl += __shfl_xor_sync(0xffffffffu, cl, o);
@@ -280,9 +284,7 @@ __global__ void pareto_scatter(int64_t C, PWs w, int64_t cap, int64_t* front_id,
                                int64_t* front_peak, double* front_lat, int64_t* front_n,
                                int64_t mem_limit, double lat_limit, int64_t* best) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    // total front size (every thread needs it for the latency-limit query)
-    int64_t nf = 0;
-    for (int64_t c2 = 0; c2 < C; c2++) nf += w.tot[c2];
+    const int64_t nf = (int64_t)w.ctr[2];              // total front size (pareto_count)
     if (t == 0) *front_n = nf;
     const int64_t c = t / kCH;
     const int i = (int)(t % kCH);
@@ -316,10 +318,9 @@ __global__ void pareto_scatter(int64_t C, PWs w, int64_t cap, int64_t* front_id,
 
 // fill front entries [front_n, cap) with padding (id -1, peak -1, lat +inf) so a
 // padded front can be all-gathered and merged directly (ids < 0 are ignored).
-__global__ void pareto_pad(int64_t C, const int32_t* tot, int64_t cap, int64_t* front_id,
+__global__ void pareto_pad(const unsigned long long* nfp, int64_t cap, int64_t* front_id,
                            int64_t* front_peak, double* front_lat) {
-    int64_t nf = 0;
-    for (int64_t c2 = 0; c2 < C; c2++) nf += tot[c2];
+    const int64_t nf = nfp ? (int64_t)*nfp : 0;
     for (int64_t r = nf + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < cap;
          r += (int64_t)gridDim.x * blockDim.x) {
         front_id[r] = -1;
@@ -345,7 +346,7 @@ cudaError_t pareto_launch(int64_t n, const int64_t* peak, const double* lat,
         pareto_init<<<1, 1, 0, stream>>>(w0, front_n, best);
         if (cap > 0)
             pareto_pad<<<(unsigned)std::min<int64_t>((cap + 255) / 256, 1024), 256, 0, stream>>>(
-                0, nullptr, cap, front_id, front_peak, front_lat);
+                nullptr, cap, front_id, front_peak, front_lat);
         return cudaGetLastError();
     }
     {
@@ -363,7 +364,7 @@ cudaError_t pareto_launch(int64_t n, const int64_t* peak, const double* lat,
                                                mem_limit, lat_limit, best);
     if (cap > 0)
         pareto_pad<<<(unsigned)std::min<int64_t>((cap + 255) / 256, 1024), 256, 0, stream>>>(
-            C, w.tot, cap, front_id, front_peak, front_lat);
+            w.ctr + 2, cap, front_id, front_peak, front_lat);
     return cudaGetLastError();
 }
 
