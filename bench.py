@@ -43,7 +43,8 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU-baseline wall time")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--e2e-int32", action="store_true", help="e2e with int32 host schedules instead of uint16")
+    ap.add_argument("--e2e-wire", default="delta8", choices=["delta8", "u16", "int32"],
+                    help="host schedule format of the e2e call (delta8 / u16 need n_total <= 65535)")
     ap.add_argument("--ghash", action="store_true",
                     help="batched GraphHash + duplicate filter of the K candidates' graphs (NEXT-2)")
     ap.add_argument("--windows", action="store_true",
@@ -324,10 +325,20 @@ def main():
         hlt = np.empty(K, np.float64)
         out_pinned = (torch.empty(K, dtype=torch.uint8).pin_memory(), torch.empty(K, dtype=torch.int64).pin_memory(),
                       torch.empty(K, dtype=torch.float64).pin_memory())
-        # schedules cross PCIe in the compact uint16 wire format when the
-        # super-graph has < 65536 nodes (magis_eval_schedules_host_u16)
-        u16 = NT <= 65535 and not args.e2e_int32
-        Ph_w = torch.from_numpy(Ph.astype(np.uint16)).pin_memory() if u16 else Ph_t
+        # schedules cross PCIe in a compact wire format when the super-graph
+        # has < 65536 nodes: delta8 (~1.1 B / step, magis_eval_schedules_host_delta8)
+        # or u16 (magis_eval_schedules_host_u16); encoded once, outside the timed region
+        wire = args.e2e_wire if NT <= 65535 else "int32"
+        from paper_conf_asplos_chend0zll024_b200 import encode_delta8
+        if wire == "delta8":
+            Ph_w = tuple(torch.from_numpy(a).pin_memory() for a in encode_delta8(Ph))
+            wire_bytes = sum(int(a.numel()) * a.element_size() for a in Ph_w)
+        elif wire == "u16":
+            Ph_w = torch.from_numpy(Ph.astype(np.uint16)).pin_memory()
+            wire_bytes = K * NT * 2
+        else:
+            Ph_w = Ph_t
+            wire_bytes = K * NT * 4
         g.eval_schedules_host(Ph_w, Dh_t, out=out_pinned)     # warm (allocates staging once)
         if world > 1:
             dist.barrier()
@@ -339,10 +350,11 @@ def main():
         te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        api = ("magis_eval_schedules_host_u16 (uint16 schedules" if u16 else
-               "magis_eval_schedules_host (int32 schedules")
+        api = {"delta8": "magis_eval_schedules_host_delta8 (delta8 schedules",
+               "u16": "magis_eval_schedules_host_u16 (uint16 schedules",
+               "int32": "magis_eval_schedules_host (int32 schedules"}[wire]
         e2e = {"value": round(world * K / te.item(), 1), "unit": UNIT,
-               "h2d_bytes_per_step": int(K * NT * (2 if u16 else 4) + K * g.dec_len), "d2h_bytes_per_step": int(K * 17),
+               "h2d_bytes_per_step": int(wire_bytes + K * g.dec_len), "d2h_bytes_per_step": int(K * 17),
                "api": api + ", pinned host buffers, chunked double-buffered copies)",
                "s_per_step": round(te.item(), 5)}
         ok_same = bool((out_pinned[1].numpy() == pk.cpu().numpy()).all())

@@ -217,6 +217,25 @@ int magis_eval_schedules_host_u16(magis_graph* g, int64_t K, const uint16_t* h_p
                                   double* h_latency, void* cuda_stream);
 
 /*
+ * As magis_eval_schedules_host with the schedules in the delta8 wire format
+ * (n_total <= 65535): per step one signed byte, the difference between this
+ * step's node id and the previous step's (a row starts from 0); the byte -128
+ * means "the next value of this row's exception list", an absolute uint16
+ * id.  h_delta [K x n_total] int8; h_exc_ptr [K + 1] int32 (row k's
+ * exceptions are h_exc[h_exc_ptr[k] .. h_exc_ptr[k+1]), nondecreasing);
+ * h_exc uint16 (may be NULL if there are none).  Random topological orders
+ * of DNN graphs move by small id steps, so this is ~1.1 bytes per step
+ * instead of 2 (u16) or 4 (int32) across PCIe; the device decodes each
+ * chunk (a segmented warp scan) before evaluating it.  Ids >= n_total (e.g. a
+ * clamped out-of-range id) give MAGIS_ST_NOT_PERM as usual.
+ * Errors as magis_eval_schedules_host_u16, plus MAGIS_E_INVAL for
+ * decreasing offsets.
+ */
+int magis_eval_schedules_host_delta8(magis_graph* g, int64_t K, const int8_t* h_delta, const int32_t* h_exc_ptr,
+                                     const uint16_t* h_exc, const uint8_t* h_dec, uint8_t* h_status,
+                                     int64_t* h_peak, double* h_latency, void* cuda_stream);
+
+/*
  * Seeded candidate generation on the device.  Candidate k
  * (global id id0 + i) depends only on (spec->seed, k), so ranks generate
  * their shards independently.  The recipe stands in for MAGIS's rule

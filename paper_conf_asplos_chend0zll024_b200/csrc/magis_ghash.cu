@@ -173,6 +173,7 @@ struct Lanes {
         return (decp[(r >> 4) * 32 + lane] >> (2 * (r & 15))) & 3u;
     }
     __device__ __forceinline__ uint64_t get(uint32_t e) const {
+        if (!(e & (kLU | kConst | kGlob))) return xs[e * 32 + lane];     // the common case first
         uint32_t s = e;
         if (e & kLU) {
             const uint4 rs = __ldg(d.rslot + (e & kIdx));
@@ -184,9 +185,8 @@ struct Lanes {
         return xs[s * 32 + lane];
     }
     __device__ __forceinline__ void put(uint32_t s, uint64_t h) const {
-        if (s == kNoSlot) return;
-        if (s & kGlob) gb[(size_t)(s & kIdx) * 32 + lane] = h;
-        else xs[s * 32 + lane] = h;
+        if (!(s & kGlob)) xs[s * 32 + lane] = h;                        // kNoSlot has every bit set
+        else if (s != kNoSlot) gb[(size_t)(s & kIdx) * 32 + lane] = h;
     }
 };
 
@@ -300,7 +300,6 @@ ghash_kernel(GhDev d, int64_t K, const uint8_t* __restrict__ dec, int vec, uint8
                     default: group_dispatch<4>(L, deg, rec, ent, sum); break;
                 }
                 i += G;
-                __syncwarp();
                 continue;
             }
             const uint4 rec = __ldg(d.nrec + i);
@@ -368,7 +367,7 @@ ghash_kernel(GhDev d, int64_t K, const uint8_t* __restrict__ dec, int vec, uint8
                 sum += h;
                 L.put(rec.z, h);
             }
-            __syncwarp();
+            // no __syncwarp: every lane reads and writes only its own column
         }
         if (valid) {
             out_status[k] = bad ? (uint8_t)MAGIS_ST_BAD_DEC : (uint8_t)0;

@@ -647,9 +647,48 @@ __global__ void widen_u16(const uint16_t* __restrict__ src, int32_t* __restrict_
         dst[i] = (int32_t)src[i];
 }
 
-// pb = bytes per perm element on the host (4: int32, 2: uint16, widened on the device)
+// delta8 wire format: per step one int8 delta to the previous step's id
+// (the row starts from 0); -128 = "take the next value of the row's
+// exception list" (an absolute uint16 id).  One warp per row: the exception
+// ranks come from a ballot, and a segmented scan over (reset, value) pairs
+// rebuilds the ids 32 steps at a time.
+__global__ void decode_delta8(const int8_t* __restrict__ delta, const int32_t* __restrict__ exc_ptr,
+                              const uint16_t* __restrict__ exc, int64_t kc, int32_t NT, int32_t* __restrict__ out) {
+    const int lane = threadIdx.x & 31;
+    const int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int32_t e0 = exc_ptr[0];
+    for (int64_t k = w0; k < kc; k += nw) {
+        const int8_t* dr = delta + k * (int64_t)NT;
+        int32_t* orow = out + k * (int64_t)NT;
+        int32_t carry = 0, ec = exc_ptr[k] - e0;
+        for (int32_t t = 0; t < NT; t += 32) {
+            const int32_t j = t + lane;
+            const int32_t b = j < NT ? (int32_t)dr[j] : 0;
+            const bool isx = j < NT && b == -128;
+            const unsigned m = __ballot_sync(0xffffffffu, isx);
+            int32_t v = isx ? (int32_t)exc[ec + __popc(m & ((1u << lane) - 1u))] : b;
+            bool rs = isx;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int32_t pv = __shfl_up_sync(0xffffffffu, v, o);
+                const bool pr = __shfl_up_sync(0xffffffffu, (int)rs, o);
+                if (lane >= o && !rs) { v += pv; rs = pr; }
+            }
+            if (!rs) v += carry;
+            if (j < NT) orow[j] = v;
+            carry = __shfl_sync(0xffffffffu, v, 31);
+            ec += __popc(m);
+        }
+    }
+}
+
+// pb = bytes per perm element on the host (4: int32, 2: uint16 widened on the
+// device, 1: delta8 decoded on the device -- h_exc_ptr / h_exc then hold the
+// exception lists)
 int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8_t* h_dec, uint8_t* h_status,
-              int64_t* h_peak, double* h_latency, void* cuda_stream) {
+              int64_t* h_peak, double* h_latency, void* cuda_stream, const int32_t* h_exc_ptr = nullptr,
+              const uint16_t* h_exc = nullptr) {
     clear_error();
     if (!g) return set_error(MAGIS_E_INVAL, "graph is NULL");
     if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
@@ -658,7 +697,13 @@ int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8
         return set_error(MAGIS_E_INVAL, "null host pointer");
     const int32_t R = g->dev.Rd, NT = g->dev.NT;          // decision row: R eligible + F regions
     if (R > 0 && !h_dec) return set_error(MAGIS_E_INVAL, "h_dec is NULL but R + n_regions > 0");
-    if (pb == 2 && NT > 65535) return set_error(MAGIS_E_UNSUPPORTED, "uint16 schedules need n_total <= 65535");
+    if (pb <= 2 && NT > 65535) return set_error(MAGIS_E_UNSUPPORTED, "compact schedules need n_total <= 65535");
+    if (pb == 1) {
+        if (!h_exc_ptr) return set_error(MAGIS_E_INVAL, "null exception pointer array");
+        for (int64_t k = 0; k < K; k++)
+            if (h_exc_ptr[k + 1] < h_exc_ptr[k]) return set_error(MAGIS_E_INVAL, "exception offsets decrease");
+        if (h_exc_ptr[K] > h_exc_ptr[0] && !h_exc) return set_error(MAGIS_E_INVAL, "null exception array");
+    }
     DeviceGuard guard(g->device);
     cudaStream_t s0 = (cudaStream_t)cuda_stream;
     // chunk of ~64 MiB of int32 perms
@@ -668,11 +713,12 @@ int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8
     const size_t narrow_b = align_up((size_t)chunk * NT * 2, 256);
     const size_t dec_b = align_up((size_t)chunk * std::max(R, 1), 256);
     const size_t out_b = align_up((size_t)chunk * 17, 256);
+    const size_t excp_b = align_up((size_t)(chunk + 1) * 4, 256);   // delta8: exception offsets, then values
     if (g->stage_K < chunk) {
         for (int i = 0; i < 2; i++) {
             if (g->stage[i]) cudaFree(g->stage[i]);
             g->stage[i] = nullptr;
-            CK(cudaMalloc(&g->stage[i], perm_b + narrow_b + dec_b + out_b + 256));
+            CK(cudaMalloc(&g->stage[i], perm_b + narrow_b + dec_b + out_b + 256 + excp_b + narrow_b + 256));
             if (!g->ev_h2d[i]) CK(cudaEventCreateWithFlags(&g->ev_h2d[i], cudaEventDisableTiming));
             if (!g->ev_done[i]) CK(cudaEventCreateWithFlags(&g->ev_done[i], cudaEventDisableTiming));
         }
@@ -695,10 +741,21 @@ int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8
         // buffer b is free once the D2H of chunk c-2 finished
         if (c >= 2) CK(cudaStreamWaitEvent(g->aux, g->ev_done[b], 0));
         const char* hp = (const char*)h_perm + (size_t)k0 * NT * pb;
+        int32_t* dxp = (int32_t*)(ob + out_b + 256);    // past the outputs (which may spill 128 B over out_b)
+        uint16_t* dxv = (uint16_t*)((char*)dxp + excp_b);
         CK(cudaMemcpyAsync(pb == 4 ? (void*)dp : (void*)dn, hp, (size_t)kc * NT * pb, cudaMemcpyHostToDevice, g->aux));
+        if (pb == 1) {
+            const int64_t x0 = h_exc_ptr[k0], x1 = h_exc_ptr[k0 + kc];
+            CK(cudaMemcpyAsync(dxp, h_exc_ptr + k0, (size_t)(kc + 1) * 4, cudaMemcpyHostToDevice, g->aux));
+            if (x1 > x0) CK(cudaMemcpyAsync(dxv, h_exc + x0, (size_t)(x1 - x0) * 2, cudaMemcpyHostToDevice, g->aux));
+        }
         if (R > 0) CK(cudaMemcpyAsync(dd, h_dec + k0 * R, (size_t)kc * R, cudaMemcpyHostToDevice, g->aux));
         CK(cudaEventRecord(g->ev_h2d[b], g->aux));
         CK(cudaStreamWaitEvent(s0, g->ev_h2d[b], 0));
+        if (pb == 1) {
+            const int blocks = (int)std::min<int64_t>((kc + 7) / 8, 4096);
+            decode_delta8<<<blocks, 256, 0, s0>>>((const int8_t*)dn, dxp, dxv, kc, NT, dp);
+        }
         if (pb == 2) {
             const int64_t ne = kc * (int64_t)NT;
             const int blocks = (int)std::min<int64_t>((ne + 255) / 256, 4096);
@@ -732,6 +789,13 @@ extern "C" int magis_eval_schedules_host_u16(magis_graph* g, int64_t K, const ui
                                              int64_t* h_peak, double* h_latency,
                                              void* cuda_stream) {
     return host_path(g, K, h_perm, 2, h_dec, h_status, h_peak, h_latency, cuda_stream);
+}
+
+extern "C" int magis_eval_schedules_host_delta8(magis_graph* g, int64_t K, const int8_t* h_delta,
+                                                const int32_t* h_exc_ptr, const uint16_t* h_exc,
+                                                const uint8_t* h_dec, uint8_t* h_status, int64_t* h_peak,
+                                                double* h_latency, void* cuda_stream) {
+    return host_path(g, K, h_delta, 1, h_dec, h_status, h_peak, h_latency, cuda_stream, h_exc_ptr, h_exc);
 }
 
 extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* spec, uint64_t id0, int64_t K,

@@ -27,7 +27,8 @@ EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magi
            "magis_base_create", "magis_base_info", "magis_base_free", "magis_eval_windows", "magis_hotspots",
            "magis_graph_idom", "magis_eval_schedules_host_u16", "magis_ghash_create", "magis_ghash_free",
            "magis_graph_hash", "magis_ghash_info", "magis_hashset_create", "magis_hashset_free",
-           "magis_hashset_clear", "magis_hashset_filter", "magis_hashset_stats", "magis_graph_load_regions"]
+           "magis_hashset_clear", "magis_hashset_filter", "magis_hashset_stats", "magis_graph_load_regions",
+           "magis_eval_schedules_host_delta8"]
 
 
 class MagisError(RuntimeError):
@@ -91,6 +92,8 @@ def lib() -> ctypes.CDLL:
     L.magis_eval_schedules_host.restype = ctypes.c_int
     L.magis_eval_schedules_host_u16.argtypes = [P, i64, P, P, P, P, P, P]
     L.magis_eval_schedules_host_u16.restype = ctypes.c_int
+    L.magis_eval_schedules_host_delta8.argtypes = [P, i64, P, P, P, P, P, P, P, P]
+    L.magis_eval_schedules_host_delta8.restype = ctypes.c_int
     L.magis_pareto_workspace_size.argtypes = [i64]
     L.magis_pareto_workspace_size.restype = i64
     L.magis_pareto_merge.argtypes = [i64, P, P, P, P, i64, i64, P, P, P, P, i64, d, P, P, i64, P]
@@ -156,6 +159,28 @@ def _stream_ptr(stream) -> Optional[ctypes.c_void_p]:
     if stream is None:
         stream = torch.cuda.current_stream()
     return ctypes.c_void_p(stream.cuda_stream)
+
+
+def encode_delta8(perm: np.ndarray):
+    """The delta8 wire format of magis_eval_schedules_host_delta8 (marshalling
+    only): per step the int8 difference to the previous step's id (rows start
+    from 0), -128 where it does not fit, with the absolute ids of those steps
+    in a per-row exception list.  Ids outside [0, 65535] are clamped to 65535
+    (still out of range for any graph the format supports, so the candidate
+    stays MAGIS_ST_NOT_PERM).  -> (delta int8 [K, n], exc_ptr int32 [K+1],
+    exc uint16 [E])."""
+    p = np.asarray(perm, np.int64)
+    if p.ndim == 1:
+        p = p[None, :]
+    p = np.where((p < 0) | (p > 65535), 65535, p)
+    prev = np.concatenate([np.zeros((p.shape[0], 1), np.int64), p[:, :-1]], axis=1)
+    d = p - prev
+    esc = (d < -127) | (d > 127)
+    delta = np.where(esc, -128, d).astype(np.int8)
+    exc = np.ascontiguousarray(p[esc], np.uint16)
+    exc_ptr = np.zeros(p.shape[0] + 1, np.int32)
+    np.cumsum(esc.sum(axis=1), out=exc_ptr[1:])
+    return np.ascontiguousarray(delta), exc_ptr, exc
 
 
 class Graph:
@@ -287,14 +312,29 @@ class Graph:
     def eval_schedules_host(self, perm: np.ndarray, dec: Optional[np.ndarray] = None, out=None,
                             stream=None):
         """End-to-end call with host buffers (pinned numpy views or torch CPU
-        tensors).  uint16 schedules use the compact wire format
-        (magis_eval_schedules_host_u16), anything else is taken as int32."""
+        tensors).  A (delta, exc_ptr, exc) tuple from encode_delta8 uses the
+        delta8 wire format (magis_eval_schedules_host_delta8); uint16
+        schedules the u16 format (magis_eval_schedules_host_u16); anything
+        else is taken as int32."""
         import torch
 
         def as_np(x, dt):
             if isinstance(x, torch.Tensor):
                 return x.numpy()
             return np.ascontiguousarray(x, dt)
+        if isinstance(perm, tuple):           # delta8 wire format (encode_delta8)
+            delta, exc_ptr, exc = (as_np(x, None) for x in perm)
+            K = delta.shape[0]
+            assert delta.dtype == np.int8 and delta.shape[1] == self.n_total and exc_ptr.shape == (K + 1,)
+            dd = as_np(dec, np.uint8) if (self.dec_len and dec is not None) else None
+            if out is None:
+                st, pk, lt = np.empty(K, np.uint8), np.empty(K, np.int64), np.empty(K, np.float64)
+            else:
+                st, pk, lt = (as_np(o, None) for o in out)
+            _check(self._L.magis_eval_schedules_host_delta8(self._h, K, _np_ptr(delta), _np_ptr(exc_ptr),
+                                                            _np_ptr(exc), _np_ptr(dd), _np_ptr(st), _np_ptr(pk),
+                                                            _np_ptr(lt), _stream_ptr(stream)))
+            return st, pk, lt
         p = as_np(perm, None)
         u16 = p.dtype == np.uint16
         if not u16:
