@@ -39,9 +39,8 @@ namespace magis {
 constexpr uint32_t kKindShift = 29;
 constexpr uint32_t kIdMask = (1u << kKindShift) - 1;
 constexpr uint32_t kHdrOut = 2, kHdrClone = 3, kNop = 7;   // kHdr = 1, kHdrCopy = 4
-constexpr int kBarMain = 1, kBarFull = 2, kBarEmpty = 4;
-constexpr int TM = kMainThreads2;
-constexpr int WM = TM / 32;
+// named barriers of team t: main 1 + 5t, FULL 2 + 5t + slot, EMPTY 4 + 5t + slot
+constexpr int kBarMain = 1, kBarFull = 2, kBarEmpty = 4, kBarTeam = 5;
 
 // -------------------------------------------------------------- packed u16 --
 template <int P> struct Pk;
@@ -107,14 +106,19 @@ template <> struct Pk<4> {
 };
 
 // ------------------------------------------------------------- barriers --
-// immediate barrier ids so ptxas reserves only the 6 barriers used
+// immediate barrier ids so ptxas reserves only the barriers used (5 per team)
 __device__ __forceinline__ void bar_sync(int id, int n) {
     switch (id) {
         case 1: asm volatile("bar.sync 1, %0;" ::"r"(n) : "memory"); break;
         case 2: asm volatile("bar.sync 2, %0;" ::"r"(n) : "memory"); break;
         case 3: asm volatile("bar.sync 3, %0;" ::"r"(n) : "memory"); break;
         case 4: asm volatile("bar.sync 4, %0;" ::"r"(n) : "memory"); break;
-        default: asm volatile("bar.sync 5, %0;" ::"r"(n) : "memory"); break;
+        case 5: asm volatile("bar.sync 5, %0;" ::"r"(n) : "memory"); break;
+        case 6: asm volatile("bar.sync 6, %0;" ::"r"(n) : "memory"); break;
+        case 7: asm volatile("bar.sync 7, %0;" ::"r"(n) : "memory"); break;
+        case 8: asm volatile("bar.sync 8, %0;" ::"r"(n) : "memory"); break;
+        case 9: asm volatile("bar.sync 9, %0;" ::"r"(n) : "memory"); break;
+        default: asm volatile("bar.sync 10, %0;" ::"r"(n) : "memory"); break;
     }
 }
 __device__ __forceinline__ void bar_arrive(int id, int n) {
@@ -122,7 +126,11 @@ __device__ __forceinline__ void bar_arrive(int id, int n) {
         case 2: asm volatile("bar.arrive 2, %0;" ::"r"(n) : "memory"); break;
         case 3: asm volatile("bar.arrive 3, %0;" ::"r"(n) : "memory"); break;
         case 4: asm volatile("bar.arrive 4, %0;" ::"r"(n) : "memory"); break;
-        default: asm volatile("bar.arrive 5, %0;" ::"r"(n) : "memory"); break;
+        case 5: asm volatile("bar.arrive 5, %0;" ::"r"(n) : "memory"); break;
+        case 7: asm volatile("bar.arrive 7, %0;" ::"r"(n) : "memory"); break;
+        case 8: asm volatile("bar.arrive 8, %0;" ::"r"(n) : "memory"); break;
+        case 9: asm volatile("bar.arrive 9, %0;" ::"r"(n) : "memory"); break;
+        default: asm volatile("bar.arrive 10, %0;" ::"r"(n) : "memory"); break;
     }
 }
 
@@ -268,27 +276,44 @@ __device__ __forceinline__ double candidate_latency(unsigned long long* key, dou
 }
 
 // MODE 0: graph tables and step slots in shared memory; 1: tables read from
-// the global image; 2: tables and step slots in global memory (large graphs)
-template <int P, int LMAX, int MODE>
-__global__ void __launch_bounds__(TM + 32 * P, 1)
+// the global image; 2: tables and step slots in global memory (large graphs).
+// TEAMS: independent teams per CTA (each TM main threads + its latency warps,
+// its own per-group state, slots and named barriers; the tables are shared),
+// so one team's barrier waits overlap the other's work.
+template <int P, int LMAX, int MODE, int TEAMS>
+__global__ void __launch_bounds__(TEAMS * (kMainThreads2 / TEAMS + 32 * P), 1)
 eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
              const int32_t* __restrict__ perm, const uint8_t* __restrict__ dec,
              uint8_t* __restrict__ out_status, int64_t* __restrict__ out_peak,
              double* __restrict__ out_lat, char* __restrict__ ovf, char* __restrict__ afg) {
     using PK = Pk<P>;
     using V = typename PK::V;
+    constexpr int TM = kMainThreads2 / TEAMS;  // main threads of a team
+    constexpr int WM = TM / 32;
     constexpr int TL = 32 * P;                 // latency warps: one per candidate of a group
-    extern __shared__ __align__(128) char sm[];
+    extern __shared__ __align__(128) char sm_all[];
     __shared__ uint64_t mbar;
-    __shared__ SlotHdr hdr[2];
-    __shared__ Ctl ctl[2];                     // per group parity (reset one group ahead)
-    __shared__ long long agg_s[2][WM];         // per slot: warp aggregates of the scan,
-    __shared__ long long agg_m[2][WM];         //   folded by the latency warps
-    __shared__ double agg_c[2][WM];
-    __shared__ double lwoff[4][WM];            // per latency warp: cost prefix of each team warp
-    __shared__ int wcnt[WM];                   // event steps per warp chunk
+    __shared__ SlotHdr hdr_t[TEAMS][2];
+    __shared__ Ctl ctl_t[TEAMS][2];            // per group parity (reset one group ahead)
+    __shared__ long long agg_s_t[TEAMS][2][WM];   // per slot: warp aggregates of the scan,
+    __shared__ long long agg_m_t[TEAMS][2][WM];   //   folded by the latency warps
+    __shared__ double agg_c_t[TEAMS][2][WM];
+    __shared__ double lwoff_t[TEAMS][4][WM];   // per latency warp: cost prefix of each team warp
+    __shared__ int wcnt_t[TEAMS][WM];          // event steps per warp chunk
 
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int team = TEAMS == 1 ? 0 : (int)(threadIdx.x / (TM + TL));
+    const int tid = (int)threadIdx.x - team * (TM + TL), lane = tid & 31, warp = tid >> 5;
+    const int bb = kBarTeam * team;            // this team's barrier ids: kBar* + bb
+    const int64_t cta = (int64_t)blockIdx.x * TEAMS + team, ncta_all = (int64_t)gridDim.x * TEAMS;
+    SlotHdr* hdr = hdr_t[team];
+    Ctl* ctl = ctl_t[team];
+    long long (*agg_s)[WM] = agg_s_t[team];
+    long long (*agg_m)[WM] = agg_m_t[team];
+    double (*agg_c)[WM] = agg_c_t[team];
+    double (*lwoff)[WM] = lwoff_t[team];
+    int* wcnt = wcnt_t[team];
+    // this team's state: the static tables (MODE 0) are shared, the state follows at + team * stride
+    char* sm = sm_all + (size_t)team * pl.state_stride;
     const int32_t NT = pl.NT, R = pl.R, n = pl.n;
     // optional phase profile (MAGIS_PROFILE=1): cycles between marks, thread 0
     // of the main warps and lane 0 of the latency warp, summed over CTAs
@@ -302,8 +327,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 
     // graph tables: staged into shared memory once per CTA (bulk copy), or
     // read in place from the global image when they do not fit
-    const char* sb = MODE ? blob : sm;
-    if (MODE == 0) bulk_stage(sm, blob, pl.static_bytes, &mbar);
+    const char* sb = MODE ? blob : sm_all;
+    if (MODE == 0) bulk_stage(sm_all, blob, pl.static_bytes, &mbar);
     const uint32_t* wtab = (const uint32_t*)(sb + pl.off_wtab);   // [WM][4]: consumer rows, input rows
     const uint2* crow = (const uint2*)(sb + pl.off_crow);
     const uint32_t* chdr = (const uint32_t*)(sb + pl.off_chdr);
@@ -321,7 +346,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const uint16_t* utr = (const uint16_t*)(sb + pl.off_utr);       // [R] t_r
     uint16_t* pos = (uint16_t*)(sm + pl.off_pos);
     uint16_t* last = (uint16_t*)(sm + pl.off_last);
-    uint2* AF = MODE == 2 ? (uint2*)(afg + (size_t)blockIdx.x * pl.af_bytes)   // [P][Sl] (alloc, free)
+    uint2* AF = MODE == 2 ? (uint2*)(afg + (size_t)cta * pl.af_bytes)         // [P][Sl] (alloc, free)
                           : (uint2*)(sm + pl.off_af);                           // size units per step
     uint8_t* dec_s = (uint8_t*)(sm + pl.off_dec);
     uint32_t* evm = (uint32_t*)(sm + pl.off_evm);          // [P][nwm] event-step marks
@@ -333,8 +358,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     unsigned long long* evi_s = (unsigned long long*)(sm + pl.off_ev + (size_t)2 * P * cap * 16);   // [2][P][cap]
 
     // pos / last of the virtual and dummy slots start (and the dummy stays) 0
-    for (int i = tid; i < pl.NTX * P; i += blockDim.x) { pos[i] = 0; last[i] = 0; }
-    for (int i = tid; i < P * nwm; i += blockDim.x) evm[i] = 0;
+    for (int i = tid; i < pl.NTX * P; i += TM + TL) { pos[i] = 0; last[i] = 0; }
+    for (int i = tid; i < P * nwm; i += TM + TL) evm[i] = 0;
     if (tid == 0) {
         for (int b = 0; b < 2; b++) {
             for (int c = 0; c < 4; c++) ctl[b].flags[c] = ctl[b].viol[c] = 0;
@@ -344,7 +369,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     __syncthreads();
 
     const int64_t ngroups = (K + P - 1) / P;
-    const int ncta = (blockIdx.x < ngroups) ? (int)((ngroups - 1 - blockIdx.x) / gridDim.x + 1) : 0;
+    const int ncta = (cta < ngroups) ? (int)((ngroups - 1 - cta) / ncta_all + 1) : 0;
     constexpr int TPC = TM / P, WT = WM / P;
 
     if (warp >= WM) {
@@ -356,7 +381,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         for (int gi = 0; gi < ncta; gi++) {
             const int slot = gi & 1;
             PROF_MARK(13);
-            bar_sync(kBarFull + slot, TM + TL);
+            bar_sync(kBarFull + slot + bb, TM + TL);
             PROF_MARK(14);
             const SlotHdr& h = hdr[slot];
             const long long k = h.k[c];
@@ -402,7 +427,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         lat = candidate_latency(evk_s + b0, evc_s + b0, evi_s + b0, ne, woff, dd, endb, wt, ctot,
                                                 lane);
                     } else {
-                        char* ob = ovf + ((size_t)blockIdx.x * 8 + slot * 4 + c) * pl.ovf_stride;
+                        char* ob = ovf + ((size_t)cta * 8 + slot * 4 + c) * pl.ovf_stride;
                         const size_t me = (size_t)pl.max_events;
                         lat = candidate_latency((unsigned long long*)ob, (double*)(ob + me * 8),
                                                 (unsigned long long*)(ob + me * 16), ne, woff, dd, endb, wt, ctot,
@@ -417,7 +442,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             }
             __syncwarp();
             PROF_MARK(15);
-            if (gi + 2 < ncta) bar_arrive(kBarEmpty + slot, TM + TL);
+            if (gi + 2 < ncta) bar_arrive(kBarEmpty + slot + bb, TM + TL);
         }
         if (prof)
 #pragma unroll
@@ -460,10 +485,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
     };
     if constexpr (LMAX <= kRegL) {
-        if (ncta > 0) load_chunk(blockIdx.x);
+        if (ncta > 0) load_chunk(cta);
     }
     for (int gi = 0; gi < ncta; gi++) {
-        const int64_t grp = blockIdx.x + (int64_t)gi * gridDim.x;
+        const int64_t grp = cta + (int64_t)gi * ncta_all;
         const int slot = gi & 1;
         Ctl& cl = ctl[slot];
         // candidate c of this group exists iff bit c of vmask is set
@@ -539,7 +564,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             for (int c = 0; c < 4; c++) { cn.flags[c] = 0; cn.viol[c] = 0; }
             cn.swm = 0;
         }
-        bar_sync(kBarMain, TM);
+        bar_sync(kBarMain + bb, TM);
         PROF_MARK(1);
         // ---- phase 2: optional nodes, virtual late-user slots, swap-event
         //      steps (producer, Store, Load and late users of swapped tensors)
@@ -578,7 +603,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 if (d == 2 && pb) atomicOr(em + ((pb - 1) >> 5), 1u << ((pb - 1) & 31));
             }
         }
-        bar_sync(kBarMain, TM);
+        bar_sync(kBarMain + bb, TM);
         PROF_MARK(2);
         // ---- phase 3: validity + last use over the consumer rows -----------------
         {
@@ -617,7 +642,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 if (viol & (1 << c)) atomicOr(&cl.viol[c], MAGIS_ST_EDGE);
             }
         }
-        bar_sync(kBarMain, TM);
+        bar_sync(kBarMain + bb, TM);
         PROF_MARK(3);
         // per-candidate status, 4 bits each; okm: valid candidates with status 0
         uint32_t stm = 0, okm = 0;
@@ -689,8 +714,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         // the slot of this group parity is free once the latency warp is done
         // with group gi - 2
         PROF_MARK(9);
-        if (gi >= 2) bar_sync(kBarEmpty + slot, TM + TL);
-        else bar_sync(kBarMain, TM);
+        if (gi >= 2) bar_sync(kBarEmpty + slot + bb, TM + TL);
+        else bar_sync(kBarMain + bb, TM);
         PROF_MARK(4);
         SlotHdr& h = hdr[slot];
         // event list of candidate cm: shared-memory slot, or global overflow
@@ -707,7 +732,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             kout = evk_s + (size_t)(slot * P + cm) * cap;
             cout_ = evc_s + (size_t)(slot * P + cm) * cap;
         } else {
-            char* ob = ovf + ((size_t)blockIdx.x * 8 + slot * 4 + cm) * pl.ovf_stride;
+            char* ob = ovf + ((size_t)cta * 8 + slot * 4 + cm) * pl.ovf_stride;
             kout = (unsigned long long*)ob;
             cout_ = (double*)(ob + (size_t)pl.max_events * 8);
         }
@@ -759,9 +784,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         // the next group's chunk is loaded while this group finishes
         if constexpr (LMAX <= kRegL) {
-            if (gi + 1 < ncta) load_chunk(grp + gridDim.x);
+            if (gi + 1 < ncta) load_chunk(grp + ncta_all);
         }
-        bar_sync(kBarMain, TM);
+        bar_sync(kBarMain + bb, TM);
         PROF_MARK(5);
         // ---- phase 6: hand-off to the latency warps (they fold the aggregates) ----
         if (tid < P) {
@@ -792,7 +817,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         // bar.arrive orders this thread's prior shared / global writes for the
         // threads that sync on the barrier (no membar: it would also wait for
         // the next group's perm loads already in flight)
-        bar_arrive(kBarFull + slot, TM + TL);
+        bar_arrive(kBarFull + slot + bb, TM + TL);
         PROF_MARK(6);
         // clear pos and the event marks for the next group
         {
@@ -802,7 +827,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             for (int i = ((nb >> 4) << 3) + tid; i < NT * P; i += TM) pos[i] = 0;
             for (int i = tid; i < P * nwm; i += TM) evm[i] = 0;
         }
-        bar_sync(kBarMain, TM);
+        bar_sync(kBarMain + bb, TM);
         PROF_MARK(7);
     }
     if (prof)
@@ -810,32 +835,37 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         for (int i = 1; i < 13; i++) atomicAdd((unsigned long long*)(ovf + pl.prof_off) + i, pt[i]);
 }
 
-template <int P, int MODE>
+template <int P, int MODE, int TEAMS>
 static const void* kernel_ptr(int lmax) {
     if constexpr (MODE == 0) {
-        if (lmax <= 4) return (const void*)eval2_kernel<P, 4, 0>;
-        if (lmax <= 8) return (const void*)eval2_kernel<P, 8, 0>;
-        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, 0>;
-        return (const void*)eval2_kernel<P, 32, 0>;
+        if (lmax <= 4) return (const void*)eval2_kernel<P, 4, 0, TEAMS>;
+        if (lmax <= 8) return (const void*)eval2_kernel<P, 8, 0, TEAMS>;
+        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, 0, TEAMS>;
+        return (const void*)eval2_kernel<P, 32, 0, TEAMS>;
     } else {
-        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, MODE>;
-        if (lmax <= 32) return (const void*)eval2_kernel<P, 32, MODE>;
-        return (const void*)eval2_kernel<P, 64, MODE>;
+        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, MODE, 1>;
+        if (lmax <= 32) return (const void*)eval2_kernel<P, 32, MODE, 1>;
+        return (const void*)eval2_kernel<P, 64, MODE, 1>;
     }
 }
 
-template <int MODE>
+template <int MODE, int TEAMS>
 static const void* kernel_mode(const Plan2& pl) {
-    return pl.P == 4 ? kernel_ptr<4, MODE>(pl.L) : pl.P == 2 ? kernel_ptr<2, MODE>(pl.L) : kernel_ptr<1, MODE>(pl.L);
+    return pl.P == 4 ? kernel_ptr<4, MODE, TEAMS>(pl.L)
+                     : pl.P == 2 ? kernel_ptr<2, MODE, TEAMS>(pl.L) : kernel_ptr<1, MODE, TEAMS>(pl.L);
 }
 
 static const void* kernel_for(const Plan2& pl) {
     const int mode = pl.gmem_af ? 2 : (pl.gmem_static ? 1 : 0);
-    return mode == 0 ? kernel_mode<0>(pl) : mode == 1 ? kernel_mode<1>(pl) : kernel_mode<2>(pl);
+    if (mode == 0) return pl.teams == 2 ? kernel_mode<0, 2>(pl) : kernel_mode<0, 1>(pl);
+    return mode == 1 ? kernel_mode<1, 1>(pl) : kernel_mode<2, 1>(pl);
 }
+
+int eval2_block(const Plan2& pl) { return kMainThreads2 + pl.teams * 32 * pl.P; }
 
 cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
     if (pl.L > 64 || (!pl.gmem_static && pl.L > 32)) { *blocks = 0; return cudaSuccess; }
+    if (pl.teams == 2 && pl.gmem_static) { *blocks = 0; return cudaSuccess; }   // teams only with smem tables
     const void* fn = kernel_for(pl);
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_total);
     if (e != cudaSuccess) return e;
@@ -844,10 +874,10 @@ cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
     if (std::getenv("MAGIS_DEBUG")) {
         cudaFuncAttributes fa;
         cudaFuncGetAttributes(&fa, fn);
-        std::fprintf(stderr, "[magis] eval2 P=%d regs=%d static_smem=%zu local=%zu\n", pl.P, fa.numRegs,
-                     fa.sharedSizeBytes, fa.localSizeBytes);
+        std::fprintf(stderr, "[magis] eval2 P=%d teams=%d regs=%d static_smem=%zu local=%zu\n", pl.P, pl.teams,
+                     fa.numRegs, fa.sharedSizeBytes, fa.localSizeBytes);
     }
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, TM + 32 * pl.P, pl.smem_total);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, fn, eval2_block(pl), pl.smem_total);
 }
 
 cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,
@@ -855,10 +885,10 @@ cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, v
                          int64_t* peak, double* lat, cudaStream_t stream) {
     if (K <= 0) return cudaSuccess;
     const int64_t ngroups = (K + pl.P - 1) / pl.P;
-    const int gr = (int)std::min<int64_t>(grid, ngroups);
+    const int gr = (int)std::min<int64_t>(grid, (ngroups + pl.teams - 1) / pl.teams);
     void* args[] = {(void*)&g, (void*)&pl, (void*)&blob, (void*)&K, (void*)&perm, (void*)&dec,
                     (void*)&status, (void*)&peak, (void*)&lat, (void*)&ovf, (void*)&afg};
-    return cudaLaunchKernel(kernel_for(pl), dim3(gr), dim3(TM + 32 * pl.P), args, pl.smem_total, stream);
+    return cudaLaunchKernel(kernel_for(pl), dim3(gr), dim3(eval2_block(pl)), args, pl.smem_total, stream);
 }
 
 }  // namespace magis

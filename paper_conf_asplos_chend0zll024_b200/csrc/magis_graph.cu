@@ -465,29 +465,41 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
             // (P x resident CTAs; ties go to more CTAs, which hide barriers).
             // Tiers, in order: graph tables and step slots in shared memory;
             // tables read from global (L2); tables and slots in global.
+            // Teams (two independent warp groups per CTA sharing the tables)
+            // count as extra resident groups: candidates in flight = P x teams
+            // x CTAs; ties prefer more independent groups (CTAs x teams),
+            // whose barrier waits overlap each other's work.
             const int cands[3] = {4, 2, 1};
-            int bestP = 0, bestOcc = 0;
+            const char* tforce = std::getenv("MAGIS_TEAMS");
+            int bestP = 0, bestOcc = 0, bestT = 1;
             Plan2 bestPl{};
             std::vector<char> bestImg;
             for (int tier = 0; tier < 3 && bestP == 0; tier++) {
                 const bool gs = tier >= 1, ga = tier >= 2;
-                for (int ci = 0; ci < 3; ci++) {
-                    const int P = cands[ci];
-                    if (pforce && std::atoi(pforce) != P) continue;
-                    Plan2 pl;
-                    std::vector<char> img;
-                    if (!plan2_build(sg, P, gs, ga, cap, &pl, &img)) continue;
-                    int occ = 0;
-                    cudaError_t oe = eval2_occupancy(pl, &occ);
-                    if (std::getenv("MAGIS_DEBUG"))
-                        std::fprintf(stderr, "[magis] plan tier=%d P=%d L=%d S=%d smem=%u static=%u occ=%d err=%d\n",
-                                     tier, P, pl.L, pl.S, pl.smem_total, pl.static_bytes, occ, (int)oe);
-                    if (oe != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
-                    if (P * occ > bestP * bestOcc || (P * occ == bestP * bestOcc && occ > bestOcc)) {
-                        bestP = P;
-                        bestOcc = occ;
-                        bestPl = pl;
-                        bestImg.swap(img);
+                for (int T = 2; T >= 1; T--) {
+                    if (tforce && std::atoi(tforce) != T) continue;
+                    if (T == 2 && gs) continue;                     // teams only with the tables in smem
+                    for (int ci = 0; ci < 3; ci++) {
+                        const int P = cands[ci];
+                        if (pforce && std::atoi(pforce) != P) continue;
+                        Plan2 pl;
+                        std::vector<char> img;
+                        if (!plan2_build(sg, P, T, gs, ga, cap, &pl, &img)) continue;
+                        int occ = 0;
+                        cudaError_t oe = eval2_occupancy(pl, &occ);
+                        if (std::getenv("MAGIS_DEBUG"))
+                            std::fprintf(stderr,
+                                         "[magis] plan tier=%d teams=%d P=%d L=%d S=%d smem=%u static=%u occ=%d err=%d\n",
+                                         tier, T, P, pl.L, pl.S, pl.smem_total, pl.static_bytes, occ, (int)oe);
+                        if (oe != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
+                        const int a = P * T * occ, b = bestP * bestT * bestOcc;
+                        if (a > b || (a == b && T * occ > bestT * bestOcc)) {
+                            bestP = P;
+                            bestT = T;
+                            bestOcc = occ;
+                            bestPl = pl;
+                            bestImg.swap(img);
+                        }
                     }
                 }
             }
@@ -498,11 +510,11 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
                 bool ok = cudaMalloc(&b2, bestImg.size()) == cudaSuccess;
                 ok = ok && cudaMemcpy(b2, bestImg.data(), bestImg.size(), cudaMemcpyHostToDevice) == cudaSuccess;
                 bestPl.prof = std::getenv("MAGIS_PROFILE") ? 1 : 0;
-                bestPl.prof_off = (uint64_t)grid * 8 * bestPl.ovf_stride;
+                bestPl.prof_off = (uint64_t)grid * bestT * 8 * bestPl.ovf_stride;   // 8 regions per team
                 ok = ok && cudaMalloc(&ov, bestPl.prof_off + 256) == cudaSuccess;
                 ok = ok && cudaMemset(ov, 0, bestPl.prof_off + 256) == cudaSuccess;
                 void* ag = nullptr;
-                if (ok && bestPl.gmem_af) ok = cudaMalloc(&ag, (size_t)grid * bestPl.af_bytes) == cudaSuccess;
+                if (ok && bestPl.gmem_af) ok = cudaMalloc(&ag, (size_t)grid * bestT * bestPl.af_bytes) == cudaSuccess;
                 g->afg2 = ag;
                 if (ok) {
                     g->plan2 = bestPl;
@@ -511,7 +523,7 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
                     g->ovf2 = ov;
                     g->cfg.variant = 2;
                     g->cfg.grid = grid;
-                    g->cfg.block = kMainThreads2 + 32 * bestPl.P;
+                    g->cfg.block = eval2_block(bestPl);
                     g->cfg.smem = bestPl.smem_total;
                 } else {
                     cudaGetLastError();

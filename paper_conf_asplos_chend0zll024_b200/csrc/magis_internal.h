@@ -103,6 +103,8 @@ struct Plan2 {
     uint64_t af_bytes;
     int32_t prof;         // MAGIS_PROFILE: accumulate per-phase cycles
     uint64_t prof_off;    // byte offset of the 16 u64 phase counters in the scratch buffer
+    int32_t teams;        // independent teams per CTA (1 or 2), each with its own per-group state and barriers
+    uint32_t state_stride;   // bytes of shared memory per team's state (team t at + t * state_stride)
 };
 
 // Base-graph adjacency for the device candidate generator (magis_gen.cu).
@@ -190,12 +192,13 @@ struct SuperGraphHost {
 // Build the variant-2 plan and its static shared-memory image for a given P.
 // Returns false if the graph does not fit (ids >= 65535, sizes beyond u32
 // units, or shared memory).
-bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af, size_t smem_cap, Plan2* plan,
+bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, size_t smem_cap, Plan2* plan,
                  std::vector<char>* image);
 cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,
                          int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status,
                          int64_t* peak, double* lat, cudaStream_t stream);
 cudaError_t eval2_occupancy(const Plan2& pl, int* blocks_per_sm);
+int eval2_block(const Plan2& pl);      // threads per CTA
 
 size_t hotspot_ws_per_cta(const DevGraph& g);
 cudaError_t hotspot_launch(const DevGraph& g, int grid, void* ws, int64_t K, const int32_t* perm, const uint8_t* dec,

@@ -96,8 +96,8 @@ Rows make_rows(const std::vector<std::vector<uint32_t>>& lists, const std::vecto
 }
 }  // namespace
 
-bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af, size_t smem_cap, Plan2* pl,
-                 std::vector<char>* img) {
+bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, size_t smem_cap,
+                 Plan2* pl, std::vector<char>* img) {
     const int32_t NT = sg.NT, n = sg.n, R = sg.R;
     const int32_t nU = R > 0 ? sg.U_ptr[R] : 0;
     const int64_t NTX = (int64_t)NT + nU + 1;
@@ -135,7 +135,12 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
         for (int32_t e = sg.in_ptr[u]; e < sg.in_ptr[u + 1]; e++)
             ins[u].push_back((kEdge << kKindShift) | (uint32_t)sg.in_ent[e].x);
     }
-    const int WM = kMainThreads2 / 32;
+    // teams: independent groups of warps in one CTA, each scoring its own
+    // candidates with its own per-group state and barriers (the graph tables
+    // are shared); main threads per team = kMainThreads2 / teams
+    if (teams != 1 && teams != 2) return false;
+    const int TMt = kMainThreads2 / teams;
+    const int WM = TMt / 32;
     const uint32_t dummy = (uint32_t)(NTX - 1);
     const uint16_t nop = (uint16_t)dummy;
     const uint32_t nophdr = (kNop << kKindShift) | dummy;
@@ -163,7 +168,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
     p.R = R;
     p.nU = nU;
     {
-        const int32_t tpc = kMainThreads2 / P;          // threads per candidate in the scan
+        const int32_t tpc = TMt / P;                    // threads per candidate in the scan
         int32_t Lmin = std::max(4, (NT + tpc - 1) / tpc), lg = 0;
         while ((1 << lg) < Lmin) lg++;
         if (lg > 6) return false;                       // LMAX <= 64 steps per thread
@@ -210,9 +215,15 @@ bool plan2_build(const SuperGraphHost& sg, int P, bool gmem_static, bool gmem_af
     p.off_ev = (uint32_t)o;
     // event steps of a candidate: at most the marked steps (<= 3R + |U|)
     int cap = std::min(std::max(p.max_events, 1), 128);
+    p.teams = teams;
     while (true) {
-        const size_t need = o + (size_t)2 * P * cap * 24;
-        if (need <= smem_cap) { p.smem_total = (uint32_t)a16(need); break; }
+        const size_t st = a16(o + (size_t)2 * P * cap * 24) - p.state_base;     // one team's state
+        const size_t need = p.state_base + (size_t)teams * st;
+        if (need <= smem_cap) {
+            p.smem_total = (uint32_t)a16(need);
+            p.state_stride = (uint32_t)st;
+            break;
+        }
         if (cap <= 8) return false;
         cap /= 2;
     }

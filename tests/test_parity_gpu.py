@@ -25,13 +25,14 @@ DEV = "cuda:0"
 
 # kernel variants: magis_eval.cu (v1, global state) and magis_eval2.cu with
 # P = 1 / 2 / 4 packed candidates; "auto" is what the loader picks.
-VARIANTS = {"auto": {}, "v1": {"MAGIS_VARIANT": "1"}, "p1": {"MAGIS_P": "1"},
-            "p2": {"MAGIS_P": "2"}, "p4": {"MAGIS_P": "4"}}
+VARIANTS = {"auto": {}, "v1": {"MAGIS_VARIANT": "1"}, "p1": {"MAGIS_P": "1", "MAGIS_TEAMS": "1"},
+            "p2": {"MAGIS_P": "2", "MAGIS_TEAMS": "1"}, "p4": {"MAGIS_P": "4", "MAGIS_TEAMS": "1"},
+            "t2p1": {"MAGIS_P": "1", "MAGIS_TEAMS": "2"}, "t2p2": {"MAGIS_P": "2", "MAGIS_TEAMS": "2"}}
 
 
 @pytest.fixture(params=list(VARIANTS))
 def variant(request, monkeypatch):
-    for k in ("MAGIS_VARIANT", "MAGIS_P"):
+    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS"):
         monkeypatch.delenv(k, raising=False)
     for k, v in VARIANTS[request.param].items():
         monkeypatch.setenv(k, v)
