@@ -467,8 +467,9 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
             // tables read from global (L2); tables and slots in global.
             // Teams (two independent warp groups per CTA sharing the tables)
             // count as extra resident groups: candidates in flight = P x teams
-            // x CTAs; ties prefer more independent groups (CTAs x teams),
-            // whose barrier waits overlap each other's work.
+            // x CTAs; ties prefer one team with the wider packing (measured on
+            // C2 / C5: 1 team x P=4 beats 2 teams x P=2 by 16-19%, the packed
+            // u16x4 work outweighs the overlapped barrier waits).
             const int cands[3] = {4, 2, 1};
             const char* tforce = std::getenv("MAGIS_TEAMS");
             int bestP = 0, bestOcc = 0, bestT = 1;
@@ -493,7 +494,7 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
                                          tier, T, P, pl.L, pl.S, pl.smem_total, pl.static_bytes, occ, (int)oe);
                         if (oe != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
                         const int a = P * T * occ, b = bestP * bestT * bestOcc;
-                        if (a > b || (a == b && T * occ > bestT * bestOcc)) {
+                        if (a > b || (a == b && (T < bestT || (T == bestT && occ > bestOcc)))) {
                             bestP = P;
                             bestT = T;
                             bestOcc = occ;
