@@ -454,6 +454,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // phases 1 and 5: candidate cm of the group is handled by team cm (TPC
     // threads, WT warps); thread tt of the team owns steps [lo, lo + L)
     const int cm = tid / TPC, tt = tid - cm * TPC;
+    // (candidate, tensor) of this thread's first item in the P x R loops and the
+    // per-iteration step (TM / R, TM % R): no division inside the group loop
+    const int c_0 = R > 0 ? tid / R : 0, r_0 = tid - c_0 * R, dc_ = R > 0 ? TM / R : 0, dr_ = TM - dc_ * R;
     const int32_t lo = tt * L;
     const bool vec4 = (NT & 3) == 0;
     // perm chunk kept in registers when short (32 steps only where the
@@ -497,8 +500,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         // ---- phase 0: decisions ---------------------------------------------
         {
             uint32_t badm = 0, swm = 0;
-            for (int i = tid; i < P * R; i += TM) {
-                const int c = i / R, r = i - c * R;
+            for (int i = tid, c = c_0, r = r_0; i < P * R; i += TM, c += dc_, r += dr_) {
+                if (r >= R) { r -= R; c++; }
                 const uint8_t d = ((vmask >> c) & 1u) ? dec[(grp * P + c) * (int64_t)R + r] : 0;
                 dec_s[i] = d;
                 if (d == 2) swm |= 1u << c;
@@ -568,8 +571,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         PROF_MARK(1);
         // ---- phase 2: optional nodes, virtual late-user slots, swap-event
         //      steps (producer, Store, Load and late users of swapped tensors)
-        for (int q = tid; q < P * R; q += TM) {
-            const int c = q / R, r = q - c * R;
+        for (int q = tid, c = c_0, r = r_0; q < P * R; q += TM, c += dc_, r += dr_) {
+            if (r >= R) { r -= R; c++; }
             if (!((vmask >> c) & 1u)) continue;
             const uint32_t ur = urow[r];                       // (U offset, |U_r|) packed
             const uint32_t u0 = ur & 0xffffu, u1 = u0 + (ur >> 16);
