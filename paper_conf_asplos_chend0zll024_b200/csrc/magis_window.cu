@@ -31,10 +31,6 @@ __device__ __forceinline__ bool gate_ok(int32_t gate, const uint8_t* dec) {
     return gate < 0 || dec[gate >> 2] == (uint8_t)(gate & 3);
 }
 
-__device__ __forceinline__ bool node_active(const DevGraph& g, int32_t v, const uint8_t* dec) {
-    return gate_ok(g.ngate[v], dec);
-}
-
 // ---------------------------------------------------------------- base ----
 // One block: pos / active / last in parallel, then thread 0 walks the steps.
 __global__ void base_kernel(DevGraph g, BaseDev b, const int32_t* __restrict__ perm, const uint8_t* __restrict__ dec) {
@@ -182,7 +178,7 @@ window_kernel(DevGraph g, BaseDev b, int64_t K, const int32_t* __restrict__ wsta
     __shared__ WarpScratch wsm[kWarpsW];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     WarpScratch& W = wsm[wid];
-    const int32_t NT = g.NT, n = g.n;
+    const int32_t NT = g.NT;
     const int64_t gw = (int64_t)blockIdx.x * kWarpsW + wid, nw = (int64_t)gridDim.x * kWarpsW;
     const uint8_t* dec = b.dec;
     for (int64_t k = gw; k < K; k += nw) {
