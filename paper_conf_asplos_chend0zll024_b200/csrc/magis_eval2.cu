@@ -291,6 +291,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     constexpr int TM = kMainThreads2 / TEAMS;  // main threads of a team
     constexpr int WM = TM / 32;
     constexpr int TL = 32 * P;                 // latency warps: one per candidate of a group
+    // per-step slots in shared memory: phase 3 scatters alloc / free into them
+    // (smem atomics); in global memory (MODE 2) phase 4 gathers the frees instead
+    constexpr bool kScatter = MODE != 2;
     extern __shared__ __align__(128) char sm_all[];
     __shared__ uint64_t mbar;
     __shared__ SlotHdr hdr_t[TEAMS][2];
@@ -360,6 +363,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // pos / last of the virtual and dummy slots start (and the dummy stays) 0
     for (int i = tid; i < pl.NTX * P; i += TM + TL) { pos[i] = 0; last[i] = 0; }
     for (int i = tid; i < P * nwm; i += TM + TL) evm[i] = 0;
+    if constexpr (kScatter) {
+        uint4* af4 = reinterpret_cast<uint4*>(AF);
+        for (int i = tid; i < P * Sl / 2; i += TM + TL) af4[i] = make_uint4(0u, 0u, 0u, 0u);
+    }
     if (tid == 0) {
         for (int b = 0; b < 2; b++) {
             for (int c = 0; c < 4; c++) ctl[b].flags[c] = ctl[b].viol[c] = 0;
@@ -632,11 +639,30 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         if (kind < kHdrClone && pc == 0) nperm |= 1 << c;
                         if (PK::get(mn, c) < pc) viol |= 1 << c;
                     }
-                    V outv;
-                    if (kind == kHdrOut) outv = PK::splat((uint32_t)NT);
-                    else if (kind >= kHdrClone) outv = PK::vand(lst, PK::nzmask(p));   // inactive halves -> 0
-                    else outv = lst;
-                    PK::store(last, id, outv);
+                    if constexpr (kScatter) {
+                        // alloc at the own step, free after the last reader's step
+                        // (a tensor without readers after its own step; graph
+                        // outputs live to the end): scattered straight into the
+                        // per-step slots, no second pass over the input rows
+                        const uint32_t A = size_s[id];
+#pragma unroll
+                        for (int c = 0; c < P; c++) {
+                            const uint32_t pc = PK::get(p, c);
+                            if (pc == 0) continue;                  // absent (inactive) in candidate c
+                            const uint32_t st = pc - 1;
+                            AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)].x = A;
+                            if (kind != kHdrOut && A != 0) {
+                                const uint32_t fs = PK::get(lst, c) - 1;
+                                atomicAdd(&AF[c * Sl + (fs & (L - 1)) * S + (fs >> lgL)].y, A);
+                            }
+                        }
+                    } else {
+                        V outv;
+                        if (kind == kHdrOut) outv = PK::splat((uint32_t)NT);
+                        else if (kind >= kHdrClone) outv = PK::vand(lst, PK::nzmask(p));   // inactive halves -> 0
+                        else outv = lst;
+                        PK::store(last, id, outv);
+                    }
                 }
             }
 #pragma unroll
@@ -673,8 +699,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             if (lane == 31) wcnt[warp] = inc;
             evx = inc - evx;
         }
-        if (okm != 0) {
-            // ---- phase 4: frees over the input rows -> per-step slots ------------
+        if (!kScatter && okm != 0) {
+            // ---- phase 4 (slots in global memory): frees over the input rows ------
             const uint32_t r0 = wtab[warp * 4 + 2], r1 = wtab[warp * 4 + 3];
             for (uint32_t r = r0; r < r1; r++) {
                 const uint2 rw = frow[r];
@@ -829,6 +855,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             for (int i = tid; i < (nb >> 4); i += TM) p4[i] = make_uint4(0u, 0u, 0u, 0u);
             for (int i = ((nb >> 4) << 3) + tid; i < NT * P; i += TM) pos[i] = 0;
             for (int i = tid; i < P * nwm; i += TM) evm[i] = 0;
+            if constexpr (kScatter) {           // the per-step slots start from 0 for the scatter
+                uint4* af4 = reinterpret_cast<uint4*>(AF);
+                for (int i = tid; i < P * Sl / 2; i += TM) af4[i] = make_uint4(0u, 0u, 0u, 0u);
+            }
         }
         bar_sync(kBarMain + bb, TM);
         PROF_MARK(7);
