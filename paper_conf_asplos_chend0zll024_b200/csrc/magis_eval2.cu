@@ -193,11 +193,6 @@ __device__ __forceinline__ unsigned long long mark_bits(const uint32_t* m, int32
     return L == 32 ? w : (w & ((1u << L) - 1u));
 }
 
-// The three in-order queues of reading P7 over one candidate's event steps
-// (in step order): at a compute op, stalls on the Loads of the swapped
-// tensors it reads, then the end of the op if it produces a swapped tensor;
-// Store / Load ops on the D2H / H2D queues.  endb[3r + 0 / 1 / 2] = end of
-// producer / Store / Load of tensor r.
 struct WalkTabs {
     const uint2* ninfo;
     const uint16_t* lul;
@@ -205,71 +200,101 @@ struct WalkTabs {
     int32_t n, lgL;
 };
 
-// What a compute step of a swapping candidate does on the queues, resolved
-// by the main warp that emits it: bits 0-30 = which of the node's late-user
-// tensors (ninfo list order) are swapped, bit 31 = it produces a swapped
-// tensor, bits 32-47 = that tensor, bits 48-63 = offset of the list in lul.
-__device__ __forceinline__ unsigned long long step_info(int32_t v, int32_t n, const uint8_t* dd, const uint2* ninfo,
-                                                        const uint16_t* lul) {
-    if (v >= n) return 0ull;
-    const uint2 x = ninfo[v];
-    const uint32_t rt = x.x & 0xffffu, cnt = x.x >> 16;
-    uint32_t m = 0;
-    for (uint32_t i = 0; i < cnt; i++) m |= (uint32_t)(dd[lul[x.y + i]] == 2) << i;
-    const bool prod = rt && dd[rt - 1] == 2;
-    return (unsigned long long)m | ((unsigned long long)prod << 31) |
-           ((unsigned long long)(prod ? rt - 1 : 0) << 32) | ((unsigned long long)x.y << 48);
+// The event steps of a swapping candidate are resolved by the whole latency
+// warp (one lane per event) into compact records, so the serial walk (lane 0)
+// only chases the queue recurrences:
+//   ia (u64): bits 62-63 kind (0 compute, 1 Store, 2 Load); compute: bits
+//             48-52 number of swapped tensors the op reads (late-user
+//             stalls), bits 0-47 the first three of them (16 bits each)
+//   ib (u64): Store / Load: r; compute: bits 0-15 r + 1 of the swapped tensor
+//             it produces (0 none), bits 16-46 the swapped mask over the node's
+//             late-user list, bits 47-62 the list's offset in lul (used only
+//             with more than three stalls)
+//   x (f64):  compute: compute-cost prefix before the step; Store / Load:
+//             the transfer time lambda + |t_r| / B
+__device__ __forceinline__ void resolve_event(unsigned long long& kslot, double& cslot, unsigned long long& islot,
+                                              const double* woff, const uint8_t* dd, const WalkTabs& t) {
+    const unsigned long long kk = kslot;
+    const int32_t stp = (int32_t)(kk >> 32), w = (int32_t)(kk & 0xffffffffu);
+    if (w < t.n) {
+        const uint2 x = t.ninfo[w];
+        const uint32_t rt = x.x & 0xffffu, cnt = x.x >> 16;
+        uint32_t m = 0, nw = 0;
+        unsigned long long pk = 0;
+        for (uint32_t i = 0; i < cnt; i++) {
+            const uint32_t r = t.lul[x.y + i];
+            if (dd[r] == 2) {
+                m |= 1u << i;
+                if (nw < 3) pk |= (unsigned long long)r << (16 * nw);
+                nw++;
+            }
+        }
+        const bool prod = rt && dd[rt - 1] == 2;
+        islot = pk | ((unsigned long long)nw << 48);
+        kslot = (unsigned long long)(prod ? rt : 0u) | ((unsigned long long)m << 16) |
+                ((unsigned long long)x.y << 47);
+        cslot += woff[(stp >> t.lgL) >> 5];
+    } else {
+        const uint32_t q = (uint32_t)(w - t.n), r = q / 3, o = q - 3 * r;   // o: 1 Store, 2 Load
+        islot = (unsigned long long)o << 62;
+        kslot = r;
+        cslot = t.rtab[r].y;
+    }
 }
 
-__device__ __forceinline__ void walk_events(const unsigned long long* key, const double* cbp,
-                                            const unsigned long long* info, int ne,
-                                            double* endb, const WalkTabs& t, double& D, double& Td, double& Th) {
-    unsigned long long kn = ne > 0 ? key[0] : 0ull, in_ = ne > 0 ? info[0] : 0ull;
-    double cn = ne > 0 ? cbp[0] : 0.0;
+// The three in-order queues of reading P7 over the resolved records (step
+// order): a compute op first stalls on the Loads of the swapped tensors it
+// reads, then ends (if it produces a swapped tensor); Store / Load ops run on
+// the D2H / H2D queues.  endb[3r + 0 / 1 / 2] = end of producer / Store /
+// Load of tensor r.
+__device__ __forceinline__ void walk_events(const unsigned long long* ia, const unsigned long long* ib,
+                                            const double* xs, int ne, double* endb, const WalkTabs& t,
+                                            double& D, double& Td, double& Th) {
+    unsigned long long an = ne > 0 ? ia[0] : 0ull, bn = ne > 0 ? ib[0] : 0ull;
+    double xn = ne > 0 ? xs[0] : 0.0;
     for (int e = 0; e < ne; e++) {
-        const unsigned long long kk = kn, inf = in_;
-        const double cp = cn;
-        if (e + 1 < ne) { kn = key[e + 1]; cn = cbp[e + 1]; in_ = info[e + 1]; }   // next event step in flight
-        const int32_t w = (int32_t)(kk & 0xffffffffu);
-        const double cw = cp;                                         // compute-cost prefix before the step
-        if (w < t.n) {
-            uint32_t m = (uint32_t)inf & 0x7fffffffu;
-            const uint32_t off = (uint32_t)(inf >> 48);
-            while (m) {                                               // stalls on the Loads it reads
-                const uint32_t i = __ffs(m) - 1;
-                m &= m - 1;
-                const uint32_t r = t.lul[off + i];
-                D = fmax(D, endb[3 * r + 2] - cw);
+        const unsigned long long a = an, b = bn;
+        const double x = xn;
+        if (e + 1 < ne) { an = ia[e + 1]; bn = ib[e + 1]; xn = xs[e + 1]; }   // next record in flight
+        const uint32_t kind = (uint32_t)(a >> 62);
+        const uint32_t r = (uint32_t)b & 0xffffu;
+        if (kind == 0) {
+            const uint32_t nw = (uint32_t)(a >> 48) & 31u;
+            if (nw <= 3) {
+                if (nw > 0) D = fmax(D, endb[3 * ((uint32_t)a & 0xffffu) + 2] - x);
+                if (nw > 1) D = fmax(D, endb[3 * ((uint32_t)(a >> 16) & 0xffffu) + 2] - x);
+                if (nw > 2) D = fmax(D, endb[3 * ((uint32_t)(a >> 32) & 0xffffu) + 2] - x);
+            } else {
+                uint32_t m = (uint32_t)(b >> 16) & 0x7fffffffu;
+                const uint32_t off = (uint32_t)(b >> 47) & 0xffffu;
+                while (m) {
+                    const uint32_t i = __ffs(m) - 1;
+                    m &= m - 1;
+                    D = fmax(D, endb[3 * (uint32_t)t.lul[off + i] + 2] - x);
+                }
             }
-            if ((inf >> 31) & 1ull) {                                 // producer of a swapped tensor ends
-                const uint32_t r = (uint32_t)(inf >> 32) & 0xffffu;
-                endb[3 * r] = cw + D + t.rtab[r].x;
-            }
+            if (r) endb[3 * (r - 1)] = x + D + t.rtab[r - 1].x;             // producer of a swapped tensor ends
+        } else if (kind == 1) {
+            Td = fmax(Td, endb[3 * r]) + x;                                  // Store
+            endb[3 * r + 1] = Td;
         } else {
-            const uint32_t q = (uint32_t)(w - t.n), r = q / 3, o = q - 3 * r;
-            if (o == 1) { Td = fmax(Td, endb[3 * r]) + t.rtab[r].y; endb[3 * r + 1] = Td; }      // Store
-            else { Th = fmax(Th, endb[3 * r + 1]) + t.rtab[r].y; endb[3 * r + 2] = Th; }       // Load
+            Th = fmax(Th, endb[3 * r + 1]) + x;                              // Load
+            endb[3 * r + 2] = Th;
         }
     }
 }
 
 // Latency of one swapping candidate from its event steps (key, cb in step
-// order): the warp resolves every step in parallel (cost prefix completed
-// with its warp offset, swap bits via step_info), then lane 0 walks them.
+// order): the warp resolves every step in parallel, then lane 0 walks them.
 __device__ __forceinline__ double candidate_latency(unsigned long long* key, double* cbp, unsigned long long* inf,
                                                     int ne, const double* woff, const uint8_t* dd, double* endb,
                                                     const WalkTabs& t, double ctot, int lane) {
-    for (int e = lane; e < ne; e += 32) {
-        const unsigned long long kk = key[e];
-        const int32_t stp = (int32_t)(kk >> 32), w = (int32_t)(kk & 0xffffffffu);
-        cbp[e] += woff[(stp >> t.lgL) >> 5];
-        inf[e] = step_info(w, t.n, dd, t.ninfo, t.lul);
-    }
+    for (int e = lane; e < ne; e += 32) resolve_event(key[e], cbp[e], inf[e], woff, dd, t);
     __syncwarp();
     double lat = 0.0;
     if (lane == 0) {
         double D = 0.0, Td = 0.0, Th = 0.0;
-        walk_events(key, cbp, inf, ne, endb, t, D, Td, Th);
+        walk_events(inf, key, cbp, ne, endb, t, D, Td, Th);
         lat = fmax(fmax(ctot + D, Td), Th);
     }
     return lat;
@@ -361,7 +386,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     unsigned long long* evi_s = (unsigned long long*)(sm + pl.off_ev + (size_t)2 * P * cap * 16);   // [2][P][cap]
 
     // pos / last of the virtual and dummy slots start (and the dummy stays) 0
-    for (int i = tid; i < pl.NTX * P; i += TM + TL) { pos[i] = 0; last[i] = 0; }
+    for (int i = tid; i < pl.NTX * P; i += TM + TL) {
+        pos[i] = 0;
+        if constexpr (!kScatter) last[i] = 0;
+    }
     for (int i = tid; i < P * nwm; i += TM + TL) evm[i] = 0;
     if constexpr (kScatter) {
         uint4* af4 = reinterpret_cast<uint4*>(AF);
@@ -418,6 +446,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     ctot = __shfl_sync(0xffffffffu, cc, WT - 1);
                     __syncwarp();
                 }
+                PROF_MARK(10);
                 if (st) {
                 } else if (!h.swp[c]) {
                     double bl = 0.0;                 // no swap: base cost + re-computations
@@ -431,8 +460,18 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     const int ne = h.nev[c];
                     if (ne <= cap) {
                         const size_t b0 = (size_t)(slot * P + c) * cap;
-                        lat = candidate_latency(evk_s + b0, evc_s + b0, evi_s + b0, ne, woff, dd, endb, wt, ctot,
-                                                lane);
+                        unsigned long long* key = evk_s + b0;
+                        unsigned long long* inf = evi_s + b0;
+                        double* cbp = evc_s + b0;
+                        for (int e = lane; e < ne; e += 32) resolve_event(key[e], cbp[e], inf[e], woff, dd, wt);
+                        __syncwarp();
+                        PROF_MARK(11);
+                        if (lane == 0) {
+                            double D = 0.0, Td = 0.0, Th = 0.0;
+                            walk_events(inf, key, cbp, ne, endb, wt, D, Td, Th);
+                            lat = fmax(fmax(ctot + D, Td), Th);
+                        }
+                        PROF_MARK(12);
                     } else {
                         char* ob = ovf + ((size_t)cta * 8 + slot * 4 + c) * pl.ovf_stride;
                         const size_t me = (size_t)pl.max_events;
@@ -453,7 +492,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         }
         if (prof)
 #pragma unroll
-            for (int i = 13; i < 16; i++) atomicAdd((unsigned long long*)(ovf + pl.prof_off) + i, pt[i]);
+            for (int i = 10; i < 16; i++) atomicAdd((unsigned long long*)(ovf + pl.prof_off) + i, pt[i]);
         return;
     }
 
@@ -531,11 +570,24 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             int bad = 0;
             const bool vc = (vmask >> cm) & 1u;
             if constexpr (LMAX <= kRegL) {
+                if (vc && L == LMAX && lo + LMAX <= NT) {
+                    // full chunk: no per-step tests; an out-of-range id goes to
+                    // the trash slot NTX (never read) and flags the candidate
+                    const uint32_t trash = (uint32_t)pl.NTX;
+                    uint16_t* pc_ = pos + cm;
 #pragma unroll
-                for (int j = 0; j < LMAX; j++) {
-                    if (vc && j < L && lo + j < NT) {
-                        const int32_t v = pr[j];
-                        if ((uint32_t)v < (uint32_t)NT) pos[v * P + cm] = (uint16_t)(lo + j + 1); else bad = 1;
+                    for (int j = 0; j < LMAX; j++) {
+                        const uint32_t v = (uint32_t)pr[j];
+                        bad |= v >= (uint32_t)NT;
+                        pc_[min(v, trash) * P] = (uint16_t)(lo + j + 1);
+                    }
+                } else {
+#pragma unroll
+                    for (int j = 0; j < LMAX; j++) {
+                        if (vc && j < L && lo + j < NT) {
+                            const int32_t v = pr[j];
+                            if ((uint32_t)v < (uint32_t)NT) pos[v * P + cm] = (uint16_t)(lo + j + 1); else bad = 1;
+                        }
                     }
                 }
             } else {
@@ -775,24 +827,48 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             int o = wpre + evx;
             const int o0 = o;
             constexpr int kUnroll5 = LR > 1 ? LMAX : 8;     // full unroll only with the chunk in registers
-#pragma unroll kUnroll5
-            for (int j = 0; j < LMAX; j++) {
-                if (j < nst) {
-                    const uint2 af = AF[cm * Sl + j * S + tt];     // alloc / free of the step (units)
+            const uint2* afp = AF + cm * Sl + tt;            // step lo + j of candidate cm at afp[j * S]
+            // memory: alloc = size of the op at each step, free = slot
+            if (L == LMAX && nst == LMAX) {
+#pragma unroll
+                for (int j = 0; j < LMAX; j++) {
+                    const uint2 af = afp[j * S];
                     s1 += af.x;
                     m1 = max(m1, s1);
                     s1 -= af.y;
-                    if (mysw) {
+                }
+            } else {
+#pragma unroll kUnroll5
+                for (int j = 0; j < LMAX; j++) {
+                    if (j < nst) {
+                        const uint2 af = afp[j * S];
+                        s1 += af.x;
+                        m1 = max(m1, s1);
+                        s1 -= af.y;
+                    }
+                }
+            }
+            if (mysw) {
+                // swapping candidate: compute-cost prefix (two partial sums
+                // halve the dependent fp64 chain) and the chunk's event steps in
+                // step order; an inactive clone (pos 0) costs nothing
+                double ca = 0.0, cb = 0.0;
+#pragma unroll kUnroll5
+                for (int j = 0; j < LMAX; j++) {
+                    if (j < nst) {
                         const int32_t v = LMAX <= kRegL ? pr[j % LR]
                                                      : __ldg(perm + (grp * P + cm) * (int64_t)NT + lo + j);
                         if ((mbits >> j) & 1ull) {
                             kout[o] = ((unsigned long long)(lo + j) << 32) | (uint32_t)v;
-                            cout_[o] = cs1;
+                            cout_[o] = ca + cb;
                             o++;
                         }
-                        if (v < n || pos[v * P + cm] != 0) cs1 += cost_s[v];
+                        double c = cost_s[v];
+                        if (v >= n && pos[v * P + cm] == 0) c = 0.0;
+                        if (j & 1) cb += c; else ca += c;
                     }
                 }
+                cs1 = ca + cb;
             }
             {
                 // warp-level monoid scan: (s1, m1) then (s2, m2) = (s1 + s2, max(m1, s1 + m2))

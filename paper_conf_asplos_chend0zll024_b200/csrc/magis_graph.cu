@@ -82,11 +82,13 @@ cudaError_t dispatch_eval(const magis_graph* g, int64_t K, const int32_t* perm, 
             cudaMemcpy(h, (char*)g->ovf2 + g->plan2.prof_off, 128, cudaMemcpyDeviceToHost);
             cudaMemset((char*)g->ovf2 + g->plan2.prof_off, 0, 128);
             unsigned long long tot = 0;
-            for (int i = 1; i < 13; i++) tot += h[i];
+            for (int i = 1; i < 10; i++) tot += h[i];
             std::fprintf(stderr, "[magis-prof] main:");
-            for (int i = 1; i < 13; i++) std::fprintf(stderr, " p%d=%.1f%%", i, tot ? 100.0 * h[i] / tot : 0.0);
-            std::fprintf(stderr, " | sweep wait=%llu busy=%llu arrive=%llu (main total %llu)\n", h[14], h[15],
-                         h[13], tot);
+            for (int i = 1; i < 10; i++) std::fprintf(stderr, " p%d=%.1f%%", i, tot ? 100.0 * h[i] / tot : 0.0);
+            std::fprintf(stderr,
+                         " | latency warp: wait=%llu fold=%llu resolve=%llu walk=%llu rest=%llu arrive=%llu"
+                         " (main total %llu)\n",
+                         h[14], h[10], h[11], h[12], h[15], h[13], tot);
         }
         return e;
     }

@@ -145,13 +145,18 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     const uint16_t nop = (uint16_t)dummy;
     const uint32_t nophdr = (kNop << kKindShift) | dummy;
     Rows cr = make_rows(cons, hdrs, nop, nophdr, WM);
-    Rows fr = make_rows(ins, hdrs, nop, nophdr, WM);
-    std::vector<uint32_t> wtab(WM * 4);
+    // input rows only where the frees are gathered (slots in global memory);
+    // with the slots in shared memory phase 3 scatters the frees instead
+    Rows fr;
+    if (gmem_af) fr = make_rows(ins, hdrs, nop, nophdr, WM);
+    std::vector<uint32_t> wtab(WM * 4, 0);
     for (int w = 0; w < WM; w++) {
         wtab[4 * w + 0] = cr.wtab[2 * w];
         wtab[4 * w + 1] = cr.wtab[2 * w + 1];
-        wtab[4 * w + 2] = fr.wtab[2 * w];
-        wtab[4 * w + 3] = fr.wtab[2 * w + 1];
+        if (gmem_af) {
+            wtab[4 * w + 2] = fr.wtab[2 * w];
+            wtab[4 * w + 3] = fr.wtab[2 * w + 1];
+        }
     }
     std::vector<uint32_t> size_u(NTX, 0);
     std::vector<double> cost_u(NTX, 0.0);
@@ -204,8 +209,10 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     p.af_bytes = (uint64_t)((P * Sl * 8 + 255) / 256 * 256);
     if (gmem_static) o = 0;
     p.state_base = (uint32_t)o;
-    p.off_pos = (uint32_t)o;  o = a16(o + (size_t)NTX * P * 2);
-    p.off_last = (uint32_t)o; o = a16(o + (size_t)NTX * P * 2);
+    // pos: NTX slots + one trash slot (out-of-range ids of a bad permutation
+    // are written there); last: only where phase 4 gathers the frees
+    p.off_pos = (uint32_t)o;  o = a16(o + (size_t)(NTX + 1) * P * 2);
+    p.off_last = (uint32_t)o; o = a16(o + (gmem_af ? (size_t)NTX * P * 2 : 0));
     p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * 8));
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
