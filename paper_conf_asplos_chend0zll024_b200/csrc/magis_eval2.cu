@@ -301,7 +301,10 @@ __device__ __forceinline__ double candidate_latency(unsigned long long* key, dou
 }
 
 // MODE 0: graph tables and step slots in shared memory; 1: tables read from
-// the global image; 2: tables and step slots in global memory (large graphs).
+// the global image; 2: tables and step slots in global memory (large graphs);
+// 3: tables read from the global image, free-only step slots (u32) in shared
+// memory, the alloc of each step gathered by the scan from the size table
+// (large graphs whose (alloc, free) slots do not fit).
 // TEAMS: independent teams per CTA (each TM main threads + its latency warps,
 // its own per-group state, slots and named barriers; the tables are shared),
 // so one team's barrier waits overlap the other's work.
@@ -319,6 +322,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // per-step slots in shared memory: phase 3 scatters alloc / free into them
     // (smem atomics); in global memory (MODE 2) phase 4 gathers the frees instead
     constexpr bool kScatter = MODE != 2;
+    constexpr bool kFO = MODE == 3;            // free-only slots, alloc gathered in the scan
     extern __shared__ __align__(128) char sm_all[];
     __shared__ uint64_t mbar;
     __shared__ SlotHdr hdr_t[TEAMS][2];
@@ -393,8 +397,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     for (int i = tid; i < P * nwm; i += TM + TL) evm[i] = 0;
     if constexpr (kScatter) {
         uint4* af4 = reinterpret_cast<uint4*>(AF);
-        for (int i = tid; i < P * Sl / 2; i += TM + TL) af4[i] = make_uint4(0u, 0u, 0u, 0u);
+        for (int i = tid; i < P * Sl / (kFO ? 4 : 2); i += TM + TL) af4[i] = make_uint4(0u, 0u, 0u, 0u);
     }
+    uint32_t* Fs = reinterpret_cast<uint32_t*>(AF);   // MODE 3: [P][Sl] free per step (size units)
     if (tid == 0) {
         for (int b = 0; b < 2; b++) {
             for (int c = 0; c < 4; c++) ctl[b].flags[c] = ctl[b].viol[c] = 0;
@@ -649,7 +654,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const bool act = (o == 0) ? (d == 1) : (d == 2);
                 const uint32_t st = p - 1;
                 if (!act) {
-                    AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
+                    // (MODE 3: no free lands on an absent node's step, its alloc is
+                    // gathered as 0 from pos)
+                    if constexpr (!kFO) AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
                     pc_[id * P] = 0;
                 } else if (o > 0) {
                     atomicOr(em + (st >> 5), 1u << (st & 31));
@@ -702,10 +709,12 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                             const uint32_t pc = PK::get(p, c);
                             if (pc == 0) continue;                  // absent (inactive) in candidate c
                             const uint32_t st = pc - 1;
-                            AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)].x = A;
+                            if constexpr (!kFO) AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)].x = A;
                             if (kind != kHdrOut && A != 0) {
                                 const uint32_t fs = PK::get(lst, c) - 1;
-                                atomicAdd(&AF[c * Sl + (fs & (L - 1)) * S + (fs >> lgL)].y, A);
+                                const uint32_t fi = c * Sl + (fs & (L - 1)) * S + (fs >> lgL);
+                                if constexpr (kFO) atomicAdd(&Fs[fi], A);
+                                else atomicAdd(&AF[fi].y, A);
                             }
                         }
                     } else {
@@ -828,6 +837,34 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             const int o0 = o;
             constexpr int kUnroll5 = LR > 1 ? LMAX : 8;     // full unroll only with the chunk in registers
             const uint2* afp = AF + cm * Sl + tt;            // step lo + j of candidate cm at afp[j * S]
+            if constexpr (kFO) {
+                // one pass: the step's op from the perm (last read of the chunk),
+                // its alloc gathered from the size table (0 if absent), the free
+                // from the slot; with swaps the cost prefix and the events too
+                const uint32_t* fp = Fs + cm * Sl + tt;
+                const int32_t* pp = perm + (grp * P + cm) * (int64_t)NT + lo;
+                double ca = 0.0, cb = 0.0;
+#pragma unroll kUnroll5
+                for (int j = 0; j < LMAX; j++) {
+                    if (j < nst) {
+                        const int32_t v = LMAX <= kRegL ? pr[j % LR] : __ldcs(pp + j);
+                        const bool act = v < n || pos[v * P + cm] != 0;
+                        s1 += act ? __ldg(size_s + v) : 0u;
+                        m1 = max(m1, s1);
+                        s1 -= fp[j * S];
+                        if (mysw) {
+                            if ((mbits >> j) & 1ull) {
+                                kout[o] = ((unsigned long long)(lo + j) << 32) | (uint32_t)v;
+                                cout_[o] = ca + cb;
+                                o++;
+                            }
+                            const double c = act ? __ldg(cost_s + v) : 0.0;
+                            if (j & 1) cb += c; else ca += c;
+                        }
+                    }
+                }
+                cs1 = ca + cb;
+            } else
             // memory: alloc = size of the op at each step, free = slot
             if (L == LMAX && nst == LMAX) {
 #pragma unroll
@@ -848,7 +885,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     }
                 }
             }
-            if (mysw) {
+            if (!kFO && mysw) {
                 // swapping candidate: compute-cost prefix (two partial sums
                 // halve the dependent fp64 chain) and the chunk's event steps in
                 // step order; an inactive clone (pos 0) costs nothing
@@ -933,7 +970,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             for (int i = tid; i < P * nwm; i += TM) evm[i] = 0;
             if constexpr (kScatter) {           // the per-step slots start from 0 for the scatter
                 uint4* af4 = reinterpret_cast<uint4*>(AF);
-                for (int i = tid; i < P * Sl / 2; i += TM) af4[i] = make_uint4(0u, 0u, 0u, 0u);
+                for (int i = tid; i < P * Sl / (kFO ? 4 : 2); i += TM) af4[i] = make_uint4(0u, 0u, 0u, 0u);
             }
         }
         bar_sync(kBarMain + bb, TM);
@@ -965,9 +1002,9 @@ static const void* kernel_mode(const Plan2& pl) {
 }
 
 static const void* kernel_for(const Plan2& pl) {
-    const int mode = pl.gmem_af ? 2 : (pl.gmem_static ? 1 : 0);
+    const int mode = pl.gmem_af ? 2 : pl.free_only ? 3 : (pl.gmem_static ? 1 : 0);
     if (mode == 0) return pl.teams == 2 ? kernel_mode<0, 2>(pl) : kernel_mode<0, 1>(pl);
-    return mode == 1 ? kernel_mode<1, 1>(pl) : kernel_mode<2, 1>(pl);
+    return mode == 1 ? kernel_mode<1, 1>(pl) : mode == 3 ? kernel_mode<3, 1>(pl) : kernel_mode<2, 1>(pl);
 }
 
 int eval2_block(const Plan2& pl) { return kMainThreads2 + pl.teams * 32 * pl.P; }

@@ -477,8 +477,12 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
             int bestP = 0, bestOcc = 0, bestT = 1;
             Plan2 bestPl{};
             std::vector<char> bestImg;
-            for (int tier = 0; tier < 3 && bestP == 0; tier++) {
-                const bool gs = tier >= 1, ga = tier >= 2;
+            // tier 2 = tables in global, free-only slots in shared memory (the
+            // scan gathers the allocs); tier 3 = tables and slots in global
+            const char* tierf = std::getenv("MAGIS_TIER");
+            for (int tier = 0; tier < 4 && bestP == 0; tier++) {
+                if (tierf && std::atoi(tierf) != tier) continue;
+                const bool gs = tier >= 1, fo = tier == 2, ga = tier == 3;
                 for (int T = 2; T >= 1; T--) {
                     if (tforce && std::atoi(tforce) != T) continue;
                     if (T == 2 && gs) continue;                     // teams only with the tables in smem
@@ -487,7 +491,7 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
                         if (pforce && std::atoi(pforce) != P) continue;
                         Plan2 pl;
                         std::vector<char> img;
-                        if (!plan2_build(sg, P, T, gs, ga, cap, &pl, &img)) continue;
+                        if (!plan2_build(sg, P, T, gs, ga, fo, cap, &pl, &img)) continue;
                         int occ = 0;
                         cudaError_t oe = eval2_occupancy(pl, &occ);
                         if (std::getenv("MAGIS_DEBUG"))

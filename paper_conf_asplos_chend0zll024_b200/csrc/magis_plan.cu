@@ -96,7 +96,8 @@ Rows make_rows(const std::vector<std::vector<uint32_t>>& lists, const std::vecto
 }
 }  // namespace
 
-bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, size_t smem_cap,
+bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, bool free_only,
+                 size_t smem_cap,
                  Plan2* pl, std::vector<char>* img) {
     const int32_t NT = sg.NT, n = sg.n, R = sg.R;
     const int32_t nU = R > 0 ? sg.U_ptr[R] : 0;
@@ -205,6 +206,8 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     // in a per-CTA global slice
     p.gmem_static = gmem_static ? 1 : 0;
     p.gmem_af = gmem_af ? 1 : 0;
+    p.free_only = (free_only && !gmem_af) ? 1 : 0;
+    if (p.free_only && !gmem_static) return false;      // MODE 3 reads the tables from the global image
     const size_t Sl = (size_t)p.L * p.S;
     p.af_bytes = (uint64_t)((P * Sl * 8 + 255) / 256 * 256);
     if (gmem_static) o = 0;
@@ -213,7 +216,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     // are written there); last: only where phase 4 gathers the frees
     p.off_pos = (uint32_t)o;  o = a16(o + (size_t)(NTX + 1) * P * 2);
     p.off_last = (uint32_t)o; o = a16(o + (gmem_af ? (size_t)NTX * P * 2 : 0));
-    p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * 8));
+    p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * (p.free_only ? 4 : 8)));
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
     p.nwm = (NT + 31) / 32 + 2;

@@ -27,12 +27,17 @@ DEV = "cuda:0"
 # P = 1 / 2 / 4 packed candidates; "auto" is what the loader picks.
 VARIANTS = {"auto": {}, "v1": {"MAGIS_VARIANT": "1"}, "p1": {"MAGIS_P": "1", "MAGIS_TEAMS": "1"},
             "p2": {"MAGIS_P": "2", "MAGIS_TEAMS": "1"}, "p4": {"MAGIS_P": "4", "MAGIS_TEAMS": "1"},
-            "t2p1": {"MAGIS_P": "1", "MAGIS_TEAMS": "2"}, "t2p2": {"MAGIS_P": "2", "MAGIS_TEAMS": "2"}}
+            "t2p1": {"MAGIS_P": "1", "MAGIS_TEAMS": "2"}, "t2p2": {"MAGIS_P": "2", "MAGIS_TEAMS": "2"},
+            # plan tiers: 1 tables in global, 2 + free-only slots (alloc gathered), 3 slots in global
+            "tier1p4": {"MAGIS_TIER": "1", "MAGIS_P": "4", "MAGIS_TEAMS": "1"},
+            "tier2p1": {"MAGIS_TIER": "2", "MAGIS_P": "1", "MAGIS_TEAMS": "1"},
+            "tier2p4": {"MAGIS_TIER": "2", "MAGIS_P": "4", "MAGIS_TEAMS": "1"},
+            "tier3p2": {"MAGIS_TIER": "3", "MAGIS_P": "2", "MAGIS_TEAMS": "1"}}
 
 
 @pytest.fixture(params=list(VARIANTS))
 def variant(request, monkeypatch):
-    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS"):
+    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER"):
         monkeypatch.delenv(k, raising=False)
     for k, v in VARIANTS[request.param].items():
         monkeypatch.setenv(k, v)
