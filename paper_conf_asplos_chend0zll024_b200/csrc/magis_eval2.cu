@@ -361,6 +361,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // read in place from the global image when they do not fit
     const char* sb = MODE ? blob : sm_all;
     if (MODE == 0) bulk_stage(sm_all, blob, pl.static_bytes, &mbar);
+    else if (pl.cost_sm) bulk_stage(sm_all, blob + pl.off_cost, (uint32_t)((pl.NTX * 8 + 15) & ~15), &mbar);
     const uint32_t* wtab = (const uint32_t*)(sb + pl.off_wtab);   // [WM][4]: consumer rows, input rows
     const uint2* crow = (const uint2*)(sb + pl.off_crow);
     const uint32_t* chdr = (const uint32_t*)(sb + pl.off_chdr);
@@ -370,7 +371,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const uint16_t* fent = (const uint16_t*)(sb + pl.off_fent);
     const uint32_t* size_s = (const uint32_t*)(sb + pl.off_size);
     const double2* rtab = (const double2*)(sb + pl.off_rtab);       // [R] (cost(t_r), swap transfer time)
-    const double* cost_s = (const double*)(sb + pl.off_cost);
+    const double* cost_s = (MODE != 0 && pl.cost_sm) ? (const double*)sm_all : (const double*)(sb + pl.off_cost);
     const uint2* ninfo = (const uint2*)(sb + pl.off_ninfo);
     const uint16_t* lul = (const uint16_t*)(sb + pl.off_lul);
     const uint32_t* urow = (const uint32_t*)(sb + pl.off_urow);     // [R] U_r offset | |U_r| << 16
@@ -541,6 +542,16 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     if constexpr (LMAX <= kRegL) {
         if (ncta > 0) load_chunk(cta);
     }
+    // the group's decisions (<= 2 bytes per thread) are prefetched into
+    // registers one group ahead, like the perm chunk
+    const bool dreg = P * R <= 2 * TM;
+    uint32_t dq0 = 0, dq1 = 0;
+    auto load_dec = [&](int64_t grp_) {
+        const int64_t b = grp_ * P * (int64_t)R, lim = K * (int64_t)R;
+        dq0 = (tid < P * R && b + tid < lim) ? (uint32_t)__ldcs(dec + b + tid) : 0u;
+        dq1 = (tid + TM < P * R && b + tid + TM < lim) ? (uint32_t)__ldcs(dec + b + tid + TM) : 0u;
+    };
+    if (dreg && R > 0 && ncta > 0) load_dec(cta);
     for (int gi = 0; gi < ncta; gi++) {
         const int64_t grp = cta + (int64_t)gi * ncta_all;
         const int slot = gi & 1;
@@ -551,9 +562,13 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         // ---- phase 0: decisions ---------------------------------------------
         {
             uint32_t badm = 0, swm = 0;
-            for (int i = tid, c = c_0, r = r_0; i < P * R; i += TM, c += dc_, r += dr_) {
+            int it = 0;
+            for (int i = tid, c = c_0, r = r_0; i < P * R; i += TM, c += dc_, r += dr_, it++) {
                 if (r >= R) { r -= R; c++; }
-                const uint8_t d = ((vmask >> c) & 1u) ? dec[(grp * P + c) * (int64_t)R + r] : 0;
+                // the group's decision rows are contiguous: dec[grp * P * R + i]
+                uint8_t d;
+                if (dreg) d = (uint8_t)(it == 0 ? dq0 : dq1);
+                else d = ((vmask >> c) & 1u) ? dec[grp * P * (int64_t)R + i] : 0;
                 dec_s[i] = d;
                 if (d == 2) swm |= 1u << c;
                 if ((d > 2) | ((d == 1) & !(__ldg(g.rflag + r) & kRHasInput))) badm |= 1u << c;
@@ -858,7 +873,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                                 cout_[o] = ca + cb;
                                 o++;
                             }
-                            const double c = act ? __ldg(cost_s + v) : 0.0;
+                            const double c = act ? cost_s[v] : 0.0;     // shared or global table
                             if (j & 1) cb += c; else ca += c;
                         }
                     }
@@ -924,10 +939,11 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 for (int e = o0; e < o; e++) cout_[e] += pre;
             }
         }
-        // the next group's chunk is loaded while this group finishes
+        // the next group's chunk and decisions are loaded while this group finishes
         if constexpr (LMAX <= kRegL) {
             if (gi + 1 < ncta) load_chunk(grp + ncta_all);
         }
+        if (dreg && R > 0 && gi + 1 < ncta) load_dec(grp + ncta_all);
         bar_sync(kBarMain + bb, TM);
         PROF_MARK(5);
         // ---- phase 6: hand-off to the latency warps (they fold the aggregates) ----

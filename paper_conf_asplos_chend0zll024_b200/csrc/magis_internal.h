@@ -99,6 +99,7 @@ struct Plan2 {
     uint32_t smem_total;
     int32_t gmem_static;  // graph tables read from the global image instead of shared memory
     int32_t gmem_af;      // per-step slots in a per-CTA global slice (af_bytes each)
+    int32_t cost_sm;      // tables in global, but the cost table staged at shared offset 0
     int32_t free_only;    // per-step slots hold only the free (u32, shared memory); the scan gathers the alloc
     uint32_t state_base;  // offset of the per-candidate state in shared memory
     uint64_t af_bytes;

@@ -210,7 +210,13 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     if (p.free_only && !gmem_static) return false;      // MODE 3 reads the tables from the global image
     const size_t Sl = (size_t)p.L * p.S;
     p.af_bytes = (uint64_t)((P * Sl * 8 + 255) / 256 * 256);
-    if (gmem_static) o = 0;
+    const size_t static_end = o;
+    // tables read from the global image: the cost table (the swap scan's
+    // random gather) is still staged into shared memory when it fits with
+    // at least 32 event slots per candidate
+    for (int csm = gmem_static ? 1 : 0; csm >= 0; csm--) {
+    o = gmem_static ? (csm ? a16((size_t)NTX * 8) : 0) : static_end;
+    p.cost_sm = csm;
     p.state_base = (uint32_t)o;
     // pos: NTX slots + one trash slot (out-of-range ids of a bad permutation
     // are written there); last: only where phase 4 gathers the frees
@@ -226,18 +232,26 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     // event steps of a candidate: at most the marked steps (<= 3R + |U|)
     int cap = std::min(std::max(p.max_events, 1), 128);
     p.teams = teams;
+    bool fit = false;
     while (true) {
         const size_t st = a16(o + (size_t)2 * P * cap * 24) - p.state_base;     // one team's state
         const size_t need = p.state_base + (size_t)teams * st;
         if (need <= smem_cap) {
             p.smem_total = (uint32_t)a16(need);
             p.state_stride = (uint32_t)st;
+            fit = true;
             break;
         }
-        if (cap <= 8) return false;
+        if (cap <= (csm ? 32 : 8)) break;
         cap /= 2;
     }
+    if (!fit) {
+        if (csm) continue;
+        return false;
+    }
     p.evcap = cap;
+    break;
+    }
     p.ovf_stride = (uint64_t)((std::max(p.max_events, 1) * 24 + 255) / 256 * 256);
     *pl = p;
     img->assign(p.static_bytes, 0);
