@@ -13,7 +13,8 @@ from typing import Optional, Sequence
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libmagis.so")
+# MAGIS_LIB: an alternative in-tree build (A/B timing of kernel variants)
+LIB_PATH = os.environ.get("MAGIS_LIB") or os.path.join(_PKG, "libmagis.so")
 
 MAGIS_SUCCESS = 0
 ERRORS = {-1: "MAGIS_E_INVAL", -2: "MAGIS_E_CYCLE", -3: "MAGIS_E_NOMEM", -4: "MAGIS_E_CUDA",
