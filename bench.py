@@ -43,7 +43,7 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle CPU-baseline wall time")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--e2e-wire", default="delta8", choices=["delta8", "u16", "int32"],
+    ap.add_argument("--e2e-wire", default="delta4", choices=["delta4", "delta8", "u16", "int32"],
                     help="host schedule format of the e2e call (delta8 / u16 need n_total <= 65535)")
     ap.add_argument("--ghash", action="store_true",
                     help="batched GraphHash + duplicate filter of the K candidates' graphs (NEXT-2)")
@@ -326,12 +326,14 @@ def main():
         out_pinned = (torch.empty(K, dtype=torch.uint8).pin_memory(), torch.empty(K, dtype=torch.int64).pin_memory(),
                       torch.empty(K, dtype=torch.float64).pin_memory())
         # schedules cross PCIe in a compact wire format when the super-graph
-        # has < 65536 nodes: delta8 (~1.1 B / step, magis_eval_schedules_host_delta8)
-        # or u16 (magis_eval_schedules_host_u16); encoded once, outside the timed region
+        # has < 65536 nodes: delta4 (a nibble per step + escapes, magis_eval_schedules_host_delta4),
+        # delta8 (~1.1 B / step, magis_eval_schedules_host_delta8) or u16
+        # (magis_eval_schedules_host_u16); encoded once, outside the timed region
         wire = args.e2e_wire if NT <= 65535 else "int32"
-        from paper_conf_asplos_chend0zll024_b200 import encode_delta8
-        if wire == "delta8":
-            Ph_w = tuple(torch.from_numpy(a).pin_memory() for a in encode_delta8(Ph))
+        from paper_conf_asplos_chend0zll024_b200 import encode_delta4, encode_delta8
+        if wire in ("delta4", "delta8"):
+            enc = encode_delta4 if wire == "delta4" else encode_delta8
+            Ph_w = tuple(torch.from_numpy(a).pin_memory() for a in enc(Ph))
             wire_bytes = sum(int(a.numel()) * a.element_size() for a in Ph_w)
         elif wire == "u16":
             Ph_w = torch.from_numpy(Ph.astype(np.uint16)).pin_memory()
@@ -350,7 +352,8 @@ def main():
         te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        api = {"delta8": "magis_eval_schedules_host_delta8 (delta8 schedules",
+        api = {"delta4": "magis_eval_schedules_host_delta4 (delta4 schedules",
+               "delta8": "magis_eval_schedules_host_delta8 (delta8 schedules",
                "u16": "magis_eval_schedules_host_u16 (uint16 schedules",
                "int32": "magis_eval_schedules_host (int32 schedules"}[wire]
         e2e = {"value": round(world * K / te.item(), 1), "unit": UNIT,

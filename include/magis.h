@@ -236,6 +236,20 @@ int magis_eval_schedules_host_delta8(magis_graph* g, int64_t K, const int8_t* h_
                                      int64_t* h_peak, double* h_latency, void* cuda_stream);
 
 /*
+ * As magis_eval_schedules_host_delta8 with one nibble per step (the delta4
+ * wire format, n_total <= 65535): row k is h_code[k * ceil(n_total / 2) ..],
+ * step j in byte j / 2, the low nibble first; nibble c = 0 means "the next
+ * value of this row's exception list" (an absolute uint16 id), any other c a
+ * difference of c - 8 (-7 .. +7) to the previous step's id (the row starts
+ * from 0); the pad nibble of an odd-length row is ignored.  ~0.5 byte per step
+ * plus 2 bytes per escaped step across PCIe (C2: 87% of steps move by at most
+ * 7 ids).  Errors as magis_eval_schedules_host_delta8.
+ */
+int magis_eval_schedules_host_delta4(magis_graph* g, int64_t K, const uint8_t* h_code, const int32_t* h_exc_ptr,
+                                     const uint16_t* h_exc, const uint8_t* h_dec, uint8_t* h_status,
+                                     int64_t* h_peak, double* h_latency, void* cuda_stream);
+
+/*
  * Seeded candidate generation on the device.  Candidate k
  * (global id id0 + i) depends only on (spec->seed, k), so ranks generate
  * their shards independently.  The recipe stands in for MAGIS's rule

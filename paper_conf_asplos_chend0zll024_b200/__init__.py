@@ -7,8 +7,8 @@ binding (magis.py) plus the multi-GPU front merge over torch.distributed
 (distributed.py).  PyTorch is used only for device memory, streams and
 process groups.
 """
-from .magis import (Base, Graph, GraphHasher, HashSet, MagisError, encode_delta8, pareto_merge, pareto_workspace_size, lib, ST_NOT_PERM,
+from .magis import (Base, Graph, GraphHasher, HashSet, MagisError, encode_delta4, encode_delta8, pareto_merge, pareto_workspace_size, lib, ST_NOT_PERM,
                     ST_EDGE, ST_BAD_DEC)
 
-__all__ = ["Base", "Graph", "GraphHasher", "HashSet", "MagisError", "encode_delta8", "pareto_merge", "pareto_workspace_size", "lib", "ST_NOT_PERM",
+__all__ = ["Base", "Graph", "GraphHasher", "HashSet", "MagisError", "encode_delta4", "encode_delta8", "pareto_merge", "pareto_workspace_size", "lib", "ST_NOT_PERM",
            "ST_EDGE", "ST_BAD_DEC"]

@@ -666,25 +666,38 @@ __global__ void widen_u16(const uint16_t* __restrict__ src, int32_t* __restrict_
         dst[i] = (int32_t)src[i];
 }
 
-// delta8 wire format: per step one int8 delta to the previous step's id
-// (the row starts from 0); -128 = "take the next value of the row's
-// exception list" (an absolute uint16 id).  One warp per row: the exception
-// ranks come from a ballot, and a segmented scan over (reset, value) pairs
-// rebuilds the ids 32 steps at a time.
-__global__ void decode_delta8(const int8_t* __restrict__ delta, const int32_t* __restrict__ exc_ptr,
-                              const uint16_t* __restrict__ exc, int64_t kc, int32_t NT, int32_t* __restrict__ out) {
+// Delta wire formats: per step the difference to the previous step's id (the
+// row starts from 0), or an escape = "take the next value of the row's
+// exception list" (an absolute uint16 id).  delta8: one int8 per step, escape
+// -128.  delta4: one nibble per step (step j in byte j / 2, low nibble first),
+// code c: 0 = escape, else delta c - 8 (-7 .. +7).  One warp per row: the
+// exception ranks come from a ballot, and a segmented scan over (reset, value)
+// pairs rebuilds the ids 32 steps at a time.
+template <int BITS>
+__global__ void decode_delta(const uint8_t* __restrict__ code, int64_t row_b, const int32_t* __restrict__ exc_ptr,
+                             const uint16_t* __restrict__ exc, int64_t kc, int32_t NT, int32_t* __restrict__ out) {
     const int lane = threadIdx.x & 31;
     const int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int32_t e0 = exc_ptr[0];
     for (int64_t k = w0; k < kc; k += nw) {
-        const int8_t* dr = delta + k * (int64_t)NT;
+        const uint8_t* dr = code + k * row_b;
         int32_t* orow = out + k * (int64_t)NT;
         int32_t carry = 0, ec = exc_ptr[k] - e0;
         for (int32_t t = 0; t < NT; t += 32) {
             const int32_t j = t + lane;
-            const int32_t b = j < NT ? (int32_t)dr[j] : 0;
-            const bool isx = j < NT && b == -128;
+            int32_t b = 0;
+            bool isx = false;
+            if (j < NT) {
+                if (BITS == 8) {
+                    b = (int32_t)(int8_t)dr[j];
+                    isx = b == -128;
+                } else {
+                    const int32_t c = (dr[j >> 1] >> ((j & 1) * 4)) & 15;
+                    isx = c == 0;
+                    b = c - 8;
+                }
+            }
             const unsigned m = __ballot_sync(0xffffffffu, isx);
             int32_t v = isx ? (int32_t)exc[ec + __popc(m & ((1u << lane) - 1u))] : b;
             bool rs = isx;
@@ -702,9 +715,9 @@ __global__ void decode_delta8(const int8_t* __restrict__ delta, const int32_t* _
     }
 }
 
-// pb = bytes per perm element on the host (4: int32, 2: uint16 widened on the
-// device, 1: delta8 decoded on the device -- h_exc_ptr / h_exc then hold the
-// exception lists)
+// pb = the host wire format (4: int32, 2: uint16 widened on the device,
+// 1: delta8, 0: delta4 -- both decoded on the device, h_exc_ptr / h_exc then
+// hold the exception lists)
 int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8_t* h_dec, uint8_t* h_status,
               int64_t* h_peak, double* h_latency, void* cuda_stream, const int32_t* h_exc_ptr = nullptr,
               const uint16_t* h_exc = nullptr) {
@@ -717,7 +730,8 @@ int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8
     const int32_t R = g->dev.Rd, NT = g->dev.NT;          // decision row: R eligible + F regions
     if (R > 0 && !h_dec) return set_error(MAGIS_E_INVAL, "h_dec is NULL but R + n_regions > 0");
     if (pb <= 2 && NT > 65535) return set_error(MAGIS_E_UNSUPPORTED, "compact schedules need n_total <= 65535");
-    if (pb == 1) {
+    const size_t row_b = pb == 0 ? (size_t)(NT + 1) / 2 : (size_t)NT * pb;   // host bytes per schedule
+    if (pb <= 1) {
         if (!h_exc_ptr) return set_error(MAGIS_E_INVAL, "null exception pointer array");
         for (int64_t k = 0; k < K; k++)
             if (h_exc_ptr[k + 1] < h_exc_ptr[k]) return set_error(MAGIS_E_INVAL, "exception offsets decrease");
@@ -759,11 +773,11 @@ int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8
         uint8_t* dst = (uint8_t*)(ob + 2 * align_up((size_t)chunk * 8, 64));
         // buffer b is free once the D2H of chunk c-2 finished
         if (c >= 2) CK(cudaStreamWaitEvent(g->aux, g->ev_done[b], 0));
-        const char* hp = (const char*)h_perm + (size_t)k0 * NT * pb;
+        const char* hp = (const char*)h_perm + (size_t)k0 * row_b;
         int32_t* dxp = (int32_t*)(ob + out_b + 256);    // past the outputs (which may spill 128 B over out_b)
         uint16_t* dxv = (uint16_t*)((char*)dxp + excp_b);
-        CK(cudaMemcpyAsync(pb == 4 ? (void*)dp : (void*)dn, hp, (size_t)kc * NT * pb, cudaMemcpyHostToDevice, g->aux));
-        if (pb == 1) {
+        CK(cudaMemcpyAsync(pb == 4 ? (void*)dp : (void*)dn, hp, (size_t)kc * row_b, cudaMemcpyHostToDevice, g->aux));
+        if (pb <= 1) {
             const int64_t x0 = h_exc_ptr[k0], x1 = h_exc_ptr[k0 + kc];
             CK(cudaMemcpyAsync(dxp, h_exc_ptr + k0, (size_t)(kc + 1) * 4, cudaMemcpyHostToDevice, g->aux));
             if (x1 > x0) CK(cudaMemcpyAsync(dxv, h_exc + x0, (size_t)(x1 - x0) * 2, cudaMemcpyHostToDevice, g->aux));
@@ -771,9 +785,10 @@ int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8
         if (R > 0) CK(cudaMemcpyAsync(dd, h_dec + k0 * R, (size_t)kc * R, cudaMemcpyHostToDevice, g->aux));
         CK(cudaEventRecord(g->ev_h2d[b], g->aux));
         CK(cudaStreamWaitEvent(s0, g->ev_h2d[b], 0));
-        if (pb == 1) {
+        if (pb <= 1) {
             const int blocks = (int)std::min<int64_t>((kc + 7) / 8, 4096);
-            decode_delta8<<<blocks, 256, 0, s0>>>((const int8_t*)dn, dxp, dxv, kc, NT, dp);
+            if (pb == 1) decode_delta<8><<<blocks, 256, 0, s0>>>((const uint8_t*)dn, (int64_t)row_b, dxp, dxv, kc, NT, dp);
+            else decode_delta<4><<<blocks, 256, 0, s0>>>((const uint8_t*)dn, (int64_t)row_b, dxp, dxv, kc, NT, dp);
         }
         if (pb == 2) {
             const int64_t ne = kc * (int64_t)NT;
@@ -815,6 +830,13 @@ extern "C" int magis_eval_schedules_host_delta8(magis_graph* g, int64_t K, const
                                                 const uint8_t* h_dec, uint8_t* h_status, int64_t* h_peak,
                                                 double* h_latency, void* cuda_stream) {
     return host_path(g, K, h_delta, 1, h_dec, h_status, h_peak, h_latency, cuda_stream, h_exc_ptr, h_exc);
+}
+
+extern "C" int magis_eval_schedules_host_delta4(magis_graph* g, int64_t K, const uint8_t* h_code,
+                                                const int32_t* h_exc_ptr, const uint16_t* h_exc,
+                                                const uint8_t* h_dec, uint8_t* h_status, int64_t* h_peak,
+                                                double* h_latency, void* cuda_stream) {
+    return host_path(g, K, h_code, 0, h_dec, h_status, h_peak, h_latency, cuda_stream, h_exc_ptr, h_exc);
 }
 
 extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* spec, uint64_t id0, int64_t K,

@@ -29,7 +29,7 @@ EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magi
            "magis_graph_idom", "magis_eval_schedules_host_u16", "magis_ghash_create", "magis_ghash_free",
            "magis_graph_hash", "magis_ghash_info", "magis_hashset_create", "magis_hashset_free",
            "magis_hashset_clear", "magis_hashset_filter", "magis_hashset_stats", "magis_graph_load_regions",
-           "magis_eval_schedules_host_delta8"]
+           "magis_eval_schedules_host_delta8", "magis_eval_schedules_host_delta4"]
 
 
 class MagisError(RuntimeError):
@@ -95,6 +95,8 @@ def lib() -> ctypes.CDLL:
     L.magis_eval_schedules_host_u16.restype = ctypes.c_int
     L.magis_eval_schedules_host_delta8.argtypes = [P, i64, P, P, P, P, P, P, P, P]
     L.magis_eval_schedules_host_delta8.restype = ctypes.c_int
+    L.magis_eval_schedules_host_delta4.argtypes = [P, i64, P, P, P, P, P, P, P, P]
+    L.magis_eval_schedules_host_delta4.restype = ctypes.c_int
     L.magis_pareto_workspace_size.argtypes = [i64]
     L.magis_pareto_workspace_size.restype = i64
     L.magis_pareto_merge.argtypes = [i64, P, P, P, P, i64, i64, P, P, P, P, i64, d, P, P, i64, P]
@@ -182,6 +184,31 @@ def encode_delta8(perm: np.ndarray):
     exc_ptr = np.zeros(p.shape[0] + 1, np.int32)
     np.cumsum(esc.sum(axis=1), out=exc_ptr[1:])
     return np.ascontiguousarray(delta), exc_ptr, exc
+
+
+def encode_delta4(perm: np.ndarray):
+    """The delta4 wire format of magis_eval_schedules_host_delta4 (marshalling
+    only): per step one nibble, c = d + 8 for a difference d in [-7, 7] to
+    the previous step's id (rows start from 0), c = 0 where it does not fit,
+    with the absolute ids of those steps in a per-row exception list; two
+    steps per byte, the even step in the low nibble.  Ids outside [0, 65535]
+    are clamped to 65535 (the candidate stays MAGIS_ST_NOT_PERM).
+    -> (code uint8 [K, ceil(n / 2)], exc_ptr int32 [K+1], exc uint16 [E])."""
+    p = np.asarray(perm, np.int64)
+    if p.ndim == 1:
+        p = p[None, :]
+    p = np.where((p < 0) | (p > 65535), 65535, p)
+    prev = np.concatenate([np.zeros((p.shape[0], 1), np.int64), p[:, :-1]], axis=1)
+    d = p - prev
+    esc = (d < -7) | (d > 7)
+    c = np.where(esc, 0, d + 8).astype(np.uint8)
+    if c.shape[1] % 2:
+        c = np.concatenate([c, np.full((c.shape[0], 1), 8, np.uint8)], axis=1)
+    code = (c[:, 0::2] | (c[:, 1::2] << 4)).astype(np.uint8)
+    exc = np.ascontiguousarray(p[esc], np.uint16)
+    exc_ptr = np.zeros(p.shape[0] + 1, np.int32)
+    np.cumsum(esc.sum(axis=1), out=exc_ptr[1:])
+    return np.ascontiguousarray(code), exc_ptr, exc
 
 
 class Graph:
@@ -314,7 +341,9 @@ class Graph:
                             stream=None):
         """End-to-end call with host buffers (pinned numpy views or torch CPU
         tensors).  A (delta, exc_ptr, exc) tuple from encode_delta8 uses the
-        delta8 wire format (magis_eval_schedules_host_delta8); uint16
+        delta8 wire format (magis_eval_schedules_host_delta8), a (code,
+        exc_ptr, exc) tuple from encode_delta4 (uint8 codes) the delta4 one
+        (magis_eval_schedules_host_delta4); uint16
         schedules the u16 format (magis_eval_schedules_host_u16); anything
         else is taken as int32."""
         import torch
@@ -323,18 +352,21 @@ class Graph:
             if isinstance(x, torch.Tensor):
                 return x.numpy()
             return np.ascontiguousarray(x, dt)
-        if isinstance(perm, tuple):           # delta8 wire format (encode_delta8)
+        if isinstance(perm, tuple):           # delta8 / delta4 wire format (encode_delta8 / encode_delta4)
             delta, exc_ptr, exc = (as_np(x, None) for x in perm)
             K = delta.shape[0]
-            assert delta.dtype == np.int8 and delta.shape[1] == self.n_total and exc_ptr.shape == (K + 1,)
+            d4 = delta.dtype == np.uint8
+            assert exc_ptr.shape == (K + 1,)
+            assert (d4 and delta.shape[1] == (self.n_total + 1) // 2) or (
+                delta.dtype == np.int8 and delta.shape[1] == self.n_total)
             dd = as_np(dec, np.uint8) if (self.dec_len and dec is not None) else None
             if out is None:
                 st, pk, lt = np.empty(K, np.uint8), np.empty(K, np.int64), np.empty(K, np.float64)
             else:
                 st, pk, lt = (as_np(o, None) for o in out)
-            _check(self._L.magis_eval_schedules_host_delta8(self._h, K, _np_ptr(delta), _np_ptr(exc_ptr),
-                                                            _np_ptr(exc), _np_ptr(dd), _np_ptr(st), _np_ptr(pk),
-                                                            _np_ptr(lt), _stream_ptr(stream)))
+            fn = self._L.magis_eval_schedules_host_delta4 if d4 else self._L.magis_eval_schedules_host_delta8
+            _check(fn(self._h, K, _np_ptr(delta), _np_ptr(exc_ptr), _np_ptr(exc), _np_ptr(dd), _np_ptr(st),
+                      _np_ptr(pk), _np_ptr(lt), _stream_ptr(stream)))
             return st, pk, lt
         p = as_np(perm, None)
         u16 = p.dtype == np.uint16

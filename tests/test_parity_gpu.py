@@ -355,6 +355,29 @@ def test_device_generator_small_graphs():
 
 
 @pytest.mark.parametrize("cfg", ["c2", "c5"])
+def test_delta4_wire_matches_device_path(cfg):
+    """End-to-end delta4 call (magis_eval_schedules_host_delta4): several
+    chunks, escapes at the row start, out-of-range ids, odd and even rows."""
+    from paper_conf_asplos_chend0zll024_b200 import encode_delta4
+    wl = build_workload(cfg)
+    g = Graph.from_workload(wl, device=0)
+    K = 20011
+    P, D = CandidateGenerator(wl, CandidateSpec(seed=22)).generate(0, K)
+    P[5, 0] = wl.n_total - 1
+    P[6, 3] = -1
+    P[7, 9] = 70000
+    st_d, pk_d, lt_d = gpu_eval(g, P, D[:, :wl.R])
+    st_w, pk_w, lt_w = g.eval_schedules_host(encode_delta4(P), np.ascontiguousarray(D[:, :wl.R]))
+    np.testing.assert_array_equal(st_w, st_d)
+    np.testing.assert_array_equal(pk_w, pk_d)
+    np.testing.assert_array_equal(lt_w, lt_d)
+    assert st_w[6] & 1 and st_w[7] & 1
+    o = OracleGraph.from_workload(wl)
+    idx = np.array([0, 5, 6, 7, 9000, K - 1])
+    assert_parity(st_w[idx], pk_w[idx], lt_w[idx], *o.eval_batch(P[idx], D[idx, :wl.R]))
+
+
+@pytest.mark.parametrize("cfg", ["c2", "c5"])
 def test_delta8_wire_matches_device_path(cfg):
     """End-to-end delta8 call (magis_eval_schedules_host_delta8): several
     chunks, rows with exceptions at the start, out-of-range ids."""
