@@ -302,9 +302,8 @@ __device__ __forceinline__ double candidate_latency(unsigned long long* key, dou
 
 // MODE 0: graph tables and step slots in shared memory; 1: tables read from
 // the global image; 2: tables and step slots in global memory (large graphs);
-// 3: tables read from the global image, free-only step slots (u32) in shared
-// memory, the alloc of each step gathered by the scan from the size table
-// (large graphs whose (alloc, free) slots do not fit).
+// 3: tables read from the global image, one signed delta per step in shared
+// memory (large graphs whose (alloc, free) slots do not fit).
 // TEAMS: independent teams per CTA (each TM main threads + its latency warps,
 // its own per-group state, slots and named barriers; the tables are shared),
 // so one team's barrier waits overlap the other's work.
@@ -322,7 +321,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // per-step slots in shared memory: phase 3 scatters alloc / free into them
     // (smem atomics); in global memory (MODE 2) phase 4 gathers the frees instead
     constexpr bool kScatter = MODE != 2;
-    constexpr bool kFO = MODE == 3;            // free-only slots, alloc gathered in the scan
+    constexpr bool kFO = MODE == 3;            // int32 delta slots: D[i] = alloc(i) - free(i - 1)
     extern __shared__ __align__(128) char sm_all[];
     __shared__ uint64_t mbar;
     __shared__ SlotHdr hdr_t[TEAMS][2];
@@ -400,7 +399,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         uint4* af4 = reinterpret_cast<uint4*>(AF);
         for (int i = tid; i < P * Sl / (kFO ? 4 : 2); i += TM + TL) af4[i] = make_uint4(0u, 0u, 0u, 0u);
     }
-    uint32_t* Fs = reinterpret_cast<uint32_t*>(AF);   // MODE 3: [P][Sl] free per step (size units)
+    // MODE 3: [P][Sl] one signed delta per step in size units, D[i] = alloc(i)
+    // - free(i - 1), so M_i = sum_{j <= i} D[j] and the peak is the max-prefix of D
+    int32_t* Ds = reinterpret_cast<int32_t*>(AF);
     if (tid == 0) {
         for (int b = 0; b < 2; b++) {
             for (int c = 0; c < 4; c++) ctl[b].flags[c] = ctl[b].viol[c] = 0;
@@ -669,8 +670,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const bool act = (o == 0) ? (d == 1) : (d == 2);
                 const uint32_t st = p - 1;
                 if (!act) {
-                    // (MODE 3: no free lands on an absent node's step, its alloc is
-                    // gathered as 0 from pos)
+                    // (MODE 3: the delta slots only receive what phase 3 adds, and
+                    // it adds nothing for an absent node)
                     if constexpr (!kFO) AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
                     pc_[id * P] = 0;
                 } else if (o > 0) {
@@ -724,12 +725,19 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                             const uint32_t pc = PK::get(p, c);
                             if (pc == 0) continue;                  // absent (inactive) in candidate c
                             const uint32_t st = pc - 1;
-                            if constexpr (!kFO) AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)].x = A;
+                            if constexpr (kFO) {
+                                if (A == 0) continue;
+                                atomicAdd(&Ds[c * Sl + (st & (L - 1)) * S + (st >> lgL)], (int32_t)A);
+                                // freed after its last reader's step: the delta of the next step
+                                const uint32_t f1 = PK::get(lst, c);
+                                if (kind != kHdrOut && f1 < (uint32_t)NT)
+                                    atomicAdd(&Ds[c * Sl + (f1 & (L - 1)) * S + (f1 >> lgL)], -(int32_t)A);
+                                continue;
+                            }
+                            AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)].x = A;
                             if (kind != kHdrOut && A != 0) {
                                 const uint32_t fs = PK::get(lst, c) - 1;
-                                const uint32_t fi = c * Sl + (fs & (L - 1)) * S + (fs >> lgL);
-                                if constexpr (kFO) atomicAdd(&Fs[fi], A);
-                                else atomicAdd(&AF[fi].y, A);
+                                atomicAdd(&AF[c * Sl + (fs & (L - 1)) * S + (fs >> lgL)].y, A);
                             }
                         }
                     } else {
@@ -853,32 +861,15 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             constexpr int kUnroll5 = LR > 1 ? LMAX : 8;     // full unroll only with the chunk in registers
             const uint2* afp = AF + cm * Sl + tt;            // step lo + j of candidate cm at afp[j * S]
             if constexpr (kFO) {
-                // one pass: the step's op from the perm (last read of the chunk),
-                // its alloc gathered from the size table (0 if absent), the free
-                // from the slot; with swaps the cost prefix and the events too
-                const uint32_t* fp = Fs + cm * Sl + tt;
-                const int32_t* pp = perm + (grp * P + cm) * (int64_t)NT + lo;
-                double ca = 0.0, cb = 0.0;
+                // memory: max-prefix of the per-step deltas
+                const int32_t* dp = Ds + cm * Sl + tt;          // step lo + j of candidate cm at dp[j * S]
 #pragma unroll kUnroll5
                 for (int j = 0; j < LMAX; j++) {
                     if (j < nst) {
-                        const int32_t v = LMAX <= kRegL ? pr[j % LR] : __ldcs(pp + j);
-                        const bool act = v < n || pos[v * P + cm] != 0;
-                        s1 += act ? __ldg(size_s + v) : 0u;
+                        s1 += dp[j * S];
                         m1 = max(m1, s1);
-                        s1 -= fp[j * S];
-                        if (mysw) {
-                            if ((mbits >> j) & 1ull) {
-                                kout[o] = ((unsigned long long)(lo + j) << 32) | (uint32_t)v;
-                                cout_[o] = ca + cb;
-                                o++;
-                            }
-                            const double c = act ? cost_s[v] : 0.0;     // shared or global table
-                            if (j & 1) cb += c; else ca += c;
-                        }
                     }
                 }
-                cs1 = ca + cb;
             } else
             // memory: alloc = size of the op at each step, free = slot
             if (L == LMAX && nst == LMAX) {
@@ -900,7 +891,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     }
                 }
             }
-            if (!kFO && mysw) {
+            if (mysw) {
                 // swapping candidate: compute-cost prefix (two partial sums
                 // halve the dependent fp64 chain) and the chunk's event steps in
                 // step order; an inactive clone (pos 0) costs nothing

@@ -111,6 +111,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
         uint64_t s = (uint64_t)sg.size[v] / gg;
         for (int32_t e = sg.in_ptr[v]; e < sg.in_ptr[v + 1]; e++) s += (uint64_t)sg.size[sg.in_ent[e].x] / gg;
         if (s > 0xffffffffull) return false;
+        if (free_only && s > 0x7fffffffull) return false;  // tier 2: signed per-step deltas (int32)
     }
     auto virt = [&](int32_t r, int32_t b) -> int32_t {
         for (int32_t j = sg.U_ptr[r]; j < sg.U_ptr[r + 1]; j++)
@@ -222,7 +223,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     // are written there); last: only where phase 4 gathers the frees
     p.off_pos = (uint32_t)o;  o = a16(o + (size_t)(NTX + 1) * P * 2);
     p.off_last = (uint32_t)o; o = a16(o + (gmem_af ? (size_t)NTX * P * 2 : 0));
-    p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * (p.free_only ? 4 : 8)));
+    p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * (p.free_only ? 4 : 8)));   // tier 2: int32 delta
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
     p.nwm = (NT + 31) / 32 + 2;
