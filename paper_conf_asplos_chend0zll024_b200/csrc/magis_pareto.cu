@@ -2,11 +2,15 @@
 // point.
 //
 // Four asynchronous kernels, no host synchronisation:
-//   K1 chunk     : each CTA sorts a chunk of 4096 points by (peak, lat, id) in
-//                  shared memory (bitonic) and keeps the staircase (strictly
-//                  decreasing latency) -- the chunk-local front.
+//   K1 chunk     : each CTA drops the points of its chunk of 1024 that one of
+//                  16 pivots (each warp's minimum by (peak, lat, id) and by
+//                  (lat, peak, id)) dominates -- they cannot be on the front --
+//                  sorts the survivors by (peak, lat, id) in shared memory
+//                  (bitonic, next power of two) and keeps the staircase
+//                  (strictly decreasing latency) -- the chunk-local front.
 //   K2 filter    : a chunk-front point survives iff no other chunk's front has
-//                  a point dominating it (binary search on that staircase).
+//                  a point dominating it (binary search on that staircase; a
+//                  warp per point, a lane per other chunk).
 //   K3 count     : per-chunk exclusive scan of the survivor flags; counts for
 //                  the best-point queries.
 //   K4 scatter   : global rank of a survivor = number of survivors with a
@@ -23,10 +27,11 @@
 
 namespace magis {
 
-constexpr int kCH = 4096;          // points per chunk
-constexpr int kPB = 512;           // threads per K1 / K3 block
-constexpr int kPer = kCH / kPB;    // 8 points per thread
-constexpr int kSmemChunk = kCH * 26;   // pk, lt, ix (8 B each) + ord (2 B)
+constexpr int kCH = 1024;          // points per chunk
+constexpr int kPB = 256;           // threads per K1 / K3 block
+constexpr int kPer = kCH / kPB;    // 4 points per thread
+constexpr int kCHS = kCH + 8;      // + a sentinel point at index kCH (padding of the survivor sort)
+constexpr int kSmemChunk = kCHS * 26;  // pk, lt, ix (8 B each) + ord (2 B)
 
 __device__ unsigned long long g_pareto_dummy[3];
 
@@ -85,11 +90,14 @@ pareto_chunk(int64_t n, const int64_t* __restrict__ peak, const double* __restri
              int64_t id_base, PWs w) {
     extern __shared__ __align__(16) char psm[];
     long long* pk = (long long*)psm;
-    double* lt = (double*)(psm + kCH * 8);
-    long long* ix = (long long*)(psm + kCH * 16);
-    unsigned short* ord = (unsigned short*)(psm + kCH * 24);
+    double* lt = (double*)(psm + kCHS * 8);
+    long long* ix = (long long*)(psm + kCHS * 16);
+    unsigned short* ord = (unsigned short*)(psm + kCHS * 24);
     __shared__ double wmin[kPB / 32];
     __shared__ int wcnt[kPB / 32 + 1];
+    constexpr int kNP = 2 * (kPB / 32);   // pivots
+    __shared__ long long vpk[kNP], vix[kNP];
+    __shared__ double vlt[kNP];
     const int c = blockIdx.x, tid = threadIdx.x;
     const int64_t base = (int64_t)c * kCH;
     for (int j = tid; j < kCH; j += kPB) {
@@ -103,13 +111,80 @@ pareto_chunk(int64_t n, const int64_t* __restrict__ peak, const double* __restri
             lt[j] = INFINITY;
             ix[j] = LLONG_MAX;
         }
-        ord[j] = (unsigned short)j;
+    }
+    if (tid == 0) { pk[kCH] = LLONG_MAX; lt[kCH] = INFINITY; ix[kCH] = LLONG_MAX; }
+    __syncthreads();
+    const int lane = tid & 31, wid = tid >> 5;
+    // pivots: per warp the minimum by (pk, lt, ix) and by (lt, pk, ix)
+    {
+        long long ap = LLONG_MAX, ai = LLONG_MAX, bp = LLONG_MAX, bi = LLONG_MAX;
+        double al = INFINITY, bl = INFINITY;
+        for (int q = 0; q < kPer; q++) {
+            const int j = tid * kPer + q;
+            const long long p = pk[j], i = ix[j];
+            const double l = lt[j];
+            if (key_less(p, l, i, ap, al, ai)) { ap = p; al = l; ai = i; }
+            if (l < bl || (l == bl && (p < bp || (p == bp && i < bi)))) { bp = p; bl = l; bi = i; }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const long long p1 = __shfl_xor_sync(0xffffffffu, ap, o), i1 = __shfl_xor_sync(0xffffffffu, ai, o);
+            const double l1 = __shfl_xor_sync(0xffffffffu, al, o);
+            if (key_less(p1, l1, i1, ap, al, ai)) { ap = p1; al = l1; ai = i1; }
+            const long long p2 = __shfl_xor_sync(0xffffffffu, bp, o), i2 = __shfl_xor_sync(0xffffffffu, bi, o);
+            const double l2 = __shfl_xor_sync(0xffffffffu, bl, o);
+            if (l2 < bl || (l2 == bl && (p2 < bp || (p2 == bp && i2 < bi)))) { bp = p2; bl = l2; bi = i2; }
+        }
+        if (lane == 0) {
+            vpk[2 * wid] = ap; vlt[2 * wid] = al; vix[2 * wid] = ai;
+            vpk[2 * wid + 1] = bp; vlt[2 * wid + 1] = bl; vix[2 * wid + 1] = bi;
+        }
     }
     __syncthreads();
-    // bitonic sort of ord[] by (pk, lt, ix)
-    for (int size = 2; size <= kCH; size <<= 1) {
+    // survivors: valid and dominated by no pivot (a pivot equal in (pk, lt)
+    // with a smaller id also removes it: duplicates keep the smallest id)
+    unsigned smask = 0;
+    int ns = 0;
+    for (int q = 0; q < kPer; q++) {
+        const int j = tid * kPer + q;
+        const long long p = pk[j], i = ix[j];
+        const double l = lt[j];
+        bool sv = p != LLONG_MAX;
+        for (int v = 0; v < kNP && sv; v++) {
+            const long long vp = vpk[v];
+            const double vl = vlt[v];
+            if (vp <= p && vl <= l && (vp < p || vl < l || vix[v] < i)) sv = false;
+        }
+        if (sv) { smask |= 1u << q; ns++; }
+    }
+    {
+        int ki = ns;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, ki, o);
+            if (lane >= o) ki += y;
+        }
+        if (lane == 31) wcnt[wid] = ki;
+        __syncthreads();
+        if (tid == 0) {
+            int acc = 0;
+            for (int q = 0; q < kPB / 32; q++) { const int t2 = wcnt[q]; wcnt[q] = acc; acc += t2; }
+            wcnt[kPB / 32] = acc;
+        }
+        __syncthreads();
+        int r = wcnt[wid] + ki - ns;
+        for (int q = 0; q < kPer; q++)
+            if (smask & (1u << q)) ord[r++] = (unsigned short)(tid * kPer + q);
+    }
+    const int m = wcnt[kPB / 32];
+    int M = 2;
+    while (M < m) M <<= 1;
+    for (int j = m + tid; j < kCH; j += kPB) ord[j] = (unsigned short)kCH;   // sentinels sort last
+    __syncthreads();
+    // bitonic sort of ord[0, M) by (pk, lt, ix)
+    for (int size = 2; size <= M; size <<= 1) {
         for (int stride = size >> 1; stride > 0; stride >>= 1) {
-            for (int t = tid; t < kCH / 2; t += kPB) {
+            for (int t = tid; t < M / 2; t += kPB) {
                 const int i = 2 * t - (t & (stride - 1));
                 const int j = i + stride;
                 const bool asc = ((i & size) == 0);
@@ -121,7 +196,6 @@ pareto_chunk(int64_t n, const int64_t* __restrict__ peak, const double* __restri
         }
     }
     // staircase: keep sorted item j iff valid and lat < min lat of all items before it
-    const int lane = tid & 31, wid = tid >> 5;
     double vals[kPer];
     double tmin = INFINITY;
 #pragma unroll
@@ -201,32 +275,33 @@ __device__ __forceinline__ int first_ge(const int64_t* spk, int cnt, long long p
     return lo;
 }
 
+// one CTA per chunk, one warp per chunk-front point, one lane per other chunk
 __global__ void pareto_filter(int64_t C, PWs w) {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int64_t c = t / kCH;
-    const int i = (int)(t % kCH);
-    if (c >= C) return;
+    const int64_t c = blockIdx.x;
+    const int lane = threadIdx.x & 31, nwarp = blockDim.x >> 5;
     const int cnt = w.cnt[c];
-    if (i >= cnt) return;
-    const int64_t s = c * kCH + i;
-    const long long p = w.spk[s];
-    const double l = w.slt[s];
-    const long long myid = w.sid[s];
-    bool dom = false;
-    for (int64_t c2 = 0; c2 < C && !dom; c2++) {
-        if (c2 == c) continue;
-        const int64_t b2 = c2 * kCH;
-        const int j = last_le(w.spk + b2, w.cnt[c2], p);
-        if (j < 0) continue;
-        const double l2 = w.slt[b2 + j];
-        const long long p2 = w.spk[b2 + j];
-        if (l2 < l) dom = true;
-        else if (l2 == l) {
-            if (p2 < p) dom = true;
-            else if (w.sid[b2 + j] < myid) dom = true;   // exact duplicate: smaller id wins
+    for (int i = threadIdx.x >> 5; i < cnt; i += nwarp) {
+        const int64_t s = c * kCH + i;
+        const long long p = w.spk[s];
+        const double l = w.slt[s];
+        const long long myid = w.sid[s];
+        bool dom = false;
+        for (int64_t c2 = lane; c2 < C && !dom; c2 += 32) {
+            if (c2 == c) continue;
+            const int64_t b2 = c2 * kCH;
+            const int j = last_le(w.spk + b2, w.cnt[c2], p);
+            if (j < 0) continue;
+            const double l2 = w.slt[b2 + j];
+            const long long p2 = w.spk[b2 + j];
+            if (l2 < l) dom = true;
+            else if (l2 == l) {
+                if (p2 < p) dom = true;
+                else if (w.sid[b2 + j] < myid) dom = true;   // exact duplicate: smaller id wins
+            }
         }
+        dom = __any_sync(0xffffffffu, dom);
+        if (lane == 0) w.flag[s] = dom ? 0 : 1;
     }
-    w.flag[s] = dom ? 0 : 1;
 }
 
 __global__ void __launch_bounds__(kPB)
@@ -280,38 +355,43 @@ pareto_count(PWs w, int64_t mem_limit, double lat_limit) {
     if (lane == 0 && cl) atomicAdd(&w.ctr[1], (unsigned long long)cl);
 }
 
+// one CTA per chunk, one warp per surviving point, one lane per chunk of the rank sum
 __global__ void pareto_scatter(int64_t C, PWs w, int64_t cap, int64_t* front_id,
                                int64_t* front_peak, double* front_lat, int64_t* front_n,
                                int64_t mem_limit, double lat_limit, int64_t* best) {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t c = blockIdx.x;
+    const int lane = threadIdx.x & 31, nwarp = blockDim.x >> 5;
     const int64_t nf = (int64_t)w.ctr[2];              // total front size (pareto_count)
-    if (t == 0) *front_n = nf;
-    const int64_t c = t / kCH;
-    const int i = (int)(t % kCH);
-    if (c >= C || i >= w.cnt[c]) return;
-    const int64_t s = c * kCH + i;
-    if (!w.flag[s]) return;
-    const long long p = w.spk[s];
-    int64_t rank = 0;
-    for (int64_t c2 = 0; c2 < C; c2++) {
-        const int64_t b2 = c2 * kCH;
-        const int cnt2 = w.cnt[c2];
-        const int j = (c2 == c) ? i : first_ge(w.spk + b2, cnt2, p);
-        rank += (j < cnt2) ? w.pref[b2 + j] : w.tot[c2];
-    }
-    if (rank < cap) {
-        front_id[rank] = w.sid[s];
-        front_peak[rank] = p;
-        front_lat[rank] = w.slt[s];
-    }
-    if (best) {
-        if (mem_limit >= 0) {
-            const int64_t cm = (int64_t)w.ctr[0];
-            if (rank == (cm > 0 ? cm - 1 : 0)) best[0] = w.sid[s];
+    if (c == 0 && threadIdx.x == 0) *front_n = nf;
+    const int cnt = w.cnt[c];
+    for (int i = threadIdx.x >> 5; i < cnt; i += nwarp) {
+        const int64_t s = c * kCH + i;
+        if (!w.flag[s]) continue;
+        const long long p = w.spk[s];
+        long long rank = 0;
+        for (int64_t c2 = lane; c2 < C; c2 += 32) {
+            const int64_t b2 = c2 * kCH;
+            const int cnt2 = w.cnt[c2];
+            const int j = (c2 == c) ? i : first_ge(w.spk + b2, cnt2, p);
+            rank += (j < cnt2) ? w.pref[b2 + j] : w.tot[c2];
         }
-        if (lat_limit >= 0.0) {
-            const int64_t cl = (int64_t)w.ctr[1];
-            if (rank == (cl < nf ? cl : nf - 1)) best[1] = w.sid[s];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) rank += __shfl_xor_sync(0xffffffffu, rank, o);
+        if (lane != 0) continue;
+        if (rank < cap) {
+            front_id[rank] = w.sid[s];
+            front_peak[rank] = p;
+            front_lat[rank] = w.slt[s];
+        }
+        if (best) {
+            if (mem_limit >= 0) {
+                const int64_t cm = (int64_t)w.ctr[0];
+                if (rank == (cm > 0 ? cm - 1 : 0)) best[0] = w.sid[s];
+            }
+            if (lat_limit >= 0.0) {
+                const int64_t cl = (int64_t)w.ctr[1];
+                if (rank == (cl < nf ? cl : nf - 1)) best[1] = w.sid[s];
+            }
         }
     }
 }
@@ -356,11 +436,9 @@ cudaError_t pareto_launch(int64_t n, const int64_t* peak, const double* lat,
     }
     pareto_init<<<1, 1, 0, stream>>>(w, front_n, best);
     pareto_chunk<<<(unsigned)C, kPB, kSmemChunk, stream>>>(n, peak, lat, status, id, id_base, w);
-    const int64_t threads = C * kCH;
-    const unsigned blocks = (unsigned)((threads + 255) / 256);
-    pareto_filter<<<blocks, 256, 0, stream>>>(C, w);
+    pareto_filter<<<(unsigned)C, 256, 0, stream>>>(C, w);
     pareto_count<<<(unsigned)C, kPB, 0, stream>>>(w, mem_limit, lat_limit);
-    pareto_scatter<<<blocks, 256, 0, stream>>>(C, w, cap, front_id, front_peak, front_lat, front_n,
+    pareto_scatter<<<(unsigned)C, 256, 0, stream>>>(C, w, cap, front_id, front_peak, front_lat, front_n,
                                                mem_limit, lat_limit, best);
     if (cap > 0)
         pareto_pad<<<(unsigned)std::min<int64_t>((cap + 255) / 256, 1024), 256, 0, stream>>>(
