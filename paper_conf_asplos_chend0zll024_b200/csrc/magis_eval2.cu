@@ -670,9 +670,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const bool act = (o == 0) ? (d == 1) : (d == 2);
                 const uint32_t st = p - 1;
                 if (!act) {
-                    // (MODE 3: the delta slots only receive what phase 3 adds, and
-                    // it adds nothing for an absent node)
-                    if constexpr (!kFO) AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
+                    // slots in shared memory start the group at 0 and phase 3 adds
+                    // nothing at an absent node's step (no alloc, and no tensor has
+                    // its last reader there); the global slots (MODE 2) are not cleared
+                    if constexpr (!kScatter) AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
                     pc_[id * P] = 0;
                 } else if (o > 0) {
                     atomicOr(em + (st >> 5), 1u << (st & 31));
