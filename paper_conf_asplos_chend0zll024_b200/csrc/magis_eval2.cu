@@ -364,6 +364,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const uint32_t* wtab = (const uint32_t*)(sb + pl.off_wtab);   // [WM][4]: consumer rows, input rows
     const uint2* crow = (const uint2*)(sb + pl.off_crow);
     const uint32_t* chdr = (const uint32_t*)(sb + pl.off_chdr);
+    const uint32_t* csize = (const uint32_t*)(sb + pl.off_csize);   // size units of each header, row order
     const uint16_t* cent = (const uint16_t*)(sb + pl.off_cent);
     const uint2* frow = (const uint2*)(sb + pl.off_frow);
     const uint32_t* fhdr = (const uint32_t*)(sb + pl.off_fhdr);
@@ -720,7 +721,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         // (a tensor without readers after its own step; graph
                         // outputs live to the end): scattered straight into the
                         // per-step slots, no second pass over the input rows
-                        const uint32_t A = size_s[id];
+                        const uint32_t A = csize[r * 32 + lane];   // conflict-free (row order)
 #pragma unroll
                         for (int c = 0; c < P; c++) {
                             const uint32_t pc = PK::get(p, c);

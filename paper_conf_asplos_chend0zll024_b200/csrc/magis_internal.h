@@ -79,6 +79,7 @@ struct Plan2 {
     uint32_t static_bytes;   // bulk-staged prefix (graph rows + size units)
     uint32_t off_wtab;       // [WM][4]: consumer rows [b, e), input rows [b, e)
     uint32_t off_crow, off_chdr, off_cent;                  // consumer rows: (offset, degree), headers, edges
+    uint32_t off_csize;                                     // consumer rows: size units per header (row order)
     uint32_t off_frow, off_fhdr, off_fent;                  // input rows
     uint32_t off_size;       // [NTX] size units
     uint32_t off_rtab;       // [R] double2 (cost(t_r), swap transfer time)

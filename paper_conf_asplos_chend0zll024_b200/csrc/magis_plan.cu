@@ -189,6 +189,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     p.off_wtab = (uint32_t)o;  o = a16(o + wtab.size() * 4);
     p.off_crow = (uint32_t)o;  o = a16(o + cr.row.size() * 4);
     p.off_chdr = (uint32_t)o;  o = a16(o + cr.hdr.size() * 4);
+    p.off_csize = (uint32_t)o; o = a16(o + cr.hdr.size() * 4);   // size units of each header, row order
     p.off_cent = (uint32_t)o;  o = a16(o + cr.ent.size() * 2);
     p.off_frow = (uint32_t)o;  o = a16(o + fr.row.size() * 4);
     p.off_fhdr = (uint32_t)o;  o = a16(o + fr.hdr.size() * 4);
@@ -262,6 +263,12 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     put(p.off_wtab, wtab.data(), wtab.size() * 4);
     put(p.off_crow, cr.row.data(), cr.row.size() * 4);
     put(p.off_chdr, cr.hdr.data(), cr.hdr.size() * 4);
+    {
+        std::vector<uint32_t> cs(cr.hdr.size(), 0);
+        for (size_t i = 0; i < cr.node.size(); i++)
+            if (cr.node[i] >= 0) cs[i] = size_u[cr.node[i]];
+        put(p.off_csize, cs.data(), cs.size() * 4);
+    }
     put(p.off_cent, cr.ent.data(), cr.ent.size() * 2);
     put(p.off_frow, fr.row.data(), fr.row.size() * 4);
     put(p.off_fhdr, fr.hdr.data(), fr.hdr.size() * 4);
