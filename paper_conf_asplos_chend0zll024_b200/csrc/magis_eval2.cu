@@ -354,7 +354,10 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     for (int i = 0; i < 16; i++) pt[i] = 0;
     long long plast = clock64();
 #define PROF_MARK(k) do { if (prof) { const long long _t = clock64(); pt[k] += _t - plast; plast = _t; } } while (0)
-    const int32_t L = pl.L, S = pl.S, Sl = pl.L * pl.S, lgL = pl.lgL;
+    // per-step slots of a candidate: step st at st + (st >> lgL) (one pad word per
+    // scan chunk of L steps), so thread tt's chunk [tt L, tt L + L) is contiguous
+    // at tt (L + 1) and the lanes of a warp read it conflict-free (odd stride)
+    const int32_t L = pl.L, S = pl.S, Sl = ((pl.L + 1) * pl.S + 3) & ~3, lgL = pl.lgL;
 
     // graph tables: staged into shared memory once per CTA (bulk copy), or
     // read in place from the global image when they do not fit
@@ -674,7 +677,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     // slots in shared memory start the group at 0 and phase 3 adds
                     // nothing at an absent node's step (no alloc, and no tensor has
                     // its last reader there); the global slots (MODE 2) are not cleared
-                    if constexpr (!kScatter) AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(0u, 0u);
+                    if constexpr (!kScatter) AF[c * Sl + st + (st >> lgL)] = make_uint2(0u, 0u);
                     pc_[id * P] = 0;
                 } else if (o > 0) {
                     atomicOr(em + (st >> 5), 1u << (st & 31));
@@ -729,17 +732,17 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                             const uint32_t st = pc - 1;
                             if constexpr (kFO) {
                                 if (A == 0) continue;
-                                atomicAdd(&Ds[c * Sl + (st & (L - 1)) * S + (st >> lgL)], (int32_t)A);
+                                atomicAdd(&Ds[c * Sl + st + (st >> lgL)], (int32_t)A);
                                 // freed after its last reader's step: the delta of the next step
                                 const uint32_t f1 = PK::get(lst, c);
                                 if (kind != kHdrOut && f1 < (uint32_t)NT)
-                                    atomicAdd(&Ds[c * Sl + (f1 & (L - 1)) * S + (f1 >> lgL)], -(int32_t)A);
+                                    atomicAdd(&Ds[c * Sl + f1 + (f1 >> lgL)], -(int32_t)A);
                                 continue;
                             }
-                            AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)].x = A;
+                            AF[c * Sl + st + (st >> lgL)].x = A;
                             if (kind != kHdrOut && A != 0) {
                                 const uint32_t fs = PK::get(lst, c) - 1;
-                                atomicAdd(&AF[c * Sl + (fs & (L - 1)) * S + (fs >> lgL)].y, A);
+                                atomicAdd(&AF[c * Sl + fs + (fs >> lgL)].y, A);
                             }
                         }
                     } else {
@@ -821,7 +824,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         const uint32_t pc = PK::get(p, c);
                         if (pc == 0 || !((okm >> c) & 1u)) continue;
                         const uint32_t st = pc - 1;
-                        AF[c * Sl + (st & (L - 1)) * S + (st >> lgL)] = make_uint2(A, fr[c]);
+                        AF[c * Sl + st + (st >> lgL)] = make_uint2(A, fr[c]);
                     }
                 }
             }
@@ -861,14 +864,14 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             int o = wpre + evx;
             const int o0 = o;
             constexpr int kUnroll5 = LR > 1 ? LMAX : 8;     // full unroll only with the chunk in registers
-            const uint2* afp = AF + cm * Sl + tt;            // step lo + j of candidate cm at afp[j * S]
+            const uint2* afp = AF + cm * Sl + tt * (L + 1);  // step lo + j of candidate cm at afp[j]
             if constexpr (kFO) {
                 // memory: max-prefix of the per-step deltas
-                const int32_t* dp = Ds + cm * Sl + tt;          // step lo + j of candidate cm at dp[j * S]
+                const int32_t* dp = Ds + cm * Sl + tt * (L + 1);   // step lo + j of candidate cm at dp[j]
 #pragma unroll kUnroll5
                 for (int j = 0; j < LMAX; j++) {
                     if (j < nst) {
-                        s1 += dp[j * S];
+                        s1 += dp[j];
                         m1 = max(m1, s1);
                     }
                 }
@@ -877,7 +880,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             if (L == LMAX && nst == LMAX) {
 #pragma unroll
                 for (int j = 0; j < LMAX; j++) {
-                    const uint2 af = afp[j * S];
+                    const uint2 af = afp[j];
                     s1 += af.x;
                     m1 = max(m1, s1);
                     s1 -= af.y;
@@ -886,7 +889,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 #pragma unroll kUnroll5
                 for (int j = 0; j < LMAX; j++) {
                     if (j < nst) {
-                        const uint2 af = afp[j * S];
+                        const uint2 af = afp[j];
                         s1 += af.x;
                         m1 = max(m1, s1);
                         s1 -= af.y;

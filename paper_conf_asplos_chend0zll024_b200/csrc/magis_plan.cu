@@ -210,7 +210,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     p.gmem_af = gmem_af ? 1 : 0;
     p.free_only = (free_only && !gmem_af) ? 1 : 0;
     if (p.free_only && !gmem_static) return false;      // MODE 3 reads the tables from the global image
-    const size_t Sl = (size_t)p.L * p.S;
+    const size_t Sl = ((size_t)(p.L + 1) * p.S + 3) & ~(size_t)3;   // padded per-candidate slots (magis_eval2.cu)
     p.af_bytes = (uint64_t)((P * Sl * 8 + 255) / 256 * 256);
     const size_t static_end = o;
     // tables read from the global image: the cost table (the swap scan's
