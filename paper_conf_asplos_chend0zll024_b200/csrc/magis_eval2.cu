@@ -920,19 +920,49 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 // halve the dependent fp64 chain) and the chunk's event steps in
                 // step order; an inactive clone (pos 0) costs nothing
                 double ca = 0.0, cb = 0.0;
+                if constexpr (LMAX <= kRegL) {
 #pragma unroll kUnroll5
-                for (int j = 0; j < LMAX; j++) {
-                    if (j < nst) {
-                        const int32_t v = LMAX <= kRegL ? pr[j % LR]
-                                                     : __ldg(perm + (grp * P + cm) * (int64_t)NT + lo + j);
-                        if ((mbits >> j) & 1ull) {
-                            kout[o] = ((unsigned long long)(lo + j) << 32) | (uint32_t)v;
-                            cout_[o] = ca + cb;
-                            o++;
+                    for (int j = 0; j < LMAX; j++) {
+                        if (j < nst) {
+                            const int32_t v = pr[j % LR];
+                            if ((mbits >> j) & 1ull) {
+                                kout[o] = ((unsigned long long)(lo + j) << 32) | (uint32_t)v;
+                                cout_[o] = ca + cb;
+                                o++;
+                            }
+                            double c = cost_s[v];
+                            if (v >= n && pos[v * P + cm] == 0) c = 0.0;
+                            if (j & 1) cb += c; else ca += c;
                         }
-                        double c = cost_s[v];
-                        if (v >= n && pos[v * P + cm] == 0) c = 0.0;
-                        if (j & 1) cb += c; else ca += c;
+                    }
+                } else {
+                    // perm chunk re-read from global: batches of 8 steps with the perm
+                    // and cost loads issued ahead of the event stores (which the
+                    // compiler cannot move loads across)
+                    const int32_t* pp = perm + (grp * P + cm) * (int64_t)NT + lo;
+                    for (int jb = 0; jb < LMAX; jb += 8) {
+                        if (jb >= nst) break;
+                        int32_t vv[8];
+                        double cv[8];
+#pragma unroll
+                        for (int u = 0; u < 8; u++) vv[u] = jb + u < nst ? __ldg(pp + jb + u) : 0;
+#pragma unroll
+                        for (int u = 0; u < 8; u++) cv[u] = jb + u < nst ? cost_s[vv[u]] : 0.0;
+#pragma unroll
+                        for (int u = 0; u < 8; u++) {
+                            const int j = jb + u;
+                            if (j < nst) {
+                                const int32_t v = vv[u];
+                                if ((mbits >> j) & 1ull) {
+                                    kout[o] = ((unsigned long long)(lo + j) << 32) | (uint32_t)v;
+                                    cout_[o] = ca + cb;
+                                    o++;
+                                }
+                                double c = cv[u];
+                                if (v >= n && pos[v * P + cm] == 0) c = 0.0;
+                                if (u & 1) cb += c; else ca += c;
+                            }
+                        }
                     }
                 }
                 cs1 = ca + cb;
