@@ -616,18 +616,19 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     }
                 }
             } else {
+                // (default caching: the swap cost loop of phase 5 reads the chunk again)
                 const int32_t* Pp = perm + (grp * P + cm) * (int64_t)NT + lo;
 #pragma unroll
                 for (int j = 0; j < LMAX; j += 4) {
                     if (vc && j < L && lo + j < NT) {
                         int4 v = make_int4(-1, -1, -1, -1);
                         if (vec4) {
-                            v = __ldcs(reinterpret_cast<const int4*>(Pp + j));
+                            v = __ldg(reinterpret_cast<const int4*>(Pp + j));
                         } else {
-                            v.x = __ldcs(Pp + j);
-                            if (lo + j + 1 < NT) v.y = __ldcs(Pp + j + 1);
-                            if (lo + j + 2 < NT) v.z = __ldcs(Pp + j + 2);
-                            if (lo + j + 3 < NT) v.w = __ldcs(Pp + j + 3);
+                            v.x = __ldg(Pp + j);
+                            if (lo + j + 1 < NT) v.y = __ldg(Pp + j + 1);
+                            if (lo + j + 2 < NT) v.z = __ldg(Pp + j + 2);
+                            if (lo + j + 3 < NT) v.w = __ldg(Pp + j + 3);
                         }
                         const uint32_t i0 = (uint32_t)(lo + j);
                         if ((uint32_t)v.x < (uint32_t)NT) pos[v.x * P + cm] = (uint16_t)(i0 + 1); else bad = 1;
@@ -945,7 +946,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         int32_t vv[8];
                         double cv[8];
 #pragma unroll
-                        for (int u = 0; u < 8; u++) vv[u] = jb + u < nst ? __ldg(pp + jb + u) : 0;
+                        for (int u = 0; u < 8; u++) vv[u] = jb + u < nst ? __ldcs(pp + jb + u) : 0;   // last read
 #pragma unroll
                         for (int u = 0; u < 8; u++) cv[u] = jb + u < nst ? cost_s[vv[u]] : 0.0;
 #pragma unroll
