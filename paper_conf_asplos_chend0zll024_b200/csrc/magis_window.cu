@@ -425,7 +425,14 @@ cudaError_t base_launch(const DevGraph& g, const BaseDev& b, const int32_t* perm
 int window_grid(int device) {
     cudaDeviceProp p;
     if (cudaGetDeviceProperties(&p, device) != cudaSuccess) return 148 * 4;
-    return p.multiProcessorCount * 4;
+    // as many resident CTAs as registers / shared memory allow: the warps are
+    // latency bound (global gathers of the base tables), so occupancy pays
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, window_kernel, kWarpsW * 32, 0) != cudaSuccess || occ < 1) {
+        cudaGetLastError();
+        occ = 4;
+    }
+    return p.multiProcessorCount * occ;
 }
 
 cudaError_t window_launch(const DevGraph& g, const BaseDev& b, int grid, double* endb_ws, int64_t K,
