@@ -186,18 +186,19 @@ struct Ctl {
 
 constexpr long long kNegInf = -(1ll << 62);
 
-// mark bits of steps [lo, lo + L) (L a power of two, lo a multiple of L)
-__device__ __forceinline__ unsigned long long mark_bits(const uint32_t* m, int32_t lo, int32_t L) {
-    if (L >= 64) return (unsigned long long)m[lo >> 5] | ((unsigned long long)m[(lo >> 5) + 1] << 32);
-    const uint32_t w = m[lo >> 5] >> (lo & 31);
-    return L == 32 ? w : (w & ((1u << L) - 1u));
+// mark bits of steps [lo, lo + 64) (the caller masks to its chunk length)
+__device__ __forceinline__ unsigned long long mark_bits(const uint32_t* m, int32_t lo) {
+    const int32_t w = lo >> 5, sh = lo & 31;
+    const unsigned long long a = (unsigned long long)m[w] | ((unsigned long long)m[w + 1] << 32);
+    return sh ? (a >> sh) | ((unsigned long long)m[w + 2] << (64 - sh)) : a;
 }
 
 struct WalkTabs {
     const uint2* ninfo;
     const uint16_t* lul;
     const double2* rtab;
-    int32_t n, lgL;
+    int32_t n;
+    uint32_t Lm;          // ceil(2^32 / L): step / L = umulhi(step, Lm) (exact for steps < 2^16)
 };
 
 // The event steps of a swapping candidate are resolved by the whole latency
@@ -233,7 +234,7 @@ __device__ __forceinline__ void resolve_event(unsigned long long& kslot, double&
         islot = pk | ((unsigned long long)nw << 48);
         kslot = (unsigned long long)(prod ? rt : 0u) | ((unsigned long long)m << 16) |
                 ((unsigned long long)x.y << 47);
-        cslot += woff[(stp >> t.lgL) >> 5];
+        cslot += woff[__umulhi((uint32_t)stp, t.Lm) >> 5];
     } else {
         const uint32_t q = (uint32_t)(w - t.n), r = q / 3, o = q - 3 * r;   // o: 1 Store, 2 Load
         islot = (unsigned long long)o << 62;
@@ -354,10 +355,12 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     for (int i = 0; i < 16; i++) pt[i] = 0;
     long long plast = clock64();
 #define PROF_MARK(k) do { if (prof) { const long long _t = clock64(); pt[k] += _t - plast; plast = _t; } } while (0)
-    // per-step slots of a candidate: step st at st + (st >> lgL) (one pad word per
-    // scan chunk of L steps), so thread tt's chunk [tt L, tt L + L) is contiguous
-    // at tt (L + 1) and the lanes of a warp read it conflict-free (odd stride)
-    const int32_t L = pl.L, S = pl.S, Sl = ((pl.L + 1) * pl.S + 3) & ~3, lgL = pl.lgL;
+    // per-step slots of a candidate: step st at st + st / L (one pad word per scan
+    // chunk of L steps, L a multiple of 4), so thread tt's chunk [tt L, tt L + L)
+    // is contiguous at tt (L + 1) and the lanes of a warp read it conflict-free
+    // (odd stride); st / L = umulhi(st, Lm)
+    const int32_t L = pl.L, S = pl.S, Sl = ((pl.L + 1) * pl.S + 3) & ~3;
+    const uint32_t Lm = pl.Lm;
 
     // graph tables: staged into shared memory once per CTA (bulk copy), or
     // read in place from the global image when they do not fit
@@ -423,7 +426,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         //      warp WM + c walks the event steps of candidate c of each group
         const int c = warp - WM;
         double* endb = (double*)(sm + pl.off_end) + (size_t)c * 3 * R;
-        const WalkTabs wt{ninfo, lul, rtab, n, lgL};
+        const WalkTabs wt{ninfo, lul, rtab, n, Lm};
         for (int gi = 0; gi < ncta; gi++) {
             const int slot = gi & 1;
             PROF_MARK(13);
@@ -678,7 +681,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     // slots in shared memory start the group at 0 and phase 3 adds
                     // nothing at an absent node's step (no alloc, and no tensor has
                     // its last reader there); the global slots (MODE 2) are not cleared
-                    if constexpr (!kScatter) AF[c * Sl + st + (st >> lgL)] = make_uint2(0u, 0u);
+                    if constexpr (!kScatter) AF[c * Sl + st + __umulhi(st, Lm)] = make_uint2(0u, 0u);
                     pc_[id * P] = 0;
                 } else if (o > 0) {
                     atomicOr(em + (st >> 5), 1u << (st & 31));
@@ -752,17 +755,17 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                             const uint32_t st = pc - 1;
                             if constexpr (kFO) {
                                 if (A == 0) continue;
-                                atomicAdd(&Ds[c * Sl + st + (st >> lgL)], (int32_t)A);
+                                atomicAdd(&Ds[c * Sl + st + __umulhi(st, Lm)], (int32_t)A);
                                 // freed after its last reader's step: the delta of the next step
                                 const uint32_t f1 = PK::get(lst, c);
                                 if (kind != kHdrOut && f1 < (uint32_t)NT)
-                                    atomicAdd(&Ds[c * Sl + f1 + (f1 >> lgL)], -(int32_t)A);
+                                    atomicAdd(&Ds[c * Sl + f1 + __umulhi(f1, Lm)], -(int32_t)A);
                                 continue;
                             }
-                            AF[c * Sl + st + (st >> lgL)].x = A;
+                            AF[c * Sl + st + __umulhi(st, Lm)].x = A;
                             if (kind != kHdrOut && A != 0) {
                                 const uint32_t fs = PK::get(lst, c) - 1;
-                                atomicAdd(&AF[c * Sl + fs + (fs >> lgL)].y, A);
+                                atomicAdd(&AF[c * Sl + fs + __umulhi(fs, Lm)].y, A);
                             }
                         }
                     } else {
@@ -796,7 +799,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         // event steps of this thread's chunk and their order within the warp
         const int32_t nst = ((okm >> cm) & 1u) ? max(0, min(L, NT - lo)) : 0;   // steps of this chunk
         const unsigned long long mbits =
-            (mysw && nst > 0) ? mark_bits(evm + cm * nwm, lo, L) & (~0ull >> (64 - nst)) : 0ull;
+            (mysw && nst > 0) ? mark_bits(evm + cm * nwm, lo) & (~0ull >> (64 - nst)) : 0ull;
         int evx = __popcll(mbits);
         {
             int inc = evx;
@@ -844,7 +847,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                         const uint32_t pc = PK::get(p, c);
                         if (pc == 0 || !((okm >> c) & 1u)) continue;
                         const uint32_t st = pc - 1;
-                        AF[c * Sl + st + (st >> lgL)] = make_uint2(A, fr[c]);
+                        AF[c * Sl + st + __umulhi(st, Lm)] = make_uint2(A, fr[c]);
                     }
                 }
             }
@@ -1048,7 +1051,11 @@ static const void* kernel_ptr(int lmax) {
     if constexpr (MODE == 0) {
         if (lmax <= 4) return (const void*)eval2_kernel<P, 4, 0, TEAMS>;
         if (lmax <= 8) return (const void*)eval2_kernel<P, 8, 0, TEAMS>;
+        if (lmax <= 12) return (const void*)eval2_kernel<P, 12, 0, TEAMS>;
         if (lmax <= 16) return (const void*)eval2_kernel<P, 16, 0, TEAMS>;
+        if (lmax <= 20) return (const void*)eval2_kernel<P, 20, 0, TEAMS>;
+        if (lmax <= 24) return (const void*)eval2_kernel<P, 24, 0, TEAMS>;
+        if (lmax <= 28) return (const void*)eval2_kernel<P, 28, 0, TEAMS>;
         return (const void*)eval2_kernel<P, 32, 0, TEAMS>;
     } else {
         if (lmax <= 16) return (const void*)eval2_kernel<P, 16, MODE, 1>;

@@ -75,7 +75,7 @@ struct Plan2 {
     int32_t L, S;         // scan chunk length / slot stride (L * S >= NT, S <= kMainThreads2)
     int64_t unit;         // bytes per size unit (gcd of sizes)
     int32_t max_events;   // 3R + |U|
-    int32_t lgL;          // L = 1 << lgL
+    uint32_t Lm;          // ceil(2^32 / L) (L a multiple of 4): st / L = umulhi(st, Lm)
     uint32_t static_bytes;   // bulk-staged prefix (graph rows + size units)
     uint32_t off_wtab;       // [WM][4]: consumer rows [b, e), input rows [b, e)
     uint32_t off_crow, off_chdr, off_cent;                  // consumer rows: (offset, degree), headers, edges

@@ -175,12 +175,13 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     p.R = R;
     p.nU = nU;
     {
+        // scan chunk: the fewest steps per thread, a multiple of 4 (int4 perm
+        // loads, odd padded slot stride); the kernel divides by L with a magic
         const int32_t tpc = TMt / P;                    // threads per candidate in the scan
-        int32_t Lmin = std::max(4, (NT + tpc - 1) / tpc), lg = 0;
-        while ((1 << lg) < Lmin) lg++;
-        if (lg > 6) return false;                       // LMAX <= 64 steps per thread
-        p.lgL = lg;
-        p.L = 1 << lg;
+        const int32_t Lmin = std::max(4, (NT + tpc - 1) / tpc);
+        p.L = (Lmin + 3) & ~3;
+        if (p.L > 64) return false;                     // LMAX <= 64 steps per thread
+        p.Lm = (uint32_t)((((uint64_t)1 << 32) + (uint64_t)p.L - 1) / (uint64_t)p.L);
         p.S = (NT + p.L - 1) / p.L;
     }
     p.unit = (int64_t)gg;
@@ -227,7 +228,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * (p.free_only ? 4 : 8)));   // tier 2: int32 delta
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
-    p.nwm = (NT + 31) / 32 + 2;
+    p.nwm = (NT + 31) / 32 + 3;                         // mark_bits reads up to 2 words past a chunk start
     p.off_evm = (uint32_t)o;  o = a16(o + (size_t)P * p.nwm * 4);
     p.off_sdec = (uint32_t)o; o = a16(o + (size_t)2 * P * ((std::max(R, 1) + 15) & ~15));
     p.off_ev = (uint32_t)o;
