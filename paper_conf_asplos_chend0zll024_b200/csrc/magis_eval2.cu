@@ -16,9 +16,9 @@
 //    inner loops carry no decision tests;
 //  * positions are stored +1 (0 = absent / inactive), so validity is one
 //    running min of (q - 1) per node: a violation iff min < pos (unsigned);
-//  * alloc/free amounts land in per-step slots (u32 size units) in a
-//    transposed layout, so the scan's per-thread contiguous chunks read
-//    conflict-free;
+//  * alloc/free amounts land in per-step slots (u32 size units; tier 2: one
+//    signed delta) laid out st + st / L, one pad word per scan chunk, so the
+//    scan's per-thread contiguous chunks read conflict-free (odd stride);
 //  * swap latency (the three in-order queues of reading P7): the steps that
 //    raise swap events are marked in a per-candidate bitmap while the gates
 //    are resolved (phase 2); the scan threads emit their marked steps with the
