@@ -1059,7 +1059,10 @@ static const void* kernel_ptr(int lmax) {
         return (const void*)eval2_kernel<P, 32, 0, TEAMS>;
     } else {
         if (lmax <= 16) return (const void*)eval2_kernel<P, 16, MODE, 1>;
+        if (lmax <= 24) return (const void*)eval2_kernel<P, 24, MODE, 1>;
+        if (lmax <= 28) return (const void*)eval2_kernel<P, 28, MODE, 1>;
         if (lmax <= 32) return (const void*)eval2_kernel<P, 32, MODE, 1>;
+        if (lmax <= 48) return (const void*)eval2_kernel<P, 48, MODE, 1>;
         return (const void*)eval2_kernel<P, 64, MODE, 1>;
     }
 }
