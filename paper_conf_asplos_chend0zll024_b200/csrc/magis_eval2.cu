@@ -322,7 +322,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // per-step slots in shared memory: phase 3 scatters alloc / free into them
     // (smem atomics); in global memory (MODE 2) phase 4 gathers the frees instead
     constexpr bool kScatter = MODE != 2;
-    constexpr bool kFO = MODE == 3;            // int32 delta slots: D[i] = alloc(i) - free(i - 1)
+    constexpr bool kFO = MODE == 3;            // (tier 2) int32 delta slots: D[i] = alloc(i) - free(i - 1)
     extern __shared__ __align__(128) char sm_all[];
     __shared__ uint64_t mbar;
     __shared__ SlotHdr hdr_t[TEAMS][2];
@@ -1074,7 +1074,7 @@ static const void* kernel_mode(const Plan2& pl) {
 }
 
 static const void* kernel_for(const Plan2& pl) {
-    const int mode = pl.gmem_af ? 2 : pl.free_only ? 3 : (pl.gmem_static ? 1 : 0);
+    const int mode = pl.gmem_af ? 2 : pl.delta_slots ? 3 : (pl.gmem_static ? 1 : 0);
     if (mode == 0) return pl.teams == 2 ? kernel_mode<0, 2>(pl) : kernel_mode<0, 1>(pl);
     return mode == 1 ? kernel_mode<1, 1>(pl) : mode == 3 ? kernel_mode<3, 1>(pl) : kernel_mode<2, 1>(pl);
 }

@@ -477,8 +477,9 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
             int bestP = 0, bestOcc = 0, bestT = 1;
             Plan2 bestPl{};
             std::vector<char> bestImg;
-            // tier 2 = tables in global, free-only slots in shared memory (the
-            // scan gathers the allocs); tier 3 = tables and slots in global
+            // tier 2 = tables in global, one signed delta per step in shared
+            // memory (alloc - free of the previous step); tier 3 = tables and
+            // slots in global
             const char* tierf = std::getenv("MAGIS_TIER");
             for (int tier = 0; tier < 4 && bestP == 0; tier++) {
                 if (tierf && std::atoi(tierf) != tier) continue;

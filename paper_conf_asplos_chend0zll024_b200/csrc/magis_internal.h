@@ -101,7 +101,7 @@ struct Plan2 {
     int32_t gmem_static;  // graph tables read from the global image instead of shared memory
     int32_t gmem_af;      // per-step slots in a per-CTA global slice (af_bytes each)
     int32_t cost_sm;      // tables in global, but the cost table staged at shared offset 0
-    int32_t free_only;    // per-step slots hold only the free (u32, shared memory); the scan gathers the alloc
+    int32_t delta_slots;  // tier 2: one signed int32 per step in shared memory, alloc(i) - free(i - 1)
     uint32_t state_base;  // offset of the per-candidate state in shared memory
     uint64_t af_bytes;
     int32_t prof;         // MAGIS_PROFILE: accumulate per-phase cycles
@@ -195,7 +195,7 @@ struct SuperGraphHost {
 // Build the variant-2 plan and its static shared-memory image for a given P.
 // Returns false if the graph does not fit (ids >= 65535, sizes beyond u32
 // units, or shared memory).
-bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, bool free_only,
+bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, bool delta_slots,
                  size_t smem_cap, Plan2* plan,
                  std::vector<char>* image);
 cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,

@@ -96,7 +96,7 @@ Rows make_rows(const std::vector<std::vector<uint32_t>>& lists, const std::vecto
 }
 }  // namespace
 
-bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, bool free_only,
+bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, bool delta_slots,
                  size_t smem_cap,
                  Plan2* pl, std::vector<char>* img) {
     const int32_t NT = sg.NT, n = sg.n, R = sg.R;
@@ -111,7 +111,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
         uint64_t s = (uint64_t)sg.size[v] / gg;
         for (int32_t e = sg.in_ptr[v]; e < sg.in_ptr[v + 1]; e++) s += (uint64_t)sg.size[sg.in_ent[e].x] / gg;
         if (s > 0xffffffffull) return false;
-        if (free_only && s > 0x7fffffffull) return false;  // tier 2: signed per-step deltas (int32)
+        if (delta_slots && s > 0x7fffffffull) return false;  // tier 2: signed per-step deltas (int32)
     }
     auto virt = [&](int32_t r, int32_t b) -> int32_t {
         for (int32_t j = sg.U_ptr[r]; j < sg.U_ptr[r + 1]; j++)
@@ -209,8 +209,8 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     // in a per-CTA global slice
     p.gmem_static = gmem_static ? 1 : 0;
     p.gmem_af = gmem_af ? 1 : 0;
-    p.free_only = (free_only && !gmem_af) ? 1 : 0;
-    if (p.free_only && !gmem_static) return false;      // MODE 3 reads the tables from the global image
+    p.delta_slots = (delta_slots && !gmem_af) ? 1 : 0;
+    if (p.delta_slots && !gmem_static) return false;      // MODE 3 reads the tables from the global image
     const size_t Sl = ((size_t)(p.L + 1) * p.S + 3) & ~(size_t)3;   // padded per-candidate slots (magis_eval2.cu)
     p.af_bytes = (uint64_t)((P * Sl * 8 + 255) / 256 * 256);
     const size_t static_end = o;
@@ -225,7 +225,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     // are written there); last: only where phase 4 gathers the frees
     p.off_pos = (uint32_t)o;  o = a16(o + (size_t)(NTX + 1) * P * 2);
     p.off_last = (uint32_t)o; o = a16(o + (gmem_af ? (size_t)NTX * P * 2 : 0));
-    p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * (p.free_only ? 4 : 8)));   // tier 2: int32 delta
+    p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * (p.delta_slots ? 4 : 8)));   // tier 2: int32 delta
     p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
     p.nwm = (NT + 31) / 32 + 3;                         // mark_bits reads up to 2 words past a chunk start

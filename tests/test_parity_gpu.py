@@ -28,7 +28,7 @@ DEV = "cuda:0"
 VARIANTS = {"auto": {}, "v1": {"MAGIS_VARIANT": "1"}, "p1": {"MAGIS_P": "1", "MAGIS_TEAMS": "1"},
             "p2": {"MAGIS_P": "2", "MAGIS_TEAMS": "1"}, "p4": {"MAGIS_P": "4", "MAGIS_TEAMS": "1"},
             "t2p1": {"MAGIS_P": "1", "MAGIS_TEAMS": "2"}, "t2p2": {"MAGIS_P": "2", "MAGIS_TEAMS": "2"},
-            # plan tiers: 1 tables in global, 2 + free-only slots (alloc gathered), 3 slots in global
+            # plan tiers: 1 tables in global, 2 + int32 delta slots, 3 slots in global
             "tier1p4": {"MAGIS_TIER": "1", "MAGIS_P": "4", "MAGIS_TEAMS": "1"},
             "tier2p1": {"MAGIS_TIER": "2", "MAGIS_P": "1", "MAGIS_TEAMS": "1"},
             "tier2p4": {"MAGIS_TIER": "2", "MAGIS_P": "4", "MAGIS_TEAMS": "1"},
