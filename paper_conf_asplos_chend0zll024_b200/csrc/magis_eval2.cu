@@ -606,8 +606,12 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 #pragma unroll
                     for (int j = 0; j < LMAX; j++) {
                         const uint32_t v = (uint32_t)pr[j];
-                        bad |= v >= (uint32_t)NT;
-                        pc_[min(v, trash) * P] = (uint16_t)(lo + j + 1);
+                        // every id >= NT (not only >= NTX) goes to the trash slot:
+                        // the virtual slots and the dummy NTX - 1 read by row padding
+                        // must stay untouched by a bad permutation
+                        const bool oob = v >= (uint32_t)NT;
+                        bad |= oob;
+                        pc_[(oob ? trash : v) * P] = (uint16_t)(lo + j + 1);
                     }
                 } else {
 #pragma unroll

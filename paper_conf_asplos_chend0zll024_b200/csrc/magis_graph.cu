@@ -109,6 +109,11 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
     if (!d) return set_error(MAGIS_E_INVAL, "desc is NULL");
     const int32_t n = d->n_nodes;
     const int32_t R = d->n_eligible;
+    if (n < 1) return set_error(MAGIS_E_INVAL, "n_nodes < 1");
+    if (R < 0) return set_error(MAGIS_E_INVAL, "n_eligible < 0");
+    if (d->n_edges < 0) return set_error(MAGIS_E_INVAL, "n_edges < 0");
+    if (!d->out_bytes || !d->cost || !d->is_output)
+        return set_error(MAGIS_E_INVAL, "null node array");
     // --- F-Trans variant regions (NEXT-4, reading F1) -------------------------
     const int32_t F = rd ? rd->n_regions : 0;
     if (F < 0) return set_error(MAGIS_E_INVAL, "n_regions < 0");
@@ -129,11 +134,6 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
                 nreg[v] = ((R + ri) << 2) | rd->node_variant[v];
             }
         }
-    if (n < 1) return set_error(MAGIS_E_INVAL, "n_nodes < 1");
-    if (R < 0) return set_error(MAGIS_E_INVAL, "n_eligible < 0");
-    if (d->n_edges < 0) return set_error(MAGIS_E_INVAL, "n_edges < 0");
-    if (!d->out_bytes || !d->cost || !d->is_output)
-        return set_error(MAGIS_E_INVAL, "null node array");
     if (d->n_edges > 0 && (!d->edge_src || !d->edge_dst))
         return set_error(MAGIS_E_INVAL, "null edge array");
     if (R > 0 && (!d->eligible_tensor || !d->late_user_ptr || !d->late_user_idx))
@@ -734,8 +734,12 @@ int host_path(magis_graph* g, int64_t K, const void* h_perm, int pb, const uint8
     const size_t row_b = pb == 0 ? (size_t)(NT + 1) / 2 : (size_t)NT * pb;   // host bytes per schedule
     if (pb <= 1) {
         if (!h_exc_ptr) return set_error(MAGIS_E_INVAL, "null exception pointer array");
-        for (int64_t k = 0; k < K; k++)
+        for (int64_t k = 0; k < K; k++) {
             if (h_exc_ptr[k + 1] < h_exc_ptr[k]) return set_error(MAGIS_E_INVAL, "exception offsets decrease");
+            // no row has more escapes than steps (bounds the staging copy)
+            if (h_exc_ptr[k + 1] - h_exc_ptr[k] > NT)
+                return set_error(MAGIS_E_INVAL, "more exceptions than steps in schedule " + std::to_string(k));
+        }
         if (h_exc_ptr[K] > h_exc_ptr[0] && !h_exc) return set_error(MAGIS_E_INVAL, "null exception array");
     }
     DeviceGuard guard(g->device);

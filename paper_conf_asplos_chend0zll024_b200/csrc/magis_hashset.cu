@@ -146,6 +146,7 @@ extern "C" int magis_hashset_clear(magis_hashset* s, void* cuda_stream) {
     GCK(cudaMemsetAsync(s->keys, 0, s->cap * 8, st));
     GCK(cudaMemsetAsync(s->owner, 0xFF, (s->cap + 1) * 8, st));
     GCK(cudaMemsetAsync(s->stats, 0, 16, st));
+    s->epoch = 0;   // the owners were reset to all-ones on the same stream
     return MAGIS_SUCCESS;
 }
 

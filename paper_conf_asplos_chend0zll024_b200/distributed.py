@@ -23,16 +23,44 @@ def shard_range(K: int, rank: int, world: int):
     return K * rank // world, K * (rank + 1) // world
 
 
+class FrontCapacityError(RuntimeError):
+    """Some rank's local front holds more points than the padded capacity, so
+    the gathered fronts would silently miss points (magis_pareto_merge returned
+    MAGIS_E_CAPACITY there and reported the size it needs)."""
+
+
+def pack_front(front: Dict[str, torch.Tensor]) -> torch.Tensor:
+    """One int64 record buffer [1 + 3 cap]: front_n, then cap ids, cap peaks
+    and cap latencies (fp64 bit patterns), so a single all-gather moves it."""
+    fid = front["front_id"].reshape(-1)
+    cap = fid.numel()
+    buf = torch.empty(1 + 3 * cap, dtype=torch.int64, device=fid.device)
+    buf[0:1] = front["front_n"].reshape(-1)[:1].to(torch.int64)
+    buf[1:1 + cap] = fid
+    buf[1 + cap:1 + 2 * cap] = front["front_peak"].reshape(-1)
+    buf[1 + 2 * cap:] = front["front_lat"].reshape(-1).contiguous().view(torch.int64)
+    return buf
+
+
 def gather_fronts(front: Dict[str, torch.Tensor], group=None) -> Dict[str, torch.Tensor]:
-    """All-gather the padded local fronts (id, peak, lat; each [cap])."""
+    """All-gather the padded local fronts (id, peak, lat; each [cap]) as one
+    packed buffer (a single collective, 24 B per point + 8 B per rank), and
+    check every rank's front size against the capacity: a front cut at cap
+    would make the merged global front wrong, so it raises on every rank."""
     world = dist.get_world_size(group)
-    out = {}
-    for key in ("front_id", "front_peak", "front_lat"):
-        t = front[key].contiguous()
-        buf = torch.empty(world * t.numel(), dtype=t.dtype, device=t.device)
-        dist.all_gather_into_tensor(buf, t, group=group)
-        out[key] = buf
-    return out
+    t = pack_front(front)
+    cap = (t.numel() - 1) // 3
+    buf = torch.empty(world * t.numel(), dtype=torch.int64, device=t.device)
+    dist.all_gather_into_tensor(buf, t, group=group)
+    rec = buf.view(world, t.numel())
+    sizes = rec[:, 0].cpu()
+    if bool((sizes > cap).any()):
+        raise FrontCapacityError(
+            f"local front sizes {sizes.tolist()} exceed the capacity {cap}: re-run with cap >= {int(sizes.max())}")
+    return {"front_id": rec[:, 1:1 + cap].reshape(-1),
+            "front_peak": rec[:, 1 + cap:1 + 2 * cap].reshape(-1),
+            "front_lat": rec[:, 1 + 2 * cap:].reshape(-1).view(torch.float64),
+            "front_n": sizes}
 
 
 def global_front(front: Dict[str, torch.Tensor], cap: int, mem_limit: int = -1,
@@ -41,7 +69,8 @@ def global_front(front: Dict[str, torch.Tensor], cap: int, mem_limit: int = -1,
     """Merge this rank's padded front with every other rank's.
 
     ``merge`` defaults to the device merge (magis_pareto_merge); the CPU gloo
-    tests pass a host implementation with the same contract."""
+    tests pass a host implementation with the same contract.  Raises
+    FrontCapacityError (on every rank) if some local front exceeded its cap."""
     g = gather_fronts(front, group)
     merge = merge or (lambda peak, lat, ids, cap, M, L: magis.pareto_merge(
         peak, lat, None, ids=ids, cap=cap, mem_limit=M, lat_limit=L))

@@ -10,6 +10,9 @@ plausible slip in either shows up as a mismatch:
 * ``literal_peak``: the same with the literal, garbled S_j <= i <= F_j
    -- used to show that the text's 1056 needs reading P1.
 * ``all_topo_orders``: brute-force enumeration of every topological order.
+* ``defn_latency``: the modelled latency as the longest path of an explicit
+  event DAG (compute / D2H / H2D queue chains + data edges, reading P7) --
+  a different formulation from the oracle's three-queue recurrence.
 """
 from __future__ import annotations
 
@@ -141,6 +144,69 @@ def defn_eval(n, edges, size, outputs, elig, U, dec, perm):
             sz[v] = 0 if k == 1 else size[elig[r]]
     pk, _ = interval_peak(order, te, sz, set(outputs))
     return 0, pk
+
+
+# ---- latency as the longest path of an explicit event DAG (reading P7) ----
+
+def event_dag(n, edges, cost, size, elig, U, dec, perm, B, lam):
+    """The schedule's execution as a DAG of timed events (P:1784-1789,
+    P:1796-1799; reading P7), built from scratch and independent of the
+    oracle's queue recurrence:
+
+    * one event per active node, weighted by its duration: a compute op v
+      takes cost(v), a clone A' takes cost(t_r) (reading P9), a Store or Load
+      of t_r takes lam + |t_r| / B;
+    * resource edges: the compute ops (with clones), the Stores and the Loads
+      each run on their own in-order queue, so consecutive events of one
+      queue in step order are chained;
+    * data edges: every edge (u, v) of the transformed graph (Fig. 8) -- in
+      particular t_r -> Store_r -> Load_r -> each late user.
+
+    -> (weights {node: duration}, arcs set of (u, v))."""
+    active, te = transformed(n, edges, elig, U, list(dec))
+    order = [v for v in perm if v in active]
+
+    def kind(v):                     # 'c' compute, 's' Store, 'l' Load
+        if v < n:
+            return "c"
+        return "csl"[(v - n) % 3]
+
+    w = {}
+    for v in order:
+        if v < n:
+            w[v] = cost[v]
+        else:
+            r, k = divmod(v - n, 3)
+            w[v] = cost[elig[r]] if k == 0 else lam + size[elig[r]] / B
+    arcs = set(te)
+    for q in "csl":
+        seq = [v for v in order if kind(v) == q]
+        arcs |= set(zip(seq, seq[1:]))
+    return w, arcs
+
+
+def longest_path_latency(w, arcs):
+    """Makespan of the event DAG: finish(v) = w(v) + max(finish(p)) over the
+    predecessors p of v (0 without any), latency = max finish.  Memoised
+    recursion over the predecessor sets -- no step order is used."""
+    import sys
+    pre = {v: [] for v in w}
+    for u, v in arcs:
+        pre[v].append(u)
+    memo = {}
+    sys.setrecursionlimit(max(10000, 4 * len(w) + 100))
+
+    def fin(v):
+        if v not in memo:
+            memo[v] = w[v] + max((fin(p) for p in pre[v]), default=0.0)
+        return memo[v]
+
+    return max((fin(v) for v in w), default=0.0)
+
+
+def defn_latency(n, edges, cost, size, elig, U, dec, perm, B, lam):
+    """Latency of a valid schedule by the event-DAG longest path."""
+    return longest_path_latency(*event_dag(n, edges, cost, size, elig, U, dec, perm, B, lam))
 
 
 # ---- NEXT-3: hot-spots, dominators, heat / score (written from the text) ----

@@ -156,3 +156,51 @@ def test_gloo_hash_filter_matches_single_rank():
         assert Xr == sorted(X)
         for b, (lo, new) in enumerate(out):
             assert new == exp[b][lo:lo + len(new)].tolist()
+
+
+def _cap_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        cap = 8
+        # rank 1's local front needed 11 points (magis_pareto_merge reports the
+        # required size in front_n and returns MAGIS_E_CAPACITY)
+        local = {"front_id": torch.arange(cap, dtype=torch.int64) + 100 * rank,
+                 "front_peak": torch.arange(cap, dtype=torch.int64),
+                 "front_lat": torch.arange(cap, 0, -1, dtype=torch.float64),
+                 "front_n": torch.tensor([cap if rank == 0 else cap + 3], dtype=torch.int64)}
+        try:
+            pdist.global_front(local, cap, merge=lambda *a: None)
+            q.put((rank, "no error"))
+        except pdist.FrontCapacityError as e:
+            q.put((rank, "raised" if "11" in str(e) else str(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_front_over_capacity_raises_on_every_rank():
+    """a local front cut at cap must not be merged silently; the
+    packed all-gather carries every rank's front_n and all ranks raise."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = free_port()
+    procs = [ctx.Process(target=_cap_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    assert res == {0: "raised", 1: "raised"}
+
+
+def test_pack_front_roundtrip():
+    cap = 5
+    fr = {"front_id": torch.tensor([3, 1, 4, -1, -1]), "front_peak": torch.tensor([10, 20, 30, -1, -1]),
+          "front_lat": torch.tensor([3.5, 2.25, 1e-300, float("inf"), float("inf")], dtype=torch.float64),
+          "front_n": torch.tensor([3])}
+    b = pdist.pack_front(fr)
+    assert b.numel() == 1 + 3 * cap and int(b[0]) == 3
+    assert torch.equal(b[1 + 2 * cap:].view(torch.float64), fr["front_lat"])

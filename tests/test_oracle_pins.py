@@ -118,6 +118,105 @@ def test_T1_swap_toy(order, dec, B, exp):
     assert lat == exp[2]
 
 
+# T3: two swaps contending on both copy queues.  a->b->c->d->e plus the skips
+# a->e, b->e; sizes a=b=100, c=d=10, e=1 (output); costs 1.0; eligible
+# r=0: (a, U={e}), r=1: (b, U={e}); B = 50 B/s, lambda = 0.5 s, so every
+# transfer takes 0.5 + 100/50 = 2.5 s.  Ids a..e = 0..4, clone0/store0/load0
+# = 5/6/7, clone1/store1/load1 = 8/9/10.
+T3_EDGES = [(0, 1), (1, 2), (2, 3), (3, 4), (0, 4), (1, 4)]
+T3_ARGS = dict(n=5, edges=T3_EDGES, size=[100, 100, 10, 10, 1], outputs=[4], cost=[1.0] * 5,
+               elig=[0, 1], U=[[4], [4]], B=50.0, lam=0.5)
+
+
+@pytest.mark.parametrize("order,dec,exp", [
+    # no swap: sum of costs; a, b, c, d all live at step 3 -> 220
+    ([0, 1, 2, 3, 4, 5, 6, 7, 8, 9, 10], (0, 0), (0, 220, 5.0)),
+    # B: a b St0 St1 c Ld1 d Ld0 e.  compute a[0,1] b[1,2] c[2,3] d[3,4];
+    #    St0 = max(Td 0, a 1) -> [1, 3.5];  St1 = max(Td 3.5, b 2) -> [3.5, 6]
+    #    (D2H contention: alone it would be [2, 4.5]);
+    #    Ld1 = max(Th 0, St1 6) -> [6, 8.5];  Ld0 = max(Th 8.5, St0 3.5) -> [8.5, 11]
+    #    (H2D contention: alone it would be [3.5, 6]);
+    #    e = max(Tc 4, Ld0 11, Ld1 8.5) -> [11, 12].  Without the D2H queue the
+    #    makespan is 10.5, without the H2D queue 9.5, without either 8.0.
+    #    Memory: a 0..2, b 1..4, c 4..6, Ld1 5..8, d 6..8, Ld0 7..8, e 8 -> 211.
+    ([0, 1, 6, 9, 2, 10, 3, 7, 4, 5, 8], (2, 2), (0, 211, 12.0)),
+    # C: a b St0 St1 c d Ld0 Ld1 e: transfer bound, Ld1 = [6, 8.5] either way,
+    #    e = [8.5, 9.5]
+    ([0, 1, 6, 9, 2, 3, 7, 10, 4, 5, 8], (2, 2), (0, 211, 9.5)),
+    # D: only a swapped: St0 [1, 3.5], Ld0 = [3.5, 6] after d [3, 4] -> e [6, 7];
+    #    b stays live to e: b + d + Ld0 + e = 211 at the last step
+    ([0, 1, 6, 2, 3, 7, 4, 5, 8, 9, 10], (2, 0), (0, 211, 7.0)),
+    # E: both swapped, Ld0 issued before St1 finished: a St0 b St1 Ld0 Ld1 c d e
+    #    St0 [1, 3.5], St1 [3.5, 6], Ld0 = max(0, 3.5) -> [3.5, 6], Ld1 = max(6, 6)
+    #    -> [6, 8.5]; c [2, 3], d [3, 4]; e = [8.5, 9.5].  The Loads come too
+    #    early for memory: b (to c), Ld0, Ld1 and c are live at step 6 -> 310
+    ([0, 6, 1, 9, 7, 10, 2, 3, 4, 5, 8], (2, 2), (0, 310, 9.5)),
+])
+def test_T3_two_swap_queue_contention(order, dec, exp):
+    """Hand-worked timelines (reading P7): rows B and E need
+    both the D2H (Td) and the H2D (Th) serialisation; the event-DAG longest
+    path (tests/_defn.py) reproduces every row."""
+    a = T3_ARGS
+    g = make(a["n"], a["edges"], a["size"], a["outputs"], cost=a["cost"], elig=a["elig"], U=a["U"],
+             B=a["B"], lam=a["lam"])
+    st, peak, lat, _ = g.eval(order, np.array(dec, np.uint8))
+    assert (st, peak) == exp[:2]
+    assert lat == exp[2]
+    assert _defn.defn_latency(a["n"], a["edges"], a["cost"], a["size"], a["elig"], a["U"], dec, order,
+                              a["B"], a["lam"]) == exp[2]
+    assert _defn.defn_eval(a["n"], a["edges"], a["size"], a["outputs"], a["elig"], a["U"], dec, order) == exp[:2]
+
+
+def test_T3_queue_ablation_changes_the_makespan():
+    """The two copy queues are what row B measures: dropping the D2H or the
+    H2D chain from the event DAG changes its makespan to 10.5 / 9.5 (the
+    values worked out in the row's comment), so an oracle without either
+    serialisation could not produce 12.0."""
+    a = T3_ARGS
+    order = [0, 1, 6, 9, 2, 10, 3, 7, 4, 5, 8]
+    w, arcs = _defn.event_dag(a["n"], a["edges"], a["cost"], a["size"], a["elig"], a["U"], (2, 2), order,
+                              a["B"], a["lam"])
+    assert _defn.longest_path_latency(w, arcs) == 12.0
+    assert _defn.longest_path_latency(w, arcs - {(6, 9)}) == 10.5          # no D2H queue
+    assert _defn.longest_path_latency(w, arcs - {(10, 7)}) == 9.5          # no H2D queue
+    assert _defn.longest_path_latency(w, arcs - {(6, 9), (10, 7)}) == 8.0
+
+
+def test_swap_latency_matches_event_dag_on_random_dags():
+    """Random DAGs with swaps (positive lambda, slow links so transfers
+    contend): the oracle's three-queue recurrence equals the event-DAG longest
+    path within fp64 rounding.  The cases are counted where dropping the D2H
+    or the H2D queue chain from the DAG changes the makespan -- there the
+    oracle could not match without that serialisation."""
+    rng = np.random.default_rng(777)
+    nswap = nd2h = nh2d = 0
+    for _ in range(8000):
+        n, edges, size, cost, outs, elig, U, dec = random_case(rng)
+        if len(elig) == 0:
+            continue
+        dec = np.where(rng.random(len(elig)) < 0.7, 2, dec).astype(np.uint8)
+        if not (dec == 2).any():
+            continue
+        B = float(rng.choice([1.0, 10.0, 1e3]))
+        lam = float(rng.random())
+        g = make(n, edges, size, outs, cost=cost, elig=elig, U=U, B=B, lam=lam)
+        perm, te, active = random_valid_perm(rng, n, edges, elig, U, dec)
+        st, pk, lat, _ = g.eval(perm, dec)
+        assert st == 0
+        w, arcs = _defn.event_dag(n, edges, cost, size, elig, U, dec, perm, B, lam)
+        ref = _defn.longest_path_latency(w, arcs)
+        assert abs(lat - ref) <= 1e-12 * max(1.0, abs(ref)), (lat, ref)
+        order = [v for v in perm if v in w]
+        st_q = [x for x in order if x >= n and (x - n) % 3 == 1]
+        ld_q = [x for x in order if x >= n and (x - n) % 3 == 2]
+        nd2h += _defn.longest_path_latency(w, arcs - set(zip(st_q, st_q[1:]))) != ref
+        nh2d += _defn.longest_path_latency(w, arcs - set(zip(ld_q, ld_q[1:]))) != ref
+        nswap += 1
+        if nswap == 800:
+            break
+    assert nswap == 800 and nd2h > 50 and nh2d > 50, (nswap, nd2h, nh2d)
+
+
 T2_EDGES = [(0, 1), (1, 2), (2, 3), (3, 4), (1, 4)]
 
 
