@@ -13,12 +13,13 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libmagis.so")
-SOURCES = ["magis_graph.cu", "magis_eval.cu", "magis_eval2.cu", "magis_plan.cu", "magis_pareto.cu", "magis_gen.cu", "magis_window.cu",
-           "magis_hotspot.cu", "magis_ghash.cu", "magis_hashset.cu"]
+SOURCES = ["magis_graph.cu", "magis_eval.cu", "magis_eval2.cu", "magis_eval2_m0t1.cu", "magis_eval2_m0t2.cu",
+           "magis_eval2_m1.cu", "magis_eval2_m2.cu", "magis_eval2_m3.cu", "magis_plan.cu", "magis_pareto.cu",
+           "magis_gen.cu", "magis_window.cu", "magis_hotspot.cu", "magis_ghash.cu", "magis_hashset.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
-         "--expt-relaxed-constexpr", "-Xptxas", "-v"]
+         "--expt-relaxed-constexpr", "-Xptxas", "-v"] + os.environ.get("MAGIS_NVCC_EXTRA", "").split()
 
 
 def _stale() -> bool:
@@ -43,7 +44,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not _stale():
         return LIB
     # recompile the objects older than their source or any header, in parallel
-    headers = [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith(".h")]
+    headers = [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith((".h", ".cuh"))]
     headers += [os.path.join(INCLUDE, "magis.h"), __file__]
     th = max(os.path.getmtime(h) for h in headers)
     todo = []
