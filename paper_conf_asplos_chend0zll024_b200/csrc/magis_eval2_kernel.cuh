@@ -41,7 +41,7 @@ namespace magis {
 
 constexpr uint32_t kKindShift = 29;
 constexpr uint32_t kIdMask = (1u << kKindShift) - 1;
-constexpr uint32_t kHdrOut = 2, kHdrClone = 3, kNop = 7;   // kHdr = 1, kHdrCopy = 4
+constexpr uint32_t kHdrOut = 2, kHdrClone = 3, kNop = 7;   // kHdr = 1, kHdrCopy = 4, kHdrGated = 5
 // named barriers of team t: main 1 + 5t, FULL 2 + 5t + slot, EMPTY 4 + 5t + slot
 constexpr int kBarMain = 1, kBarFull = 2, kBarEmpty = 4, kBarTeam = 5;
 
@@ -350,6 +350,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // this team's state: the static tables (MODE 0) are shared, the state follows at + team * stride
     char* sm = sm_all + (size_t)team * pl.state_stride;
     const int32_t NT = pl.NT, R = pl.R, n = pl.n;
+    const int32_t gate_lo = pl.gate_lo;      // ids >= gate_lo may be absent in a candidate
     // optional phase profile (MAGIS_PROFILE=1): cycles between marks, thread 0
     // of the main warps and lane 0 of the latency warp, summed over CTAs
     const bool prof = pl.prof && (tid == 0 || tid == TM);
@@ -393,7 +394,12 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     uint8_t* dec_s = (uint8_t*)(sm + pl.off_dec);
     uint32_t* evm = (uint32_t*)(sm + pl.off_evm);          // [P][nwm] event-step marks
     uint8_t* sdec = (uint8_t*)(sm + pl.off_sdec);          // [2][P][Rw] decisions for the latency warp
-    const int32_t Rw = (R + 15) & ~15;                     // padded row of sdec
+    // decision row: R eligible tensors, then F F-Trans regions (NEXT-4)
+    const int32_t F = pl.F, Rd = pl.Rd;
+    const int32_t Rw = (Rd + 15) & ~15;                    // padded row of sdec
+    const uint32_t* rnl = (const uint32_t*)(sb + pl.off_rn);        // [nRN] region nodes
+    const uint8_t* nvarr = (const uint8_t*)(sb + pl.off_nvar);      // [F]
+    const double* vcost = (const double*)(sb + pl.off_vcost);        // [4F]
     const int32_t nwm = pl.nwm, cap = pl.evcap;
     unsigned long long* evk_s = (unsigned long long*)(sm + pl.off_ev);             // [2][P][cap]
     double* evc_s = (double*)(sm + pl.off_ev + (size_t)2 * P * cap * 8);          // [2][P][cap]
@@ -469,6 +475,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     double bl = 0.0;                 // no swap: base cost + re-computations
                     for (int r = lane; r < R; r += 32)
                         if (dd[r] == 1) bl += rtab[r].x;
+                    for (int i = lane; i < F; i += 32) bl += vcost[4 * i + dd[R + i]];   // chosen variants
 #pragma unroll
                     for (int o = 16; o > 0; o >>= 1) bl += __shfl_xor_sync(0xffffffffu, bl, o);
                     lat = g.base_cost + bl;
@@ -520,6 +527,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // (candidate, tensor) of this thread's first item in the P x R loops and the
     // per-iteration step (TM / R, TM % R): no division inside the group loop
     const int c_0 = R > 0 ? tid / R : 0, r_0 = tid - c_0 * R, dc_ = R > 0 ? TM / R : 0, dr_ = TM - dc_ * R;
+    // the same over the whole decision row (R + F)
+    const int c_0d = Rd > 0 ? tid / Rd : 0, r_0d = tid - c_0d * Rd, dc_d = Rd > 0 ? TM / Rd : 0, dr_d = TM - dc_d * Rd;
     const int32_t lo = tt * L;
     const bool vec4 = (NT & 3) == 0;
     // perm chunk kept in registers when short (32 steps only where the
@@ -555,14 +564,14 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     }
     // the group's decisions (<= 2 bytes per thread) are prefetched into
     // registers one group ahead, like the perm chunk
-    const bool dreg = P * R <= 2 * TM;
+    const bool dreg = P * Rd <= 2 * TM;
     uint32_t dq0 = 0, dq1 = 0;
     auto load_dec = [&](int64_t grp_) {
-        const int64_t b = grp_ * P * (int64_t)R, lim = K * (int64_t)R;
-        dq0 = (tid < P * R && b + tid < lim) ? (uint32_t)__ldcs(dec + b + tid) : 0u;
-        dq1 = (tid + TM < P * R && b + tid + TM < lim) ? (uint32_t)__ldcs(dec + b + tid + TM) : 0u;
+        const int64_t b = grp_ * P * (int64_t)Rd, lim = K * (int64_t)Rd;
+        dq0 = (tid < P * Rd && b + tid < lim) ? (uint32_t)__ldcs(dec + b + tid) : 0u;
+        dq1 = (tid + TM < P * Rd && b + tid + TM < lim) ? (uint32_t)__ldcs(dec + b + tid + TM) : 0u;
     };
-    if (dreg && R > 0 && ncta > 0) load_dec(cta);
+    if (dreg && Rd > 0 && ncta > 0) load_dec(cta);
     for (int gi = 0; gi < ncta; gi++) {
         const int64_t grp = cta + (int64_t)gi * ncta_all;
         const int slot = gi & 1;
@@ -574,15 +583,19 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         {
             uint32_t badm = 0, swm = 0;
             int it = 0;
-            for (int i = tid, c = c_0, r = r_0; i < P * R; i += TM, c += dc_, r += dr_, it++) {
-                if (r >= R) { r -= R; c++; }
-                // the group's decision rows are contiguous: dec[grp * P * R + i]
+            for (int i = tid, c = c_0d, r = r_0d; i < P * Rd; i += TM, c += dc_d, r += dr_d, it++) {
+                if (r >= Rd) { r -= Rd; c++; }
+                // the group's decision rows are contiguous: dec[grp * P * Rd + i]
                 uint8_t d;
                 if (dreg) d = (uint8_t)(it == 0 ? dq0 : dq1);
-                else d = ((vmask >> c) & 1u) ? dec[grp * P * (int64_t)R + i] : 0;
+                else d = ((vmask >> c) & 1u) ? dec[grp * P * (int64_t)Rd + i] : 0;
                 dec_s[i] = d;
-                if (d == 2) swm |= 1u << c;
-                if ((d > 2) | ((d == 1) & !(__ldg(g.rflag + r) & kRHasInput))) badm |= 1u << c;
+                if (r < R) {
+                    if (d == 2) swm |= 1u << c;
+                    if ((d > 2) | ((d == 1) & !(__ldg(g.rflag + r) & kRHasInput))) badm |= 1u << c;
+                } else if (d >= nvarr[r - R]) {
+                    badm |= 1u << c;                       // reading F1: not a variant of region r - R
+                }
             }
             // one shared atomic per warp
             swm = __reduce_or_sync(0xffffffffu, swm);
@@ -671,7 +684,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             if (!((vmask >> c) & 1u)) continue;
             const uint32_t ur = urow[r];                       // (U offset, |U_r|) packed
             const uint32_t u0 = ur & 0xffffu, u1 = u0 + (ur >> 16);
-            const uint8_t d = dec_s[c * R + r];
+            const uint8_t d = dec_s[c * Rd + r];
             uint32_t* em = evm + c * nwm;
             uint16_t* pc_ = pos + c;
 #pragma unroll
@@ -702,6 +715,24 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const uint32_t pb = pc_[(uint32_t)ubs[j] * P];
                 pc_[(NT + j) * P] = (d == 0) ? (uint16_t)pb : (uint16_t)0;
                 if (d == 2 && pb) atomicOr(em + ((pb - 1) >> 5), 1u << ((pb - 1) & 31));
+            }
+        }
+        // F-Trans regions (NEXT-4, reading F1): a node of an unchosen variant is
+        // absent (position 0); every region node must still be in the
+        // permutation
+        if (F > 0) {
+            const int32_t nRN = pl.nRN;
+            // (candidate, node) of item q = tid + i TM, stepped without divisions
+            const int dcr = TM / nRN, drr = TM - dcr * nRN;
+            int c = tid / nRN, k = tid - c * nRN;
+            for (int q = tid; q < P * nRN; q += TM, c += dcr, k += drr) {
+                if (k >= nRN) { k -= nRN; c++; }
+                if (!((vmask >> c) & 1u)) continue;
+                const uint32_t e = rnl[k];
+                const uint32_t id = e & 0xffffu, reg = (e >> 16) & 0x3fffu, var = e >> 30;
+                uint16_t* pp = pos + id * P + c;
+                if (*pp == 0) atomicOr(&cl.flags[c], MAGIS_ST_NOT_PERM);
+                else if (dec_s[c * Rd + R + reg] != var) *pp = 0;
             }
         }
         bar_sync(kBarMain + bb, TM);
@@ -986,7 +1017,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                                 o++;
                             }
                             double c = cost_s[v];
-                            if (v >= n && pos[v * P + cm] == 0) c = 0.0;
+                            if (v >= gate_lo && pos[v * P + cm] == 0) c = 0.0;
                             if (j & 1) cb += c; else ca += c;
                         }
                     }
@@ -1014,7 +1045,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                                     o++;
                                 }
                                 double c = cv[u];
-                                if (v >= n && pos[v * P + cm] == 0) c = 0.0;
+                                if (v >= gate_lo && pos[v * P + cm] == 0) c = 0.0;
                                 if (u & 1) cb += c; else ca += c;
                             }
                         }
@@ -1043,7 +1074,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         if constexpr (LMAX <= kRegL) {
             if (gi + 1 < ncta) load_chunk(grp + ncta_all);
         }
-        if (dreg && R > 0 && gi + 1 < ncta) load_dec(grp + ncta_all);
+        if (dreg && Rd > 0 && gi + 1 < ncta) load_dec(grp + ncta_all);
         bar_sync(kBarMain + bb, TM);
         PROF_MARK(5);
         // ---- phase 6: hand-off to the latency warps (they fold the aggregates) ----
@@ -1057,7 +1088,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             h.swp[c] = (int)((swm >> c) & 1u);
             h.nev[c] = ne;
         }
-        if (R > 0) {
+        if (Rd > 0) {
             // decisions of the group -> the slot (rows padded to 16 bytes)
             const int nw = Rw >> 2;
             uint32_t* dst = reinterpret_cast<uint32_t*>(sdec + (size_t)slot * P * Rw);
@@ -1067,7 +1098,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 #pragma unroll
                 for (int b = 0; b < 4; b++) {
                     const int r = 4 * w + b;
-                    if (r < R) x |= (uint32_t)dec_s[c * R + r] << (8 * b);
+                    if (r < Rd) x |= (uint32_t)dec_s[c * Rd + r] << (8 * b);
                 }
                 dst[i] = x;
             }

@@ -454,14 +454,14 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
     {
         const char* force = std::getenv("MAGIS_VARIANT");
         const char* pforce = std::getenv("MAGIS_P");
-        const bool allow2 = !(force && std::atoi(force) != 2) && F == 0;   // variant 2 folds only Fig. 8 gates
+        const bool allow2 = !(force && std::atoi(force) != 2);
         cudaDeviceProp prop;
         if (allow2 && cudaGetDeviceProperties(&prop, device) == cudaSuccess) {
             std::vector<double> rtab((size_t)2 * R);
             for (int32_t r = 0; r < R; r++) { rtab[2 * r] = tcost[r]; rtab[2 * r + 1] = xfer[r]; }
             SuperGraphHost sg{n, R, NT, cons_ptr.data(), cons_ent.data(), in_ptr.data(), in_ent.data(),
                               size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data(), rtab.data(),
-                              elig.data()};
+                              elig.data(), F, ngate.data(), nvar.data(), vcost.data()};
             const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
             // pick the packing with the most candidates in flight per SM
             // (P x resident CTAs; ties go to more CTAs, which hide barriers).

@@ -90,6 +90,12 @@ struct Plan2 {
     uint32_t off_urow;       // [R] u32: offset of U_r in ubs | |U_r| << 16
     uint32_t off_ubs;        // [nU] u16 late users, grouped by r
     uint32_t off_utr;        // [R] u16 t_r
+    int32_t F, Rd;           // F-Trans regions (NEXT-4) and the decision row length R + F
+    int32_t nRN;             // nodes inside regions (every variant)
+    uint32_t off_rn;         // [nRN] u32: node id | region << 16 | variant << 30
+    uint32_t off_nvar;       // [F] u8 variants per region
+    uint32_t off_vcost;      // [4F] f64 cost sum of (region, variant)
+    int32_t gate_lo;         // smallest id of a node that may be absent (region nodes, then n)
     uint32_t off_pos, off_last, off_af, off_dec, off_end;
     uint32_t off_evm;        // [P][NW] swap-event step marks (bit per step)
     uint32_t off_sdec;       // [2][P][Rw] decisions handed to the latency warp
@@ -190,6 +196,11 @@ struct SuperGraphHost {
     const int32_t* U_idx;
     const double* rtab;        // [R][2] (cost(t_r), swap transfer time)
     const int32_t* elig;       // [R] t_r
+    // F-Trans variant regions (NEXT-4, reading F1); F = 0: none
+    int32_t F;
+    const int32_t* ngate;      // [n] gate of an original node: -1 or (R + region) << 2 | variant
+    const int32_t* nvar;       // [F] variants per region
+    const double* vcost;       // [4F] cost sum of (region, variant)
 };
 
 // Build the variant-2 plan and its static shared-memory image for a given P.

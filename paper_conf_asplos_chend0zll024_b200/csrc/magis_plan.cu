@@ -24,7 +24,8 @@ namespace magis {
 
 namespace {
 constexpr uint32_t kKindShift = 29;
-constexpr uint32_t kEdge = 0, kHdr = 1, kHdrOut = 2, kHdrClone = 3, kHdrCopy = 4, kNop = 7;
+// kHdrGated: an original node inside an F-Trans region (present iff its variant is chosen)
+constexpr uint32_t kEdge = 0, kHdr = 1, kHdrOut = 2, kHdrClone = 3, kHdrCopy = 4, kHdrGated = 5, kNop = 7;
 
 uint64_t gcd64(uint64_t a, uint64_t b) {
     while (b) { uint64_t t = a % b; a = b; b = t; }
@@ -120,15 +121,29 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     };
     std::vector<std::vector<uint32_t>> cons(NT), ins(NT);
     std::vector<uint32_t> hdrs(NT);
+    // F-Trans regions (reading F1): every node of every variant is listed; the
+    // kernel zeroes the positions of the nodes of unchosen variants per
+    // candidate, so edges need no gates (an edge exists iff both ends do)
+    const int32_t F = sg.F;
+    std::vector<uint32_t> rn;
+    int32_t gate_lo = n;
+    for (int32_t v = 0; v < n && F > 0; v++) {
+        const int32_t gt = sg.ngate[v];
+        if (gt < 0) continue;
+        const int32_t reg = (gt >> 2) - R, var = gt & 3;
+        if (reg < 0 || reg >= F || reg >= (1 << 14) || (sg.nflag[v] & kFlagOutput)) return false;
+        rn.push_back((uint32_t)v | ((uint32_t)reg << 16) | ((uint32_t)var << 30));
+        gate_lo = std::min(gate_lo, v);
+    }
     for (int32_t u = 0; u < NT; u++) {
         uint32_t kind;
-        if (u < n) kind = (sg.nflag[u] & kFlagOutput) ? kHdrOut : kHdr;
+        if (u < n) kind = (sg.nflag[u] & kFlagOutput) ? kHdrOut : (F > 0 && sg.ngate[u] >= 0) ? kHdrGated : kHdr;
         else kind = ((u - n) % 3 == 0) ? kHdrClone : kHdrCopy;
         hdrs[u] = (kind << kKindShift) | (uint32_t)u;
         for (int32_t e = sg.cons_ptr[u]; e < sg.cons_ptr[u + 1]; e++) {
             const int2 ce = sg.cons_ent[e];
             int32_t c = ce.x;
-            if (ce.y >= 0 && (ce.y & 3) == 0) {       // t_r -> b, b in U_r
+            if (ce.y >= 0 && (ce.y >> 2) < R && (ce.y & 3) == 0) {   // t_r -> b, b in U_r (region gates have r >= R)
                 c = virt(ce.y >> 2, ce.x);
                 if (c < 0) return false;
             }
@@ -203,6 +218,13 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     p.off_urow = (uint32_t)o;  o = a16(o + (size_t)std::max(R, 1) * 4);
     p.off_ubs = (uint32_t)o;   o = a16(o + (size_t)std::max(nU, 1) * 2);
     p.off_utr = (uint32_t)o;   o = a16(o + (size_t)std::max(R, 1) * 2);
+    p.F = F;
+    p.Rd = R + F;
+    p.nRN = (int32_t)rn.size();
+    p.gate_lo = gate_lo;
+    p.off_rn = (uint32_t)o;    o = a16(o + std::max<size_t>(rn.size(), 1) * 4);
+    p.off_nvar = (uint32_t)o;  o = a16(o + (size_t)std::max(F, 1));
+    p.off_vcost = (uint32_t)o; o = a16(o + (size_t)4 * std::max(F, 1) * 8);
     p.static_bytes = (uint32_t)o;
     // graph tables in shared memory (staged) or read from the global image
     // (L1/L2; the row reads stay coalesced); per-step slots in shared memory or
@@ -226,11 +248,11 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     p.off_pos = (uint32_t)o;  o = a16(o + (size_t)(NTX + 1) * P * 2);
     p.off_last = (uint32_t)o; o = a16(o + (gmem_af ? (size_t)NTX * P * 2 : 0));
     p.off_af = (uint32_t)o;   o = a16(o + (gmem_af ? 0 : (size_t)P * Sl * (p.delta_slots ? 4 : 8)));   // tier 2: int32 delta
-    p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R, 1));
+    p.off_dec = (uint32_t)o;  o = a16(o + (size_t)P * std::max(R + F, 1));
     p.off_end = (uint32_t)o;  o = a16(o + (size_t)P * 3 * std::max(R, 1) * 8);
     p.nwm = (NT + 31) / 32 + 3;                         // mark_bits reads up to 2 words past a chunk start
     p.off_evm = (uint32_t)o;  o = a16(o + (size_t)P * p.nwm * 4);
-    p.off_sdec = (uint32_t)o; o = a16(o + (size_t)2 * P * ((std::max(R, 1) + 15) & ~15));
+    p.off_sdec = (uint32_t)o; o = a16(o + (size_t)2 * P * ((std::max(R + F, 1) + 15) & ~15));
     p.off_ev = (uint32_t)o;
     // event steps of a candidate: at most the marked steps (<= 3R + |U|)
     int cap = std::min(std::max(p.max_events, 1), 128);
@@ -303,7 +325,14 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
             utr[r] = (uint16_t)sg.elig[r];
             for (int32_t j = u0; j < u0 + cnt; j++) ubs[j] = (uint16_t)sg.U_idx[j];
         }
-        put(p.off_urow, urow.data(), (size_t)R * 4);
+        put(p.off_rn, rn.data(), rn.size() * 4);
+    if (F > 0) {
+        std::vector<uint8_t> nv(F);
+        for (int32_t i = 0; i < F; i++) nv[i] = (uint8_t)sg.nvar[i];
+        put(p.off_nvar, nv.data(), (size_t)F);
+        put(p.off_vcost, sg.vcost, (size_t)4 * F * 8);
+    }
+    put(p.off_urow, urow.data(), (size_t)R * 4);
         put(p.off_ubs, ubs.data(), (size_t)nU * 2);
         put(p.off_utr, utr.data(), (size_t)R * 2);
     }

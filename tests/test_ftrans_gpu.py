@@ -23,14 +23,24 @@ def gpu_eval(g, P, D):
     return st.cpu().numpy(), pk.cpu().numpy(), lt.cpu().numpy()
 
 
-@pytest.mark.parametrize("layers,variant", [(2, "auto"), (2, "1"), (24, "auto")])
+# the packed kernel (variant 2) on every plan tier, and the gated v1 kernel
+REGION_VARIANTS = {"auto": {}, "v1": {"MAGIS_VARIANT": "1"},
+                   "p1": {"MAGIS_P": "1", "MAGIS_TEAMS": "1"},
+                   "tier1p4": {"MAGIS_TIER": "1", "MAGIS_P": "4", "MAGIS_TEAMS": "1"},
+                   "tier2p1": {"MAGIS_TIER": "2", "MAGIS_P": "1", "MAGIS_TEAMS": "1"},
+                   "tier3p2": {"MAGIS_TIER": "3", "MAGIS_P": "2", "MAGIS_TEAMS": "1"}}
+
+
+@pytest.mark.parametrize("layers,variant", [(2, v) for v in REGION_VARIANTS] + [(24, "auto"), (24, "v1")])
 def test_regions_parity(layers, variant, monkeypatch):
-    monkeypatch.delenv("MAGIS_VARIANT", raising=False)
-    if variant != "auto":
-        monkeypatch.setenv("MAGIS_VARIANT", variant)
+    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER"):
+        monkeypatch.delenv(k, raising=False)
+    for k, v in REGION_VARIANTS[variant].items():
+        monkeypatch.setenv(k, v)
     wl = build_workload("c3f", layers=layers)
     g = Graph.from_workload(wl, device=0)
-    assert g.F == wl.F > 0 and g.info["variant"] in (0, 1)
+    assert g.F == wl.F > 0
+    assert (g.info["variant"] in (0, 1)) if variant == "v1" else g.info["variant"] == 2
     o = OracleGraph.from_workload(wl)
     K = 1000 if layers == 2 else 300
     P, D = CandidateGenerator(wl, CandidateSpec(seed=11)).generate(0, K)
