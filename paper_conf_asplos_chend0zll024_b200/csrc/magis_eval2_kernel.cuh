@@ -312,7 +312,7 @@ __device__ __forceinline__ double candidate_latency(unsigned long long* key, dou
 // its own per-group state, slots and named barriers; the tables are shared),
 // so one team's barrier waits overlap the other's work.
 template <int P, int LMAX, int MODE, int TEAMS>
-__global__ void __launch_bounds__(TEAMS * (kMainThreads2 / TEAMS + 32 * P), 1)
+__global__ void __launch_bounds__(TEAMS * (kMainThreads2 / TEAMS + 32 * P) < 1024 ? TEAMS * (kMainThreads2 / TEAMS + 32 * P) : 1024, 1)
 eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
              const int32_t* __restrict__ perm, const uint8_t* __restrict__ dec,
              uint8_t* __restrict__ out_status, int64_t* __restrict__ out_peak,
@@ -370,7 +370,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // read in place from the global image when they do not fit
     const char* sb = MODE ? blob : sm_all;
     if (MODE == 0) bulk_stage(sm_all, blob, pl.static_bytes, &mbar);
-    else if (pl.cost_sm) bulk_stage(sm_all, blob + pl.off_cost, (uint32_t)((pl.NTX * 8 + 15) & ~15), &mbar);
+    else if (pl.cost_sm) bulk_stage(sm_all, blob + (pl.cost_cls ? pl.off_ccls : pl.off_cost), pl.stage_bytes, &mbar);
     const uint32_t* wtab = (const uint32_t*)(sb + pl.off_wtab);   // [WM][4]: consumer rows, input rows
     const uint2* crow = (const uint2*)(sb + pl.off_crow);
     const uint32_t* chdr = (const uint32_t*)(sb + pl.off_chdr);
@@ -382,6 +382,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const uint32_t* size_s = (const uint32_t*)(sb + pl.off_size);
     const double2* rtab = (const double2*)(sb + pl.off_rtab);       // [R] (cost(t_r), swap transfer time)
     const double* cost_s = (MODE != 0 && pl.cost_sm) ? (const double*)sm_all : (const double*)(sb + pl.off_cost);
+    // tier 2 with cost classes: cost(v) = class value [class index of v], both staged
+    const bool ccls = MODE == 3 && pl.cost_sm && pl.cost_cls;
+    const uint8_t* ccls_idx = (const uint8_t*)(sm_all + pl.ccls_idx_off);
     const uint2* ninfo = (const uint2*)(sb + pl.off_ninfo);
     const uint16_t* lul = (const uint16_t*)(sb + pl.off_lul);
     const uint32_t* urow = (const uint32_t*)(sb + pl.off_urow);     // [R] U_r offset | |U_r| << 16
@@ -1016,7 +1019,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                                 cout_[o] = ca + cb;
                                 o++;
                             }
-                            double c = cost_s[v];
+                            double c = ccls ? cost_s[ccls_idx[v]] : cost_s[v];
                             if (v >= gate_lo && pos[v * P + cm] == 0) c = 0.0;
                             if (j & 1) cb += c; else ca += c;
                         }
@@ -1033,7 +1036,8 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 #pragma unroll
                         for (int u = 0; u < 8; u++) vv[u] = jb + u < nst ? __ldcs(pp + jb + u) : 0;   // last read
 #pragma unroll
-                        for (int u = 0; u < 8; u++) cv[u] = jb + u < nst ? cost_s[vv[u]] : 0.0;
+                        for (int u = 0; u < 8; u++)
+                            cv[u] = jb + u < nst ? (ccls ? cost_s[ccls_idx[vv[u]]] : cost_s[vv[u]]) : 0.0;
 #pragma unroll
                         for (int u = 0; u < 8; u++) {
                             const int j = jb + u;

@@ -67,7 +67,10 @@ struct DevGraph {
 // Variant-2 plan (magis_eval2.cu): graph as per-thread streams in shared
 // memory, P candidates packed per u16 lane group.  Built on the host by
 // plan2_build; all offsets are bytes into the dynamic shared memory.
-constexpr int kMainThreads2 = 512;
+#ifndef MAGIS_MAIN_THREADS
+#define MAGIS_MAIN_THREADS 512
+#endif
+constexpr int kMainThreads2 = MAGIS_MAIN_THREADS;   // main (non-latency) threads of a variant-2 CTA
 
 struct Plan2 {
     int32_t P;            // candidates per group (1, 2, 4); 0 = not applicable
@@ -96,6 +99,11 @@ struct Plan2 {
     uint32_t off_nvar;       // [F] u8 variants per region
     uint32_t off_vcost;      // [4F] f64 cost sum of (region, variant)
     int32_t gate_lo;         // smallest id of a node that may be absent (region nodes, then n)
+    int32_t cost_cls;        // tier 2: the cost table staged as u8 class indices + <= 256 class values
+    uint32_t off_ccls;       // image offset of [class values f64 (a16) | class index u8 [NTX]]
+    uint32_t ccls_idx_off;   // offset of the class index inside that region
+    uint32_t stage_bytes;    // bytes staged into shared memory on tiers 1 / 2 (cost table or classes)
+    uint32_t image_bytes;    // whole device image (static_bytes staged on tier 0, then the class tables)
     uint32_t off_pos, off_last, off_af, off_dec, off_end;
     uint32_t off_evm;        // [P][NW] swap-event step marks (bit per step)
     uint32_t off_sdec;       // [2][P][Rw] decisions handed to the latency warp
