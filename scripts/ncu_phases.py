@@ -25,7 +25,7 @@ for r in rows[hi + 1:]:
             a[j] += int(float(r[col] or 0))
         except ValueError:
             pass
-src = open("paper_conf_asplos_chend0zll024_b200/csrc/magis_eval2.cu").read().split("\n")
+src = open("paper_conf_asplos_chend0zll024_b200/csrc/magis_eval2_kernel.cuh").read().split("\n")
 marks = [("helpers", r"^// -+ packed u16"), ("latency helpers", r"^// The event steps of a swapping"),
          ("kernel setup", r"^template <int P, int LMAX, int MODE, int TEAMS>"),
          ("latency warps", r"latency warps \(reading P7\)"), ("main setup", r"= main warps ="),
