@@ -11,12 +11,9 @@
 // nodes last in id order, and 1% one random transposition.  It is bit-exact
 // with the CPU generator used to produce test inputs (tests compare them).
 //
-// One thread builds one candidate (Kahn is sequential).  The top kHS entries
-// of its ready heap (the levels every pop walks) live in shared memory,
-// deeper entries and the in-degree / position arrays in a graph-owned global
-// scratch laid out index-major across threads so a warp's accesses to one
-// index coalesce.  (The ready set of these graphs peaks at their number of
-// sources -- weights and inputs, 163-502 -- so most heap levels are on chip.)
+// One thread builds one candidate (Kahn is sequential); its heap, in-degree
+// and position arrays live in a graph-owned global scratch laid out
+// index-major across threads so a warp's accesses to one index coalesce.
 #include <climits>
 
 #include "magis_internal.h"
@@ -40,22 +37,15 @@ __device__ __forceinline__ uint64_t rnd(uint64_t seed, uint64_t k, uint32_t stre
     return mix64(h ^ i);
 }
 
-constexpr int kGenBlock = 192;   // threads per CTA
-constexpr int kHS = 128;         // heap entries per thread in shared memory (kGenBlock x kHS x 8 B = 192 KB)
-
 struct Scratch {
     int32_t* indeg;   // [n][T]
-    uint64_t* heap;   // [n][T] (entries >= kHS)
+    uint64_t* heap;   // [n][T]
     int32_t* base;    // [n][T]
     int32_t* posb;    // [n][T]
     int64_t* opt;     // [2R][T]
     int64_t T;
-    uint64_t* hs;     // shared: [kHS][kGenBlock]
-    int tl;           // thread index in the CTA
     __device__ __forceinline__ int32_t& I(int32_t i, int64_t t) const { return indeg[(int64_t)i * T + t]; }
-    __device__ __forceinline__ uint64_t& H(int32_t i, int64_t t) const {
-        return i < kHS ? hs[i * kGenBlock + tl] : heap[(int64_t)i * T + t];
-    }
+    __device__ __forceinline__ uint64_t& H(int32_t i, int64_t t) const { return heap[(int64_t)i * T + t]; }
     __device__ __forceinline__ int32_t& B(int32_t i, int64_t t) const { return base[(int64_t)i * T + t]; }
     __device__ __forceinline__ int32_t& Q(int32_t i, int64_t t) const { return posb[(int64_t)i * T + t]; }
     __device__ __forceinline__ int64_t& O(int32_t i, int64_t t) const { return opt[(int64_t)i * T + t]; }
@@ -119,12 +109,9 @@ __device__ void keyed_kahn(const DevGraph& g, const GenTables& gt, const Scratch
     (void)g;
 }
 
-__global__ void __launch_bounds__(kGenBlock)
+__global__ void __launch_bounds__(128)
 gen_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32_t* __restrict__ perms,
            uint8_t* __restrict__ decs, Scratch w) {
-    extern __shared__ uint64_t gen_hs[];
-    w.hs = gen_hs;
-    w.tl = (int)threadIdx.x;
     const int32_t n = g.n, R = g.R, NT = g.NT;
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     for (int64_t kk = t; kk < K; kk += w.T) {
@@ -210,8 +197,8 @@ size_t gen_scratch_bytes(const DevGraph& g, int64_t T) {
 
 int64_t gen_threads(int device) {
     cudaDeviceProp p;
-    if (cudaGetDeviceProperties(&p, device) != cudaSuccess) return 148 * kGenBlock;
-    return (int64_t)p.multiProcessorCount * kGenBlock;   // one CTA per SM (shared-memory heaps)
+    if (cudaGetDeviceProperties(&p, device) != cudaSuccess) return 148 * 256;
+    return (int64_t)p.multiProcessorCount * 256;
 }
 
 cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp, uint64_t id0, int64_t K,
@@ -226,13 +213,10 @@ cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp
     w.base = (int32_t*)b;    b += (size_t)g.n * 4 * T;
     w.posb = (int32_t*)b;
     const int64_t threads = std::min<int64_t>(T, K);
-    const unsigned blocks = (unsigned)((threads + kGenBlock - 1) / kGenBlock);
-    const size_t smem = (size_t)kHS * kGenBlock * 8;
-    cudaError_t e = cudaFuncSetAttribute(gen_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
+    const unsigned blocks = (unsigned)((threads + 127) / 128);
     // the kernel strides over candidates by w.T; with fewer threads than T the
     // surplus threads see kk >= K and exit
-    gen_kernel<<<blocks, kGenBlock, smem, stream>>>(g, gt, sp, id0, K, perm, dec, w);
+    gen_kernel<<<blocks, 128, 0, stream>>>(g, gt, sp, id0, K, perm, dec, w);
     return cudaGetLastError();
 }
 
