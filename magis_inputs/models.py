@@ -38,22 +38,25 @@ def diamond(branches, seed: int = 1):
 # C2: ResNet-50 training, b64, 224^2, fp32 (Table 2)
 # --------------------------------------------------------------------------
 
-def _bn(ag: AG, name: str, x: T, C: int) -> T:
-    """BatchNorm as 4 primitives: mean, var, normalize, affine."""
+def _bn(ag: AG, name: str, x: T, C: int, stat_shape=None) -> T:
+    """BatchNorm as 4 primitives: mean, var, normalize, affine.
+    With ``stat_shape`` the statistics have that shape (LayerNorm: one mean /
+    variance per token, affine over the last dim C)."""
     g = ag.param(name + ".gamma", (C,))
     bt = ag.param(name + ".beta", (C,))
     N = numel(x.shape)
+    sshape = (C,) if stat_shape is None else tuple(stat_shape)
 
     def mean_bwd(ag_, dy, out, ins):
         x_, = ins
         return [(x_, ag_._g(name + ".mean.d", [dy], x_, N))]
-    mu = ag.op(name + ".mean", [x], (C,), N, mean_bwd)
+    mu = ag.op(name + ".mean", [x], sshape, N, mean_bwd)
 
     def var_bwd(ag_, dy, out, ins):
         x_, m_ = ins
         return [(x_, ag_._g(name + ".var.dx", [dy, x_, m_], x_, 3 * N)),
                 (m_, ag_._g(name + ".var.dm", [dy, x_, m_], m_, 2 * N))]
-    var = ag.op(name + ".var", [x, mu], (C,), 3 * N, var_bwd)
+    var = ag.op(name + ".var", [x, mu], sshape, 3 * N, var_bwd)
 
     def norm_bwd(ag_, dy, out, ins):
         x_, m_, v_ = ins
@@ -151,12 +154,16 @@ def _ffn(ag: AG, p: str, x: T, D: int, Fd: int, tag: str | None) -> T:
     return h
 
 
-def _ln(ag: AG, p: str, x: T, D: int) -> T:
+def _ln(ag: AG, p: str, x: T, D: int, prims: bool = False) -> T:
+    """LayerNorm: one fused op, or (``prims``) 4 primitives like BN with
+    per-token statistics."""
+    if prims:
+        return _bn(ag, p, x, D, stat_shape=x.shape[:-1])
     return ag.norm(p, x, ag.param(p + ".g", (D,)), ag.param(p + ".b", (D,)))
 
 
 def transformer(name: str, layers: int, D: int, H: int, Fd: int, vocab: int, B: int, S: int,
-                dtype_bytes: int, pre_ln: bool, ftrans: int = 1):
+                dtype_bytes: int, pre_ln: bool, ftrans: int = 1, ln_prims: bool = False):
     """BERT-style (post-LN) or GPT-style (pre-LN) training graph.  With
     ftrans > 1 the attention core and the FFN sub-graph of every layer are
     tagged as F-Trans sets (split along the batch dim) for ftrans.apply."""
@@ -177,7 +184,7 @@ def transformer(name: str, layers: int, D: int, H: int, Fd: int, vocab: int, B: 
         tag_a = f"{p}.attn" if ftrans > 1 else None
         tag_f = f"{p}.ffn" if ftrans > 1 else None
         res = x
-        h = _ln(ag, p + ".ln1", x, D) if pre_ln else x
+        h = _ln(ag, p + ".ln1", x, D, ln_prims) if pre_ln else x
         wqkv = ag.param(p + ".wqkv", (D, 3 * D))
         bqkv = ag.param(p + ".bqkv", (3 * D,))
         wo = ag.param(p + ".wo", (D, D))
@@ -196,7 +203,7 @@ def transformer(name: str, layers: int, D: int, H: int, Fd: int, vocab: int, B: 
         if not pre_ln:
             x = _ln(ag, p + ".ln1", x, D)
         res = x
-        h = _ln(ag, p + ".ln2", x, D) if pre_ln else x
+        h = _ln(ag, p + ".ln2", x, D, ln_prims) if pre_ln else x
         f = _ffn(ag, p + ".ffn", h, D, Fd, tag_f)
         ag.tag = tag_f
         f = ag.unary(p + ".drop2", f, save="y")
@@ -205,7 +212,7 @@ def transformer(name: str, layers: int, D: int, H: int, Fd: int, vocab: int, B: 
         if not pre_ln:
             x = _ln(ag, p + ".ln2", x, D)
     if pre_ln:
-        x = _ln(ag, "ln_f", x, D)
+        x = _ln(ag, "ln_f", x, D, ln_prims)
     else:
         wt = ag.param("mlm.w", (D, D))
         x = ag.matmul("mlm.dense", x, wt, (B, S, D))
@@ -224,8 +231,10 @@ def bert_large(B: int = 32, S: int = 512, ftrans: int = 4, layers: int = 24):
 
 
 def gpt_neo_1p3b(B: int = 32, S: int = 512, layers: int = 24):
+    """GPT-Neo-1.3B shape; LayerNorm as 4 primitives (SURVEY §8 config sheet:
+    ~2.3-2.6k ops, n_total ~3k with R = 128)."""
     return transformer(f"gpt_neo_1.3b_s{S}_b{B}", layers, 2048, 16, 8192, 50257, B, S, 2,
-                       pre_ln=True, ftrans=1)
+                       pre_ln=True, ftrans=1, ln_prims=True)
 
 
 # --------------------------------------------------------------------------
