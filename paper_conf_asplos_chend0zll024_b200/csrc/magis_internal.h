@@ -164,6 +164,8 @@ struct BaseDev {
     uint8_t* dec;       // [R]
     double* endb;       // [3R] scratch of the base sweep
     unsigned long long* evk;   // swap events of the base, step order
+    double* snap;       // [(max_events + 1) * 3] (D, Td, Th) of the base sweep before each event
+    int32_t* evix;      // [3R] index of the base event that writes endb[x] (INT_MAX: none)
 };
 size_t base_bytes(const DevGraph& g);
 BaseDev base_layout(const DevGraph& g, void* mem);

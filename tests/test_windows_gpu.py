@@ -75,3 +75,26 @@ def test_windows_small_graphs_with_swaps_and_bad_windows():
         E = wg.expand(ws, wln, wp)
         ref = o.eval_batch(E, np.repeat(d[None], len(ws), 0) if R else None)
         assert_parity(*res, *ref)
+
+
+@pytest.mark.parametrize("cfg", ["c2", "c5"])
+def test_windows_dense_swap_events(cfg):
+    """A base with P(swap) = 40%: most windows hold swap events, so the walk
+    starts at the window from the base's state (end times written before the
+    window read through from the base), and rejoins the base after it when
+    its state is unchanged -- every window against the oracle."""
+    wl = build_workload(cfg)
+    P, D = CandidateGenerator(wl, CandidateSpec(seed=6, p_swap=4000, p_remat=500)).generate(0, 16)
+    o = OracleGraph.from_workload(wl)
+    st, pk, lt = o.eval_batch(P, D)
+    i = int(np.argmax(st == 0))
+    assert st[i] == 0 and (D[i][:wl.R] == 2).sum() > wl.R // 4
+    wg = WindowGenerator(wl, P[i], D[i], seed=13, pct_bad=1)
+    ws, wln, wp = wg.generate(0, 2000)
+    g = Graph.from_workload(wl)
+    b, res = run_windows(g, P[i], D[i], ws, wln, wp)
+    E = wg.expand(ws, wln, wp)
+    Dk = np.repeat(D[i][None], len(ws), axis=0)
+    ref = o.eval_batch(E, Dk)
+    assert (ref[0] == 0).mean() > 0.9
+    assert_parity(*res, *ref)
