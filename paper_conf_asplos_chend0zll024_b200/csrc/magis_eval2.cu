@@ -48,6 +48,26 @@ cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, v
     const int gr = (int)std::min<int64_t>(grid, (ngroups + pl.teams - 1) / pl.teams);
     void* args[] = {(void*)&g, (void*)&pl, (void*)&blob, (void*)&K, (void*)&perm, (void*)&dec,
                     (void*)&status, (void*)&peak, (void*)&lat, (void*)&ovf, (void*)&afg};
+    if (pl.gmem_static && pl.l2win_bytes > 0) {
+        // tiers reading the graph image from global memory: an L2 persisting
+        // access window over it for this launch (the streamed candidate rows
+        // must not evict the rows every group re-reads); no stream state changes
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(gr);
+        cfg.blockDim = dim3(eval2_block(pl));
+        cfg.dynamicSmemBytes = pl.smem_total;
+        cfg.stream = stream;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        at[0].val.accessPolicyWindow.base_ptr = const_cast<void*>(blob);
+        at[0].val.accessPolicyWindow.num_bytes = pl.l2win_bytes;
+        at[0].val.accessPolicyWindow.hitRatio = 1.0f;
+        at[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        return cudaLaunchKernelExC(&cfg, kernel_for(pl), args);
+    }
     return cudaLaunchKernel(kernel_for(pl), dim3(gr), dim3(eval2_block(pl)), args, pl.smem_total, stream);
 }
 

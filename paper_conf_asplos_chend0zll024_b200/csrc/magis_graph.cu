@@ -518,6 +518,19 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
                 bool ok = cudaMalloc(&b2, bestImg.size()) == cudaSuccess;
                 ok = ok && cudaMemcpy(b2, bestImg.data(), bestImg.size(), cudaMemcpyHostToDevice) == cudaSuccess;
                 bestPl.prof = std::getenv("MAGIS_PROFILE") ? 1 : 0;
+                // graph image read from global memory: reserve persisting L2 for it
+                // (SURVEY §8(a) a0 "L2 window"); the launch sets the window
+                bestPl.l2win_bytes = 0;
+                if (bestPl.gmem_static && !std::getenv("MAGIS_NO_L2WIN") && prop.persistingL2CacheMaxSize > 0) {
+                    const size_t want = std::min<size_t>(bestImg.size(), (size_t)prop.accessPolicyMaxWindowSize);
+                    size_t cur = 0;
+                    cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+                    const size_t lim = std::min<size_t>((size_t)prop.persistingL2CacheMaxSize, std::max(cur, want));
+                    if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim) == cudaSuccess)
+                        bestPl.l2win_bytes = std::min(want, lim);
+                    else
+                        cudaGetLastError();
+                }
                 bestPl.prof_off = (uint64_t)grid * bestT * 8 * bestPl.ovf_stride;   // 8 regions per team
                 ok = ok && cudaMalloc(&ov, bestPl.prof_off + 256) == cudaSuccess;
                 ok = ok && cudaMemset(ov, 0, bestPl.prof_off + 256) == cudaSuccess;

@@ -99,6 +99,7 @@ struct Plan2 {
     uint32_t off_nvar;       // [F] u8 variants per region
     uint32_t off_vcost;      // [4F] f64 cost sum of (region, variant)
     int32_t gate_lo;         // smallest id of a node that may be absent (region nodes, then n)
+    uint64_t l2win_bytes;    // tiers 1-3: bytes of the graph image under an L2 persisting window (0: none)
     int32_t cost_cls;        // tier 2: the cost table staged as u8 class indices + <= 256 class values
     uint32_t off_ccls;       // image offset of [class values f64 (a16) | class index u8 [NTX]]
     uint32_t ccls_idx_off;   // offset of the class index inside that region
