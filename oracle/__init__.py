@@ -7,9 +7,11 @@ be imported by ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
 ``cpu_baseline`` / ``--impl reference`` legs.
 
 Pins (tests/test_oracle_*.py): Fig. 2(a) = 1056 (P:455-461), Fig. 2(b) = 96
-(P:469-476), hand-computed toys T1/T2, closed forms, brute-force
-enumeration of all topological orders against an independently written
-interval formula, invariants, Eq. (1) = 98/56/52.
+(P:469-476), hand-computed toys T1/T2/T3 (T3: two swaps
+contending on both copy queues), closed forms, brute-force enumeration of all
+topological orders against an independently written interval formula, the
+swap latency against an independent event-DAG longest path (reading P7,
+P:1784-1789), invariants, Eq. (1) = 98/56/52 (P:1057-1069).
 
 Parity status per function:
   * peak / status / argmax ....... pinned (paper numbers + brute force)
