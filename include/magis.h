@@ -120,7 +120,12 @@ typedef struct magis_graph_info {
 /*
  * Validate and upload a graph.  Builds, on `device`, the consumer and input
  * CSRs of the super-graph with per-edge activation gates, the node tables and
- * the swap-event tables, plus the eval workspace.
+ * the swap-event tables, plus the eval workspace (Table 1
+ * P:356-369).  When the evaluation plan reads its graph image from global
+ * memory (large graphs), the call raises the device's persisting-L2 limit
+ * (cudaLimitPersistingL2CacheSize) to cover the image, and every evaluation
+ * launch carries an L2 access-policy window over it; no stream attribute is
+ * changed.
  * Errors: MAGIS_E_INVAL (null pointer, n_nodes < 1, id out of range, self
  * loop, negative size or cost, non-finite cost, output marked eligible,
  * duplicate eligible tensor, empty U_r, U_r not a subset of cons(t_r),
