@@ -169,7 +169,7 @@ def peaks():
         return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-EVAL_SOURCES = ("magis_eval2.cu", "magis_plan.cu", "magis_internal.h")
+EVAL_SOURCES = ("magis_eval2_kernel.cuh", "magis_eval2.cu", "magis_plan.cu", "magis_internal.h")
 
 
 def eval_src_sha() -> str:
