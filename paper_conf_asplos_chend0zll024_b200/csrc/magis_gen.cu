@@ -12,8 +12,13 @@
 // with the CPU generator used to produce test inputs (tests compare them).
 //
 // One thread builds one candidate (Kahn is sequential); its heap, in-degree
-// and position arrays live in a graph-owned global scratch laid out
-// index-major across threads so a warp's accesses to one index coalesce.
+// and position arrays live in a graph-owned global scratch, contiguous per
+// thread: a node's successors are mostly near it in id, so a thread's
+// in-degree decrements share cache lines (an index-major layout put every
+// access on its own line).  The scratch is sized for up to one thread per
+// candidate of the call (within a memory budget): the kernel is latency
+// bound on that scratch, so threads in flight are what pays (ncu, C2: 7
+// warps per SM and 60% long-scoreboard stalls with 148 x 256 threads).
 #include <climits>
 
 #include "magis_internal.h"
@@ -44,11 +49,12 @@ struct Scratch {
     int32_t* posb;    // [n][T]
     int64_t* opt;     // [2R][T]
     int64_t T;
-    __device__ __forceinline__ int32_t& I(int32_t i, int64_t t) const { return indeg[(int64_t)i * T + t]; }
-    __device__ __forceinline__ uint64_t& H(int32_t i, int64_t t) const { return heap[(int64_t)i * T + t]; }
-    __device__ __forceinline__ int32_t& B(int32_t i, int64_t t) const { return base[(int64_t)i * T + t]; }
-    __device__ __forceinline__ int32_t& Q(int32_t i, int64_t t) const { return posb[(int64_t)i * T + t]; }
-    __device__ __forceinline__ int64_t& O(int32_t i, int64_t t) const { return opt[(int64_t)i * T + t]; }
+    int64_t n, no;    // per-thread row lengths (nodes, 2R)
+    __device__ __forceinline__ int32_t& I(int32_t i, int64_t t) const { return indeg[t * n + i]; }
+    __device__ __forceinline__ uint64_t& H(int32_t i, int64_t t) const { return heap[t * n + i]; }
+    __device__ __forceinline__ int32_t& B(int32_t i, int64_t t) const { return base[t * n + i]; }
+    __device__ __forceinline__ int32_t& Q(int32_t i, int64_t t) const { return posb[t * n + i]; }
+    __device__ __forceinline__ int64_t& O(int32_t i, int64_t t) const { return opt[t * no + i]; }
 };
 
 __device__ void heap_push(const Scratch& w, int64_t t, int32_t& nh, uint64_t x) {
@@ -195,10 +201,13 @@ size_t gen_scratch_bytes(const DevGraph& g, int64_t T) {
     return (size_t)T * ((size_t)g.n * (4 + 8 + 4 + 4) + (size_t)2 * (g.R ? g.R : 1) * 8) + 256;
 }
 
-int64_t gen_threads(int device) {
+int64_t gen_threads(int device, const DevGraph& g, int64_t K) {
     cudaDeviceProp p;
-    if (cudaGetDeviceProperties(&p, device) != cudaSuccess) return 148 * 256;
-    return (int64_t)p.multiProcessorCount * 256;
+    const int64_t base = (cudaGetDeviceProperties(&p, device) == cudaSuccess ? p.multiProcessorCount : 148) * 256LL;
+    // up to one thread per candidate, within a scratch budget of 16 GiB
+    const int64_t per = (int64_t)gen_scratch_bytes(g, 1);
+    const int64_t cap = std::max<int64_t>(base, (16LL << 30) / std::max<int64_t>(per, 1));
+    return std::max<int64_t>(base, std::min<int64_t>(K, cap)) / 128 * 128;
 }
 
 cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp, uint64_t id0, int64_t K,
@@ -207,6 +216,8 @@ cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp
     Scratch w;
     char* b = (char*)scratch;
     w.T = T;
+    w.n = g.n;
+    w.no = 2 * (g.R ? g.R : 1);
     w.heap = (uint64_t*)b;   b += (size_t)g.n * 8 * T;
     w.opt = (int64_t*)b;     b += (size_t)2 * (g.R ? g.R : 1) * 8 * T;
     w.indeg = (int32_t*)b;   b += (size_t)g.n * 4 * T;

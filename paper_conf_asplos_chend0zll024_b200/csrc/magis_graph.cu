@@ -870,10 +870,15 @@ extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* s
         spec->slack < 0)
         return set_error(MAGIS_E_INVAL, "bad generator spec");
     DeviceGuard guard(g->device);
-    if (!g->gen_scratch) {
-        const int64_t T = gen_threads(g->device);
-        CK(cudaMalloc(&g->gen_scratch, gen_scratch_bytes(g->dev, T)));
-        g->gen_T = T;
+    {
+        // scratch for up to one thread per candidate (grown on demand)
+        const int64_t T = gen_threads(g->device, g->dev, K);
+        if (!g->gen_scratch || g->gen_T < T) {
+            if (g->gen_scratch) cudaFree(g->gen_scratch);
+            g->gen_scratch = nullptr;
+            CK(cudaMalloc(&g->gen_scratch, gen_scratch_bytes(g->dev, T)));
+            g->gen_T = T;
+        }
     }
     GenSpec sp{spec->seed, spec->pct_random, spec->pct_local, spec->p_remat, spec->p_swap, spec->wmax, spec->slack};
     cudaError_t e = gen_launch(g->dev, g->gen, sp, id0, K, d_perm, d_dec, g->gen_scratch, g->gen_T,

@@ -139,7 +139,7 @@ struct GenSpec {
 };
 
 size_t gen_scratch_bytes(const DevGraph& g, int64_t T);
-int64_t gen_threads(int device);
+int64_t gen_threads(int device, const DevGraph& g, int64_t K);   // scratch threads for a call of K
 cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp, uint64_t id0, int64_t K,
                        int32_t* perm, uint8_t* dec, void* scratch, int64_t T, cudaStream_t stream);
 
