@@ -199,6 +199,21 @@ int magis_eval_schedules(const magis_graph* g, int64_t K, const int32_t* d_perm,
                          double* d_latency, void* cuda_stream);
 
 /*
+ * magis_eval_schedules plus the optional output of step a7:
+ * d_argmax [K] int32 out: the first step of the candidate's permutation
+ * (0-based index into d_perm's row, inactive optional nodes included) whose
+ * allocation brings the memory M_i to M_peak -- the first step of the
+ * memory hot-spot; -1 if status != 0.  It is always the step of
+ * an active node.  Same execution as magis_eval_schedules (one launch, the
+ * argmax is a third field of the scan's (sum, max-prefix) monoid).
+ * Errors: as magis_eval_schedules, plus MAGIS_E_UNSUPPORTED when the graph
+ * is evaluated by the simple kernel (n_total + |U| >= 65,535).
+ */
+int magis_eval_schedules_argmax(const magis_graph* g, int64_t K, const int32_t* d_perm, const uint8_t* d_dec,
+                                uint8_t* d_status, int64_t* d_peak, double* d_latency, int32_t* d_argmax,
+                                void* cuda_stream);
+
+/*
  * The same evaluation with HOST buffers (end-to-end path): the candidates are
  * copied host->device in chunks on `cuda_stream` and a second graph-owned
  * stream, overlapped with evaluation, and the results copied back.  Pinned

@@ -14,9 +14,12 @@ const void* eval2_kernel_m0t2(const Plan2& pl);
 const void* eval2_kernel_m1(const Plan2& pl);
 const void* eval2_kernel_m2(const Plan2& pl);
 const void* eval2_kernel_m3(const Plan2& pl);
+// with the first-argmax output (magis_eval2_am.cu)
+const void* eval2_kernel_am(const Plan2& pl, int mode);
 
-static const void* kernel_for(const Plan2& pl) {
+static const void* kernel_for(const Plan2& pl, bool am = false) {
     const int mode = pl.gmem_af ? 2 : pl.delta_slots ? 3 : (pl.gmem_static ? 1 : 0);
+    if (am) return eval2_kernel_am(pl, mode);
     if (mode == 0) return pl.teams == 2 ? eval2_kernel_m0t2(pl) : eval2_kernel_m0t1(pl);
     return mode == 1 ? eval2_kernel_m1(pl) : mode == 3 ? eval2_kernel_m3(pl) : eval2_kernel_m2(pl);
 }
@@ -42,12 +45,20 @@ cudaError_t eval2_occupancy(const Plan2& pl, int* blocks) {
 
 cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,
                          int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status,
-                         int64_t* peak, double* lat, cudaStream_t stream) {
+                         int64_t* peak, double* lat, cudaStream_t stream, int32_t* argmax) {
     if (K <= 0) return cudaSuccess;
+    const void* fn = kernel_for(pl, argmax != nullptr);
+    if (!fn) return cudaErrorNotSupported;
+    if (argmax) {
+        cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pl.smem_total);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
+        if (e != cudaSuccess) return e;
+    }
     const int64_t ngroups = (K + pl.P - 1) / pl.P;
     const int gr = (int)std::min<int64_t>(grid, (ngroups + pl.teams - 1) / pl.teams);
     void* args[] = {(void*)&g, (void*)&pl, (void*)&blob, (void*)&K, (void*)&perm, (void*)&dec,
-                    (void*)&status, (void*)&peak, (void*)&lat, (void*)&ovf, (void*)&afg};
+                    (void*)&status, (void*)&peak, (void*)&lat, (void*)&ovf, (void*)&afg, (void*)&argmax};
     if (pl.gmem_static && pl.l2win_bytes > 0) {
         // tiers reading the graph image from global memory: an L2 persisting
         // access window over it for this launch (the streamed candidate rows
@@ -66,9 +77,9 @@ cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, v
         at[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
         cfg.attrs = at;
         cfg.numAttrs = 1;
-        return cudaLaunchKernelExC(&cfg, kernel_for(pl), args);
+        return cudaLaunchKernelExC(&cfg, fn, args);
     }
-    return cudaLaunchKernel(kernel_for(pl), dim3(gr), dim3(eval2_block(pl)), args, pl.smem_total, stream);
+    return cudaLaunchKernel(fn, dim3(gr), dim3(eval2_block(pl)), args, pl.smem_total, stream);
 }
 
 }  // namespace magis

@@ -311,12 +311,17 @@ __device__ __forceinline__ double candidate_latency(unsigned long long* key, dou
 // TEAMS: independent teams per CTA (each TM main threads + its latency warps,
 // its own per-group state, slots and named barriers; the tables are shared),
 // so one team's barrier waits overlap the other's work.
-template <int P, int LMAX, int MODE, int TEAMS>
+// AM: also emit the first argmax step of the memory curve (SURVEY §8(a) a7's
+// optional output: the step whose allocation first reaches M_peak),
+// carried as a third monoid field; a separate instantiation, so the default
+// kernels are unchanged.
+template <int P, int LMAX, int MODE, int TEAMS, bool AM>
 __global__ void __launch_bounds__(TEAMS * (kMainThreads2 / TEAMS + 32 * P) < 1024 ? TEAMS * (kMainThreads2 / TEAMS + 32 * P) : 1024, 1)
 eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
              const int32_t* __restrict__ perm, const uint8_t* __restrict__ dec,
              uint8_t* __restrict__ out_status, int64_t* __restrict__ out_peak,
-             double* __restrict__ out_lat, char* __restrict__ ovf, char* __restrict__ afg) {
+             double* __restrict__ out_lat, char* __restrict__ ovf, char* __restrict__ afg,
+             int32_t* __restrict__ out_arg) {
     using PK = Pk<P>;
     using V = typename PK::V;
     constexpr int TM = kMainThreads2 / TEAMS;  // main threads of a team
@@ -332,6 +337,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     __shared__ Ctl ctl_t[TEAMS][2];            // per group parity (reset one group ahead)
     __shared__ long long agg_s_t[TEAMS][2][WM];   // per slot: warp aggregates of the scan,
     __shared__ long long agg_m_t[TEAMS][2][WM];   //   folded by the latency warps
+    __shared__ int agg_a_t[TEAMS][2][AM ? WM : 1];   // AM: first argmax step of each warp's max-prefix
     __shared__ double agg_c_t[TEAMS][2][WM];
     __shared__ double lwoff_t[TEAMS][4][WM];   // per latency warp: cost prefix of each team warp
     __shared__ int wcnt_t[TEAMS][WM];          // event steps per warp chunk
@@ -344,6 +350,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     Ctl* ctl = ctl_t[team];
     long long (*agg_s)[WM] = agg_s_t[team];
     long long (*agg_m)[WM] = agg_m_t[team];
+    int (*agg_a)[AM ? WM : 1] = agg_a_t[team];
     double (*agg_c)[WM] = agg_c_t[team];
     double (*lwoff)[WM] = lwoff_t[team];
     int* wcnt = wcnt_t[team];
@@ -451,6 +458,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 const uint8_t* dd = sdec + (size_t)(slot * P + c) * Rw;
                 double lat = __longlong_as_double(0x7ff0000000000000ll);
                 long long pk = 0;
+                int am_step = -1;
                 double ctot = 0.0;
                 if (!st) {
                     // fold the team's WT warp aggregates: (sum, max-prefix) -> peak,
@@ -459,15 +467,23 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     long long ss = lane < WT ? agg_s[slot][a] : 0;
                     long long mm = lane < WT ? agg_m[slot][a] : kNegInf;
                     double cc = lane < WT ? agg_c[slot][a] : 0.0;
+                    int aa = 0;
+                    if constexpr (AM) aa = lane < WT ? agg_a[slot][a] : -1;
                     const double c0 = cc;
 #pragma unroll
                     for (int o = 1; o < WT; o <<= 1) {
                         const long long ps = __shfl_up_sync(0xffffffffu, ss, o);
                         const long long pm = __shfl_up_sync(0xffffffffu, mm, o);
                         const double pc = __shfl_up_sync(0xffffffffu, cc, o);
+                        if constexpr (AM) {
+                            // the earlier part keeps the argmax on ties (first argmax)
+                            const int pa = __shfl_up_sync(0xffffffffu, aa, o);
+                            if (lane >= o && pm >= ps + mm) aa = pa;
+                        }
                         if (lane >= o) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
                     }
                     if (lane < WT) lwoff[c][lane] = cc - c0;
+                    if constexpr (AM) am_step = __shfl_sync(0xffffffffu, aa, WT - 1);
                     pk = __shfl_sync(0xffffffffu, mm, WT - 1);
                     ctot = __shfl_sync(0xffffffffu, cc, WT - 1);
                     __syncwarp();
@@ -510,6 +526,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 if (lane == 0) {
                     out_status[k] = (uint8_t)st;
                     out_peak[k] = st ? -1 : pk * pl.unit;
+                    if constexpr (AM) out_arg[k] = st ? -1 : am_step;
                     out_lat[k] = lat;
                 }
             }
@@ -968,6 +985,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
             //      free = slot; with swaps also the compute-cost prefix, and the
             //      event steps of the chunk are emitted in order
             long long s1 = 0, m1 = kNegInf;
+            int a1 = -1;                                     // AM: first step reaching m1
             double cs1 = 0.0;
             int o = wpre + evx;
             const int o0 = o;
@@ -980,7 +998,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 for (int j = 0; j < LMAX; j++) {
                     if (j < nst) {
                         s1 += dp[j];
-                        m1 = max(m1, s1);
+                        if constexpr (AM) { if (s1 > m1) { m1 = s1; a1 = lo + j; } } else m1 = max(m1, s1);
                     }
                 }
             } else
@@ -990,7 +1008,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 for (int j = 0; j < LMAX; j++) {
                     const uint2 af = afp[j];
                     s1 += af.x;
-                    m1 = max(m1, s1);
+                    if constexpr (AM) { if (s1 > m1) { m1 = s1; a1 = lo + j; } } else m1 = max(m1, s1);
                     s1 -= af.y;
                 }
             } else {
@@ -999,7 +1017,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     if (j < nst) {
                         const uint2 af = afp[j];
                         s1 += af.x;
-                        m1 = max(m1, s1);
+                        if constexpr (AM) { if (s1 > m1) { m1 = s1; a1 = lo + j; } } else m1 = max(m1, s1);
                         s1 -= af.y;
                     }
                 }
@@ -1061,14 +1079,22 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 // warp-level monoid scan: (s1, m1) then (s2, m2) = (s1 + s2, max(m1, s1 + m2))
                 long long ss = s1, mm = m1;
                 double cc = cs1;
+                int aa = a1;
 #pragma unroll
                 for (int o2 = 1; o2 < 32; o2 <<= 1) {
                     const long long ps = __shfl_up_sync(0xffffffffu, ss, o2);
                     const long long pm = __shfl_up_sync(0xffffffffu, mm, o2);
                     const double pc = __shfl_up_sync(0xffffffffu, cc, o2);
+                    if constexpr (AM) {
+                        const int pa = __shfl_up_sync(0xffffffffu, aa, o2);
+                        if (lane >= o2 && pm >= ps + mm) aa = pa;      // earlier steps win ties
+                    }
                     if (lane >= o2) { mm = max(pm, ps + mm); ss = ps + ss; cc = pc + cc; }
                 }
-                if (lane == 31) { agg_s[slot][warp] = ss; agg_m[slot][warp] = mm; agg_c[slot][warp] = cc; }
+                if (lane == 31) {
+                    agg_s[slot][warp] = ss; agg_m[slot][warp] = mm; agg_c[slot][warp] = cc;
+                    if constexpr (AM) agg_a[slot][warp] = aa;
+                }
                 // add the lane's exclusive cost prefix within the warp to its events
                 const double pre = cc - cs1;
                 for (int e = o0; e < o; e++) cout_[e] += pre;
@@ -1133,31 +1159,31 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
 }
 
 
-template <int P, int MODE, int TEAMS>
+template <int P, int MODE, int TEAMS, bool AM>
 static const void* kernel_ptr(int lmax) {
     if constexpr (MODE == 0) {
-        if (lmax <= 4) return (const void*)eval2_kernel<P, 4, 0, TEAMS>;
-        if (lmax <= 8) return (const void*)eval2_kernel<P, 8, 0, TEAMS>;
-        if (lmax <= 12) return (const void*)eval2_kernel<P, 12, 0, TEAMS>;
-        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, 0, TEAMS>;
-        if (lmax <= 20) return (const void*)eval2_kernel<P, 20, 0, TEAMS>;
-        if (lmax <= 24) return (const void*)eval2_kernel<P, 24, 0, TEAMS>;
-        if (lmax <= 28) return (const void*)eval2_kernel<P, 28, 0, TEAMS>;
-        return (const void*)eval2_kernel<P, 32, 0, TEAMS>;
+        if (lmax <= 4) return (const void*)eval2_kernel<P, 4, 0, TEAMS, AM>;
+        if (lmax <= 8) return (const void*)eval2_kernel<P, 8, 0, TEAMS, AM>;
+        if (lmax <= 12) return (const void*)eval2_kernel<P, 12, 0, TEAMS, AM>;
+        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, 0, TEAMS, AM>;
+        if (lmax <= 20) return (const void*)eval2_kernel<P, 20, 0, TEAMS, AM>;
+        if (lmax <= 24) return (const void*)eval2_kernel<P, 24, 0, TEAMS, AM>;
+        if (lmax <= 28) return (const void*)eval2_kernel<P, 28, 0, TEAMS, AM>;
+        return (const void*)eval2_kernel<P, 32, 0, TEAMS, AM>;
     } else {
-        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, MODE, 1>;
-        if (lmax <= 24) return (const void*)eval2_kernel<P, 24, MODE, 1>;
-        if (lmax <= 28) return (const void*)eval2_kernel<P, 28, MODE, 1>;
-        if (lmax <= 32) return (const void*)eval2_kernel<P, 32, MODE, 1>;
-        if (lmax <= 48) return (const void*)eval2_kernel<P, 48, MODE, 1>;
-        return (const void*)eval2_kernel<P, 64, MODE, 1>;
+        if (lmax <= 16) return (const void*)eval2_kernel<P, 16, MODE, 1, AM>;
+        if (lmax <= 24) return (const void*)eval2_kernel<P, 24, MODE, 1, AM>;
+        if (lmax <= 28) return (const void*)eval2_kernel<P, 28, MODE, 1, AM>;
+        if (lmax <= 32) return (const void*)eval2_kernel<P, 32, MODE, 1, AM>;
+        if (lmax <= 48) return (const void*)eval2_kernel<P, 48, MODE, 1, AM>;
+        return (const void*)eval2_kernel<P, 64, MODE, 1, AM>;
     }
 }
 
-template <int MODE, int TEAMS>
+template <int MODE, int TEAMS, bool AM = false>
 static const void* kernel_mode(const Plan2& pl) {
-    return pl.P == 4 ? kernel_ptr<4, MODE, TEAMS>(pl.L)
-                     : pl.P == 2 ? kernel_ptr<2, MODE, TEAMS>(pl.L) : kernel_ptr<1, MODE, TEAMS>(pl.L);
+    return pl.P == 4 ? kernel_ptr<4, MODE, TEAMS, AM>(pl.L)
+                     : pl.P == 2 ? kernel_ptr<2, MODE, TEAMS, AM>(pl.L) : kernel_ptr<1, MODE, TEAMS, AM>(pl.L);
 }
 
 }  // namespace magis

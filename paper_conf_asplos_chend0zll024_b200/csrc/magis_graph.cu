@@ -631,6 +631,29 @@ extern "C" int magis_eval_schedules(const magis_graph* g, int64_t K, const int32
     return MAGIS_SUCCESS;
 }
 
+// a7's optional output: the step that first reaches the peak, in the batch call
+extern "C" int magis_eval_schedules_argmax(const magis_graph* g, int64_t K, const int32_t* d_perm,
+                                           const uint8_t* d_dec, uint8_t* d_status, int64_t* d_peak,
+                                           double* d_latency, int32_t* d_argmax, void* cuda_stream) {
+    clear_error();
+    if (!g) return set_error(MAGIS_E_INVAL, "graph is NULL");
+    if (K < 0) return set_error(MAGIS_E_INVAL, "K < 0");
+    if (K == 0) return MAGIS_SUCCESS;
+    if (!d_perm || !d_status || !d_peak || !d_latency || !d_argmax)
+        return set_error(MAGIS_E_INVAL, "null device pointer");
+    if (g->dev.Rd > 0 && !d_dec) return set_error(MAGIS_E_INVAL, "d_dec is NULL but R + n_regions > 0");
+    if (g->cfg.variant != 2)
+        return set_error(MAGIS_E_UNSUPPORTED, "argmax output needs the packed kernel (the graph is too large for it)");
+    DeviceGuard guard(g->device);
+    cudaError_t e = eval2_launch(g->dev, g->plan2, g->blob2, g->ovf2, g->afg2, g->cfg.grid, K, d_perm, d_dec,
+                                 d_status, d_peak, d_latency, (cudaStream_t)cuda_stream, d_argmax);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return set_error(MAGIS_E_CUDA, std::string("eval launch: ") + cudaGetErrorString(e));
+    }
+    return MAGIS_SUCCESS;
+}
+
 // NEXT-3: hot-spots and heat / score of selected candidates.
 extern "C" int magis_hotspots(magis_graph* g, int64_t K, const int32_t* d_perm, const uint8_t* d_dec,
                               int32_t nsplit, uint8_t* d_status, int64_t* d_peak, uint8_t* d_hot,

@@ -222,7 +222,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
                  std::vector<char>* image);
 cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,
                          int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status,
-                         int64_t* peak, double* lat, cudaStream_t stream);
+                         int64_t* peak, double* lat, cudaStream_t stream, int32_t* argmax = nullptr);
 cudaError_t eval2_occupancy(const Plan2& pl, int* blocks_per_sm);
 int eval2_block(const Plan2& pl);      // threads per CTA
 

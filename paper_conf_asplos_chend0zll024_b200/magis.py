@@ -29,7 +29,7 @@ EXPORTS = ["magis_graph_load", "magis_graph_free", "magis_graph_info_get", "magi
            "magis_graph_idom", "magis_eval_schedules_host_u16", "magis_ghash_create", "magis_ghash_free",
            "magis_graph_hash", "magis_ghash_info", "magis_hashset_create", "magis_hashset_free",
            "magis_hashset_clear", "magis_hashset_filter", "magis_hashset_stats", "magis_graph_load_regions",
-           "magis_eval_schedules_host_delta8", "magis_eval_schedules_host_delta4"]
+           "magis_eval_schedules_host_delta8", "magis_eval_schedules_host_delta4", "magis_eval_schedules_argmax"]
 
 
 class MagisError(RuntimeError):
@@ -89,6 +89,8 @@ def lib() -> ctypes.CDLL:
     L.magis_graph_info_get.restype = ctypes.c_int
     L.magis_eval_schedules.argtypes = [P, i64, P, P, P, P, P, P]
     L.magis_eval_schedules.restype = ctypes.c_int
+    L.magis_eval_schedules_argmax.argtypes = [P, i64, P, P, P, P, P, P, P]
+    L.magis_eval_schedules_argmax.restype = ctypes.c_int
     L.magis_eval_schedules_host.argtypes = [P, i64, P, P, P, P, P, P]
     L.magis_eval_schedules_host.restype = ctypes.c_int
     L.magis_eval_schedules_host_u16.argtypes = [P, i64, P, P, P, P, P, P]
@@ -275,9 +277,11 @@ class Graph:
         except Exception:
             pass
 
-    def eval_schedules(self, perm, dec=None, status=None, peak=None, latency=None, stream=None):
+    def eval_schedules(self, perm, dec=None, status=None, peak=None, latency=None, stream=None, argmax=None):
         """perm: cuda int32 [K, n_total]; dec: cuda uint8 [K, R + F] (or None if R + F == 0).
-        Returns (status uint8 [K], peak int64 [K], latency float64 [K]) device tensors."""
+        Returns (status uint8 [K], peak int64 [K], latency float64 [K]) device tensors;
+        with ``argmax`` (True, or an int32 [K] cuda tensor) also the first step
+        reaching the peak (magis_eval_schedules_argmax) as a fourth tensor."""
         import torch
         K = int(perm.shape[0])
         assert perm.dtype == torch.int32 and perm.is_cuda and perm.is_contiguous()
@@ -289,6 +293,12 @@ class Graph:
         status = torch.empty(K, dtype=torch.uint8, device=dev) if status is None else status
         peak = torch.empty(K, dtype=torch.int64, device=dev) if peak is None else peak
         latency = torch.empty(K, dtype=torch.float64, device=dev) if latency is None else latency
+        if argmax is not None and argmax is not False:
+            am = torch.empty(K, dtype=torch.int32, device=dev) if argmax is True else argmax
+            _check(self._L.magis_eval_schedules_argmax(self._h, K, _tptr(perm), _tptr(dec) if self.dec_len else None,
+                                                       _tptr(status), _tptr(peak), _tptr(latency), _tptr(am),
+                                                       _stream_ptr(stream)))
+            return status, peak, latency, am
         _check(self._L.magis_eval_schedules(self._h, K, _tptr(perm), _tptr(dec) if self.dec_len else None,
                                             _tptr(status), _tptr(peak), _tptr(latency),
                                             _stream_ptr(stream)))
