@@ -116,7 +116,7 @@ def test_event_overflow_path(cfg, K, variant):
     assert_parity(*res, *ref)
 
 
-@pytest.mark.parametrize("cfg", ["c2", "c3", "c4"])
+@pytest.mark.parametrize("cfg", ["c2", "c3", "c4", "c5"])
 def test_full_bench_size_sampled_parity(cfg):
     """The bench's launch: the config's full K generated on the device (a1),
     scored in one call; 768 candidates spread over the launch (every CTA,
@@ -144,3 +144,24 @@ def test_full_bench_size_sampled_parity(cfg):
         assert np.array_equal(Dd[idt, :wl.R].cpu().numpy(), Dh[:, :wl.R])
     ref = eval_parallel(OracleGraph.from_workload(wl), Ph, Dh)
     assert_parity(st[idt].cpu().numpy(), pk[idt].cpu().numpy(), lt[idt].cpu().numpy(), *ref)
+
+
+def test_c3f_full_size_sampled_parity():
+    """C3f (F-Trans variant regions, NEXT-4) at the bench's K = 65,536 on the
+    packed kernel: the host generator's candidates (the device generator does
+    not cover regions), 512 of them spread over the launch checked by the
+    oracle."""
+    from magis_inputs import CONFIGS
+    wl = wl_of("c3f")
+    K = CONFIGS["c3f"]["K"]
+    P, D = CandidateGenerator(wl, CandidateSpec(seed=1)).generate(0, K)
+    g = Graph.from_workload(wl)
+    assert g.info["variant"] == 2
+    Dd = torch.from_numpy(np.ascontiguousarray(D[:, :g.dec_len])).cuda()
+    st, pk, lt = (t.cpu().numpy() for t in g.eval_schedules(torch.from_numpy(P).cuda(), Dd))
+    rng = np.random.default_rng(3)
+    ids = np.unique(np.concatenate([np.arange(0, 128), np.arange(K - 128, K), rng.integers(0, K, 256)]))
+    ref = eval_parallel(OracleGraph.from_workload(wl), P[ids], D[ids])
+    assert (ref[0] == 0).mean() > 0.9
+    assert_parity(st[ids], pk[ids], lt[ids], *ref)
+
