@@ -340,7 +340,8 @@ def main():
     tr, tr_src = ncu_traffic(cfg, K)
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak_gbs, "unit": "GB/s",
             "frac": round(achieved / peak_gbs, 4), "traffic": tr, "traffic_source": tr_src, "peak_source": peak_src,
-            "kernel": {0: "magis::eval_kernel<smem>", 1: "magis::eval_kernel<global>", 2: "magis::eval2_kernel"}[g.info["variant"]],
+            "kernel": {0: "magis::eval_kernel<smem>", 1: "magis::eval_kernel<global>", 2: "magis::eval2_kernel",
+                       3: "magis::evalb_kernel (2-CTA cluster per candidate)"}[g.info["variant"]],
             "alg_bytes_per_launch": alg_bytes,
             "bytes_per_candidate": bytes_per_cand, "kernel_ms_avg": round(kern_avg, 4),
             "kernel_share_of_step": round(kern_avg / ms_per_step, 4)}

@@ -14,7 +14,7 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libmagis.so")
 SOURCES = ["magis_graph.cu", "magis_eval.cu", "magis_eval2.cu", "magis_eval2_m0t1.cu", "magis_eval2_m0t2.cu",
-           "magis_eval2_m1.cu", "magis_eval2_m2.cu", "magis_eval2_m3.cu", "magis_eval2_am.cu", "magis_plan.cu", "magis_pareto.cu",
+           "magis_eval2_m1.cu", "magis_eval2_m2.cu", "magis_eval2_m3.cu", "magis_eval2_am.cu", "magis_evalb.cu", "magis_plan.cu", "magis_pareto.cu",
            "magis_gen.cu", "magis_window.cu", "magis_hotspot.cu", "magis_ghash.cu", "magis_hashset.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

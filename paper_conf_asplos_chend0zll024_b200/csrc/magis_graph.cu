@@ -92,6 +92,8 @@ cudaError_t dispatch_eval(const magis_graph* g, int64_t K, const int32_t* perm, 
         }
         return e;
     }
+    if (g->cfg.variant == 3)
+        return evalb_launch(g->dev, g->plan2, g->layb, g->blob2, g->clustersb, K, perm, dec, st, pk, lt, g->evb, s);
     return eval_launch(g->dev, g->cfg, g->gws, K, perm, dec, st, pk, lt, s);
 }
 
@@ -554,6 +556,51 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
             }
         }
     }
+    // --- kernel B (magis_evalb.cu): one candidate per two-CTA cluster, opt-in
+    //     (MAGIS_KERNELB=1; measured against the single-CTA plans)
+    const char* kbenv = std::getenv("MAGIS_KERNELB");
+    if (kbenv && kbenv[0] == '1' && F == 0) {
+        cudaDeviceProp prop;
+        if (cudaGetDeviceProperties(&prop, device) == cudaSuccess) {
+            std::vector<double> rtab((size_t)2 * R);
+            for (int32_t r = 0; r < R; r++) { rtab[2 * r] = tcost[r]; rtab[2 * r + 1] = xfer[r]; }
+            SuperGraphHost sg{n, R, NT, cons_ptr.data(), cons_ent.data(), in_ptr.data(), in_ent.data(),
+                              size.data(), cost.data(), nflag.data(), U_ptr.data(), U_idx.data(), rtab.data(),
+                              elig.data(), F, ngate.data(), nvar.data(), vcost.data()};
+            const size_t cap = (size_t)prop.sharedMemPerBlockOptin - 4096;
+            Plan2 pl;
+            std::vector<char> img;
+            BLayout lay;
+            if (plan2_build(sg, 1, 1, true, false, true, cap, &pl, &img, 2) && evalb_layout(pl, cap, &lay)) {
+                const int clusters = prop.multiProcessorCount / 2;
+                void* b2 = nullptr;
+                void* ev = nullptr;
+                bool ok = cudaMalloc(&b2, img.size()) == cudaSuccess;
+                ok = ok && cudaMemcpy(b2, img.data(), img.size(), cudaMemcpyHostToDevice) == cudaSuccess;
+                ok = ok && cudaMalloc(&ev, evalb_scratch_bytes(pl, clusters)) == cudaSuccess;
+                if (ok) {
+                    if (g->blob2) cudaFree(g->blob2);
+    if (g->evb) cudaFree(g->evb);
+                    if (g->ovf2) { cudaFree(g->ovf2); g->ovf2 = nullptr; }
+                    if (g->afg2) { cudaFree(g->afg2); g->afg2 = nullptr; }
+                    g->plan2 = pl;
+                    g->blob2 = b2;
+                    g->blob2_bytes = img.size();
+                    g->layb = lay;
+                    g->clustersb = clusters;
+                    g->evb = ev;
+                    g->cfg.variant = 3;
+                    g->cfg.grid = 2 * clusters;
+                    g->cfg.block = 512;
+                    g->cfg.smem = lay.total;
+                } else {
+                    cudaGetLastError();
+                    if (b2) cudaFree(b2);
+                    if (ev) cudaFree(ev);
+                }
+            }
+        }
+    }
     if (g->cfg.variant == 1) {
         g->gws_bytes = g->cfg.state_bytes * (size_t)g->cfg.grid;
         e = cudaMalloc(&g->gws, g->gws_bytes);
@@ -576,6 +623,7 @@ extern "C" int magis_graph_free(magis_graph* g) {
     if (g->blob) cudaFree(g->blob);
     if (g->gws) cudaFree(g->gws);
     if (g->blob2) cudaFree(g->blob2);
+    if (g->evb) cudaFree(g->evb);
     if (g->ovf2) cudaFree(g->ovf2);
     if (g->hs_ws) cudaFree(g->hs_ws);
     if (g->afg2) cudaFree(g->afg2);

@@ -219,11 +219,29 @@ struct SuperGraphHost {
 // units, or shared memory).
 bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, bool delta_slots,
                  size_t smem_cap, Plan2* plan,
-                 std::vector<char>* image);
+                 std::vector<char>* image, int row_groups = 1);
 cudaError_t eval2_launch(const DevGraph& g, const Plan2& pl, const void* blob, void* ovf, void* afg, int grid,
                          int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status,
                          int64_t* peak, double* lat, cudaStream_t stream, int32_t* argmax = nullptr);
 cudaError_t eval2_occupancy(const Plan2& pl, int* blocks_per_sm);
+
+// Kernel B (magis_evalb.cu): one candidate per two-CTA cluster, tier-2
+// semantics; a plan built with row_groups = 2.  Shared-memory layout per CTA:
+struct BLayout {
+    int32_t L, S, S0;     // steps per scan chunk, chunks, chunks of CTA 0
+    uint32_t Lm;          // ceil(2^32 / L)
+    int32_t Sl;           // padded per-step delta slots (step st at st + st / L)
+    int32_t nwm;          // u32 words of event-step marks
+    uint32_t stage;       // staged cost-class bytes at offset 0 (0: none)
+    uint32_t pos, D, marks, dec, end, total;
+    uint32_t rec;         // resolved event records [evcap]: u64 key, f64 time, u32 producer
+    int32_t evcap;
+};
+bool evalb_layout(const Plan2& pl, size_t smem_cap, BLayout* lay);
+cudaError_t evalb_launch(const DevGraph& g, const Plan2& pl, const BLayout& lay, const void* blob, int clusters,
+                         int64_t K, const int32_t* perm, const uint8_t* dec, uint8_t* status, int64_t* peak,
+                         double* lat, void* evscratch, cudaStream_t stream);
+size_t evalb_scratch_bytes(const Plan2& pl, int clusters);
 int eval2_block(const Plan2& pl);      // threads per CTA
 
 size_t hotspot_ws_per_cta(const DevGraph& g);
@@ -257,7 +275,10 @@ struct magis_graph {
     void* blob = nullptr;          // device tables
     size_t blob_bytes = 0;
     void* gws = nullptr;           // global per-CTA workspace (variant 1)
-    magis::Plan2 plan2{};          // variant 2 plan
+    magis::Plan2 plan2{};          // variant 2 plan (also kernel B's tables, variant 3)
+    magis::BLayout layb{};         // variant 3 (kernel B) shared-memory layout
+    int clustersb = 0;             // variant 3: two-CTA clusters in the grid
+    void* evb = nullptr;           // variant 3: event scratch
     void* blob2 = nullptr;         // variant 2 static shared-memory image
     size_t blob2_bytes = 0;
     void* ovf2 = nullptr;          // variant 2 event overflow scratch

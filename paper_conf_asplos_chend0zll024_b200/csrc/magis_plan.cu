@@ -100,7 +100,7 @@ Rows make_rows(const std::vector<std::vector<uint32_t>>& lists, const std::vecto
 
 bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, bool gmem_af, bool delta_slots,
                  size_t smem_cap,
-                 Plan2* pl, std::vector<char>* img) {
+                 Plan2* pl, std::vector<char>* img, int row_groups) {
     const int32_t NT = sg.NT, n = sg.n, R = sg.R;
     const int32_t nU = R > 0 ? sg.U_ptr[R] : 0;
     const int64_t NTX = (int64_t)NT + nU + 1;
@@ -163,13 +163,16 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     const uint32_t dummy = (uint32_t)(NTX - 1);
     const uint16_t nop = (uint16_t)dummy;
     const uint32_t nophdr = (kNop << kKindShift) | dummy;
-    Rows cr = make_rows(cons, hdrs, nop, nophdr, WM);
+    // row_groups > 1 (kernel B): rows dealt onto row_groups x WM warps, the
+    // warps of CTA r of a cluster take [r WM, (r + 1) WM)
+    const int WMr = WM * row_groups;
+    Rows cr = make_rows(cons, hdrs, nop, nophdr, WMr);
     // input rows only where the frees are gathered (slots in global memory);
     // with the slots in shared memory phase 3 scatters the frees instead
     Rows fr;
-    if (gmem_af) fr = make_rows(ins, hdrs, nop, nophdr, WM);
-    std::vector<uint32_t> wtab(WM * 4, 0);
-    for (int w = 0; w < WM; w++) {
+    if (gmem_af) fr = make_rows(ins, hdrs, nop, nophdr, WMr);
+    std::vector<uint32_t> wtab(WMr * 4, 0);
+    for (int w = 0; w < WMr; w++) {
         wtab[4 * w + 0] = cr.wtab[2 * w];
         wtab[4 * w + 1] = cr.wtab[2 * w + 1];
         if (gmem_af) {

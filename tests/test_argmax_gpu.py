@@ -57,7 +57,7 @@ def check(g, o, P, D, n, R):
 
 @pytest.fixture(params=["auto", "p2", "tier1p4", "tier2p1", "tier3p2"])
 def variant(request, monkeypatch):
-    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER"):
+    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER", "MAGIS_KERNELB"):
         monkeypatch.delenv(k, raising=False)
     for k, v in VARIANTS[request.param].items():
         monkeypatch.setenv(k, v)

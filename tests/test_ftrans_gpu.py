@@ -33,7 +33,7 @@ REGION_VARIANTS = {"auto": {}, "v1": {"MAGIS_VARIANT": "1"},
 
 @pytest.mark.parametrize("layers,variant", [(2, v) for v in REGION_VARIANTS] + [(24, "auto"), (24, "v1")])
 def test_regions_parity(layers, variant, monkeypatch):
-    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER"):
+    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER", "MAGIS_KERNELB"):
         monkeypatch.delenv(k, raising=False)
     for k, v in REGION_VARIANTS[variant].items():
         monkeypatch.setenv(k, v)

@@ -37,9 +37,9 @@ def wl_of(name):
     return _WL[name]
 
 
-@pytest.fixture(params=["auto", "p2", "tier1p4", "tier2p1", "tier2p4", "tier3p2"])
+@pytest.fixture(params=["auto", "p2", "tier1p4", "tier2p1", "tier2p4", "tier3p2", "kb"])
 def variant(request, monkeypatch):
-    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER"):
+    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER", "MAGIS_KERNELB"):
         monkeypatch.delenv(k, raising=False)
     for k, v in VARIANTS[request.param].items():
         monkeypatch.setenv(k, v)

@@ -32,12 +32,14 @@ VARIANTS = {"auto": {}, "v1": {"MAGIS_VARIANT": "1"}, "p1": {"MAGIS_P": "1", "MA
             "tier1p4": {"MAGIS_TIER": "1", "MAGIS_P": "4", "MAGIS_TEAMS": "1"},
             "tier2p1": {"MAGIS_TIER": "2", "MAGIS_P": "1", "MAGIS_TEAMS": "1"},
             "tier2p4": {"MAGIS_TIER": "2", "MAGIS_P": "4", "MAGIS_TEAMS": "1"},
-            "tier3p2": {"MAGIS_TIER": "3", "MAGIS_P": "2", "MAGIS_TEAMS": "1"}}
+            "tier3p2": {"MAGIS_TIER": "3", "MAGIS_P": "2", "MAGIS_TEAMS": "1"},
+            # kernel B: one candidate per two-CTA cluster (magis_evalb.cu)
+            "kb": {"MAGIS_KERNELB": "1"}}
 
 
 @pytest.fixture(params=list(VARIANTS))
 def variant(request, monkeypatch):
-    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER"):
+    for k in ("MAGIS_VARIANT", "MAGIS_P", "MAGIS_TEAMS", "MAGIS_TIER", "MAGIS_KERNELB"):
         monkeypatch.delenv(k, raising=False)
     for k, v in VARIANTS[request.param].items():
         monkeypatch.setenv(k, v)
@@ -182,6 +184,8 @@ def test_workload_parity(workload, variant):
         assert g.info["pack"] == int(variant[1])
     if variant == "v1":
         assert g.info["variant"] in (0, 1)
+    if variant == "kb":
+        assert g.info["variant"] == 3
     res = gpu_eval(g, P, D)
     ref = o.eval_batch(P, D)
     assert_parity(*res, *ref)
@@ -194,7 +198,7 @@ def test_c4_large_graph_parity(variant):
     gen = CandidateGenerator(wl, CandidateSpec(seed=3))
     P, D = gen.generate(0, 96)
     g = Graph.from_workload(wl)
-    assert g.info["variant"] in (1, 2)
+    assert g.info["variant"] in (1, 2, 3)
     o = OracleGraph.from_workload(wl)
     assert_parity(*gpu_eval(g, P, D), *o.eval_batch(P, D))
 
