@@ -16,7 +16,8 @@
  *   dec[r]:  x = rnd(DEC,r) % 10000; x < p_remat (and t_r has inputs) -> 1;
  *            x < p_remat + p_swap -> 2; else 0
  *   F1: Kahn over the base graph, ready node with the smallest
- *       (key(v) = rnd(KEY,v) >> 32, v) first.
+ *       (key(v) = rnd(KEY,v) >> 48, v) first (a 16-bit priority, ties by id:
+ *       the device generator compares (key, id) as one u32).
  *   F2: natural order; window length w = 2 + rnd(WIN,0) % (wmax-1) (<= n),
  *       start b = rnd(WIN,1) % (n-w+1); the window re-ordered by the same
  *       keyed Kahn restricted to its induced sub-DAG.
@@ -134,7 +135,7 @@ static void keyed_kahn(const gen_cfg *c, gen_ws *w, uint64_t k, int32_t lo, int3
     }
     for (v = lo; v < hi; v++)
         if (w->indeg[v] == 0 && (!w->act || w->act[v]))
-            heap_push(w->heap, &nh, ((rnd(c->seed, k, S_KEY, (uint64_t)v) >> 32) << 32) | (uint32_t)v);
+            heap_push(w->heap, &nh, ((rnd(c->seed, k, S_KEY, (uint64_t)v) >> 48) << 32) | (uint32_t)v);
     while (nh > 0) {
         uint64_t x = heap_pop(w->heap, &nh);
         int32_t u = (int32_t)(x & 0xffffffffu);
@@ -143,7 +144,7 @@ static void keyed_kahn(const gen_cfg *c, gen_ws *w, uint64_t k, int32_t lo, int3
             int32_t s = c->succ_idx[e];
             if (s >= hi || (w->act && !w->act[s])) continue;
             if (--w->indeg[s] == 0)
-                heap_push(w->heap, &nh, ((rnd(c->seed, k, S_KEY, (uint64_t)s) >> 32) << 32) | (uint32_t)s);
+                heap_push(w->heap, &nh, ((rnd(c->seed, k, S_KEY, (uint64_t)s) >> 48) << 32) | (uint32_t)s);
         }
     }
 }

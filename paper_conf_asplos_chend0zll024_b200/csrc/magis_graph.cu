@@ -377,6 +377,46 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
     size_t o_xfer = add(xfer.data(), xfer.size() * 8);
     size_t o_tcost = add(tcost.data(), tcost.size() * 8);
     size_t o_rflag = add(rflag.data(), rflag.size());
+    // generator fast path: sources, and the slot map of the nodes whose base
+    // position places the optional nodes (t_r, pre(t_r), U_r)
+    std::vector<int32_t> gsrc, gqnode;
+    std::vector<uint16_t> gqmap(n, 0xffffu);
+    for (int32_t v = 0; v < n; v++)
+        if (pred_ptr[v + 1] == pred_ptr[v]) gsrc.push_back(v);
+    auto addq = [&](int32_t v) {
+        if (gqmap[v] == 0xffffu && gqnode.size() < 0xffffu) {
+            gqmap[v] = (uint16_t)gqnode.size();
+            gqnode.push_back(v);
+        }
+    };
+    for (int32_t r = 0; r < R; r++) {
+        addq(elig[r]);
+        for (int32_t e = pred_ptr[elig[r]]; e < pred_ptr[elig[r] + 1]; e++) addq(pred[e]);
+        for (int32_t j = U_ptr[r]; j < U_ptr[r + 1]; j++) addq(U_idx[j]);
+    }
+    std::vector<uint32_t> gsinfo((size_t)2 * n), grec((size_t)2 * std::max<int64_t>(E, 1), 0);
+    for (int32_t u = 0; u < n; u++) {
+        gsinfo[2 * u] = (uint32_t)succ_ptr[u];
+        gsinfo[2 * u + 1] = (uint32_t)(succ_ptr[u + 1] - succ_ptr[u]) | ((uint32_t)gqmap[u] << 16);
+        for (int32_t e = succ_ptr[u]; e < succ_ptr[u + 1]; e++) {
+            const int32_t s2 = succ[e];
+            uint32_t o[3] = {0xffffu, 0xffffu, 0xffffu};
+            int no = 0;
+            for (int32_t f = pred_ptr[s2]; f < pred_ptr[s2 + 1]; f++) {
+                if (pred[f] == u) continue;
+                if (no < 3) o[no] = (uint32_t)pred[f];
+                no++;
+            }
+            if (no > 3) o[0] = 0xfffeu;
+            grec[2 * e] = (uint32_t)s2 | (o[0] << 16);
+            grec[2 * e + 1] = o[1] | (o[2] << 16);
+        }
+    }
+    size_t o_gsinfo = add(gsinfo.data(), gsinfo.size() * 4);
+    size_t o_grec = add(grec.data(), grec.size() * 4);
+    size_t o_gsrc = add(gsrc.data(), gsrc.size() * 4);
+    size_t o_gqmap = add(gqmap.data(), gqmap.size() * 2);
+    size_t o_gqnode = add(gqnode.data(), gqnode.size() * 4);
     size_t o_sp = add(succ_ptr.data(), succ_ptr.size() * 4);
     size_t o_s = add(succ.data(), succ.size() * 4);
     size_t o_pp = add(pred_ptr.data(), pred_ptr.size() * 4);
@@ -444,6 +484,14 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
     g->gen.succ = (const int32_t*)(b + o_s);
     g->gen.pred_ptr = (const int32_t*)(b + o_pp);
     g->gen.pred = (const int32_t*)(b + o_p);
+    g->gen.src = (const int32_t*)(b + o_gsrc);
+    g->gen.qmap = (const uint16_t*)(b + o_gqmap);
+    g->gen.qnode = (const int32_t*)(b + o_gqnode);
+    g->gen.sinfo = (const uint2*)(b + o_gsinfo);
+    g->gen.rec = (const uint2*)(b + o_grec);
+    g->gen.S = (int32_t)gsrc.size();
+    g->gen.nq = (int32_t)gqnode.size();
+    g->gen.fast = (n < 0xffff && gqnode.size() < 0xffffu && R < 32768) ? 1 : 0;
 
     e = eval_configure(dg, device, &g->cfg);
     if (e != cudaSuccess) {
@@ -941,18 +989,17 @@ extern "C" int magis_generate_candidates(magis_graph* g, const magis_gen_spec* s
         spec->slack < 0)
         return set_error(MAGIS_E_INVAL, "bad generator spec");
     DeviceGuard guard(g->device);
-    {
-        // scratch for up to one thread per candidate (grown on demand)
-        const int64_t T = gen_threads(g->device, g->dev, K);
-        if (!g->gen_scratch || g->gen_T < T) {
-            if (g->gen_scratch) cudaFree(g->gen_scratch);
-            g->gen_scratch = nullptr;
-            CK(cudaMalloc(&g->gen_scratch, gen_scratch_bytes(g->dev, T)));
-            g->gen_T = T;
-        }
+    // scratch of the launch plan (grown on demand)
+    const GenPlan gp = gen_plan(g->device, g->dev, g->gen, K);
+    if (!g->gen_scratch || g->gen_bytes < gp.bytes) {
+        if (g->gen_scratch) cudaFree(g->gen_scratch);
+        g->gen_scratch = nullptr;
+        g->gen_bytes = 0;
+        CK(cudaMalloc(&g->gen_scratch, gp.bytes));
+        g->gen_bytes = gp.bytes;
     }
     GenSpec sp{spec->seed, spec->pct_random, spec->pct_local, spec->p_remat, spec->p_swap, spec->wmax, spec->slack};
-    cudaError_t e = gen_launch(g->dev, g->gen, sp, id0, K, d_perm, d_dec, g->gen_scratch, g->gen_T,
+    cudaError_t e = gen_launch(g->dev, g->gen, sp, id0, K, d_perm, d_dec, g->gen_scratch, gp,
                                (cudaStream_t)cuda_stream);
     if (e != cudaSuccess) {
         cudaGetLastError();

@@ -131,6 +131,17 @@ struct GenTables {
     const int32_t* succ;
     const int32_t* pred_ptr;   // [n+1]
     const int32_t* pred;
+    // fast path (magis_gen.cu gen2_kernel): sources of G in id order, and the
+    // nodes whose base position the optional-node placement reads (t_r, its
+    // inputs, U_r) as a compact slot map
+    const int32_t* src;        // [S]
+    const uint16_t* qmap;      // [n] slot or 0xffff
+    const int32_t* qnode;      // [nq] node of each slot
+    const uint2* sinfo;        // [n] (successor offset, count | slot << 16)
+    const uint2* rec;          // [E] successor records in succ order: s | o0 << 16, o1 | o2 << 16
+                               //     (the other inputs of s, 0xffff none; o0 = 0xfffe: more than 3)
+    int32_t S, nq;
+    int32_t fast;              // n, nq < 65535 and R < 32768: the fast kernel applies
 };
 
 struct GenSpec {
@@ -138,10 +149,19 @@ struct GenSpec {
     int32_t pct_random, pct_local, p_remat, p_swap, wmax, slack;
 };
 
-size_t gen_scratch_bytes(const DevGraph& g, int64_t T);
-int64_t gen_threads(int device, const DevGraph& g, int64_t K);   // scratch threads for a call of K
+// One launch plan of the generator for a call of K candidates: grid threads of
+// the fast kernel (0: the fast kernel does not apply) and of the sequential
+// kernel (the whole call, or the re-run of the candidates whose ready set
+// outgrew the fast kernel's on-chip heap), and the scratch they need.
+struct GenPlan {
+    int64_t T2 = 0, T1 = 0;
+    int hc = 0, bsm = 0;       // fast kernel: on-chip heap entries, bitset on chip
+    size_t w2 = 0;             // fast kernel scratch bytes per thread
+    size_t bytes = 0;          // total scratch
+};
+GenPlan gen_plan(int device, const DevGraph& g, const GenTables& gt, int64_t K);
 cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp, uint64_t id0, int64_t K,
-                       int32_t* perm, uint8_t* dec, void* scratch, int64_t T, cudaStream_t stream);
+                       int32_t* perm, uint8_t* dec, void* scratch, const GenPlan& gp, cudaStream_t stream);
 
 // Base schedule for windowed delta evaluation (magis_window.cu).
 struct BaseHdr {
@@ -285,7 +305,7 @@ struct magis_graph {
     void* afg2 = nullptr;          // variant 2 per-CTA global step slots (gmem_af)
     magis::GenTables gen{};        // base-graph adjacency (device)
     void* gen_scratch = nullptr;   // candidate generator scratch (lazily allocated)
-    int64_t gen_T = 0;
+    size_t gen_bytes = 0;
     size_t gws_bytes = 0;
     int64_t n_edges = 0;
     int64_t n_super_edges = 0;

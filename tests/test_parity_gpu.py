@@ -321,7 +321,7 @@ def test_pareto_shard_merge_identical_to_single():
 
 # --------------------------------------------------- device generator (a1) --
 
-@pytest.mark.parametrize("cfg", ["c2", "c3", "c5"])
+@pytest.mark.parametrize("cfg", ["c1", "c2", "c3", "c4", "c5"])
 def test_device_generator_bit_exact(cfg):
     """magis_generate_candidates == the CPU generator (magis_inputs) byte for
     byte, on a shard that does not start at id 0."""
@@ -333,6 +333,52 @@ def test_device_generator_bit_exact(cfg):
     torch.cuda.synchronize()
     np.testing.assert_array_equal(Pg.cpu().numpy(), Pc)
     np.testing.assert_array_equal(Dg.cpu().numpy(), Dc)
+
+
+def _gen_both(wl, spec, id0, K):
+    Pc, Dc = CandidateGenerator(wl, spec).generate(id0, K)
+    g = Graph.from_workload(wl)
+    Pg, Dg = g.generate_candidates(id0, K, seed=spec.seed, pct_random=spec.pct_random, pct_local=spec.pct_local,
+                                   p_remat=spec.p_remat, p_swap=spec.p_swap, wmax=spec.wmax, slack=spec.slack)
+    torch.cuda.synchronize()
+    return Pc, Dc, Pg.cpu().numpy(), Dg.cpu().numpy()
+
+
+def test_device_generator_sequential_kernel(monkeypatch):
+    """MAGIS_GEN_SEQ=1 forces the sequential kernel (the fast kernel's re-run
+    path) for the whole call: the same bytes as the CPU generator."""
+    monkeypatch.setenv("MAGIS_GEN_SEQ", "1")
+    wl = build_workload("c2")
+    Pc, Dc, Pg, Dg = _gen_both(wl, CandidateSpec(seed=5), 300, 400)
+    np.testing.assert_array_equal(Pg, Pc)
+    np.testing.assert_array_equal(Dg, Dc)
+
+
+def test_device_generator_heap_overflow_rerun():
+    """A fan-out wider than the fast kernel's on-chip heap (150 nodes ready at
+    once; 64 entries on chip for n <= 3,072): every random-order candidate is
+    flagged and re-generated by the sequential kernel, windows longer than the
+    heap too, and the result is still the CPU generator's, byte for byte; mixed
+    with candidates that stay on the fast kernel in the same launch."""
+    from magis_inputs.graph import Workload
+    rng = np.random.default_rng(3)
+    fan = 150
+    n = fan + 12
+    edges = [(0, i) for i in range(1, fan + 1)] + [(i, fan + 1) for i in range(1, fan + 1)]
+    edges += [(v, v + 1) for v in range(fan + 1, n - 1)]
+    edges += [(v, v + 2) for v in range(fan + 1, n - 2)]
+    size = (rng.integers(1, 1 << 12, n) * 512).astype(np.int64)
+    elig = [fan + 2, fan + 4]
+    U = [[fan + 4], [fan + 6]]
+    wl = Workload("fan", size, rng.uniform(1e-6, 1e-4, n), np.eye(1, n, n - 1, dtype=np.uint8)[0],
+                  np.asarray([u for u, _ in edges], np.int32), np.asarray([v for _, v in edges], np.int32),
+                  [""] * n, ["op"] * n, np.asarray(elig, np.int32), U)
+    for spec in (CandidateSpec(seed=11, p_remat=3000, p_swap=3000),
+                 CandidateSpec(seed=12, pct_random=0, pct_local=100, wmax=n),
+                 CandidateSpec(seed=13, pct_random=50, pct_local=20, wmax=40)):
+        Pc, Dc, Pg, Dg = _gen_both(wl, spec, 7, 3000)
+        np.testing.assert_array_equal(Pg, Pc)
+        np.testing.assert_array_equal(Dg, Dc)
 
 
 def test_device_generator_small_graphs():
