@@ -13,6 +13,7 @@ import pytest
 import oracle
 from oracle import OracleGraph
 from tests import _defn
+from tests.golden import PAPER
 
 
 # ---------------------------------------------------------------- fixtures --
@@ -53,11 +54,11 @@ def test_fig2a_peak_is_1056_at_step_33():
     order = list(range(64))  # f1..f32, b1..b32
     st, peak, lat, arg = g.eval(order)
     assert st == 0
-    assert peak == 1056
-    assert arg == 32            # 0-based step 32 == the 33rd operator
+    assert peak == PAPER["fig2a.peak"] == PAPER["fig2a.live_tensors_at_peak"] * PAPER["fig2a.tensor_size"]
+    assert arg == PAPER["fig2a.peak_operator"] - 1     # 0-based step 32 == the 33rd operator
     # the independent interval-sum definition agrees
     pk, a2 = _defn.interval_peak(order, edges, dict(enumerate(size)), set(outs))
-    assert (pk, a2) == (1056, 32)
+    assert (pk, a2) == (PAPER["fig2a.peak"], PAPER["fig2a.peak_operator"] - 1)
 
 
 def test_fig2a_literal_formula_is_off_by_one():
@@ -90,10 +91,10 @@ def test_fig2b_swapping_peak_is_96():
     assert sorted(order) == list(range(n + 3 * R))
     dec = np.full(R, 2, np.uint8)
     st, peak, lat, arg = g.eval(order, dec)
-    assert st == 0 and peak == 96
+    assert st == 0 and peak == PAPER["fig2b.peak"] <= PAPER["fig2b.memory_limit"]
     # forward phase alone peaks at 64
     st2, pk2 = _defn.defn_eval(n, edges, size, outs, elig, U, dec, order)
-    assert (st2, pk2) == (0, 96)
+    assert (st2, pk2) == (0, PAPER["fig2b.peak"])
 
 
 # ------------------------------------------------ hand-computed toy timelines --
@@ -477,12 +478,12 @@ def test_eq1_reproduces_fig2_cde():
     hot = [f"h{i}" for i in range(33)]
     for h in hot:
         size[h] = 32
-    assert oracle.eq1_estimate(H=hot, S=hot, I=[X], size=size, n=16) == 98.0
+    assert oracle.eq1_estimate(H=hot, S=hot, I=[X], size=size, n=16) == PAPER["fig2c.peak"]
     hot3 = hot[:3]
-    assert oracle.eq1_estimate(H=hot3, S=hot3, I=[X], size=size, n=4) == 56.0
+    assert oracle.eq1_estimate(H=hot3, S=hot3, I=[X], size=size, n=4) == PAPER["fig2d.peak"]
     size["s8"] = 8
-    assert oracle.eq1_estimate(H=hot3, S=hot3, I=[X, "s8"], size=size, n=8) == 52.0
-    assert oracle.eq1_m0(hot, size) == 1056.0
+    assert oracle.eq1_estimate(H=hot3, S=hot3, I=[X, "s8"], size=size, n=8) == PAPER["fig2e.peak"]
+    assert oracle.eq1_m0(hot, size) == PAPER["fig2a.peak"]
 
 
 # ------------------------------------------------------------------ Pareto --
