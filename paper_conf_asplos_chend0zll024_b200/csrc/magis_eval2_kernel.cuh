@@ -138,8 +138,10 @@ __device__ __forceinline__ void bar_arrive(int id, int n) {
 }
 
 // ------------------------------------------------- bulk copy (TMA engine) --
+// one or two global ranges -> shared memory (sizes and addresses 16-byte aligned)
 __device__ __forceinline__ void bulk_stage(void* smem_dst, const void* gsrc, uint32_t bytes,
-                                           uint64_t* mbar) {
+                                           uint64_t* mbar, void* smem_dst2 = nullptr,
+                                           const void* gsrc2 = nullptr, uint32_t bytes2 = 0) {
     const uint32_t bar = (uint32_t)__cvta_generic_to_shared(mbar);
     if (threadIdx.x == 0) {
         asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(bar) : "memory");
@@ -147,15 +149,20 @@ __device__ __forceinline__ void bulk_stage(void* smem_dst, const void* gsrc, uin
     }
     __syncthreads();
     if (threadIdx.x == 0) {
-        asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+        asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes + bytes2) : "memory");
         const uint32_t chunk = 1u << 15;
-        for (uint32_t o = 0; o < bytes; o += chunk) {
-            const uint32_t nb = min(chunk, bytes - o);
-            const uint32_t dst = (uint32_t)__cvta_generic_to_shared((char*)smem_dst + o);
-            asm volatile(
-                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-                "l"((const char*)gsrc + o), "r"(nb), "r"(bar)
-                : "memory");
+        for (int part = 0; part < 2; part++) {
+            char* d = (char*)(part ? smem_dst2 : smem_dst);
+            const char* src = (const char*)(part ? gsrc2 : gsrc);
+            const uint32_t nbytes = part ? bytes2 : bytes;
+            for (uint32_t o = 0; o < nbytes; o += chunk) {
+                const uint32_t nb = min(chunk, nbytes - o);
+                const uint32_t dst = (uint32_t)__cvta_generic_to_shared(d + o);
+                asm volatile(
+                    "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+                    "l"(src + o), "r"(nb), "r"(bar)
+                    : "memory");
+            }
         }
     }
     uint32_t done = 0;
@@ -377,12 +384,16 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     // read in place from the global image when they do not fit
     const char* sb = MODE ? blob : sm_all;
     if (MODE == 0) bulk_stage(sm_all, blob, pl.static_bytes, &mbar);
-    else if (pl.cost_sm) bulk_stage(sm_all, blob + (pl.cost_cls ? pl.off_ccls : pl.off_cost), pl.stage_bytes, &mbar);
-    const uint32_t* wtab = (const uint32_t*)(sb + pl.off_wtab);   // [WM][4]: consumer rows, input rows
-    const uint2* crow = (const uint2*)(sb + pl.off_crow);
-    const uint32_t* chdr = (const uint32_t*)(sb + pl.off_chdr);
+    else if (pl.cost_sm)
+        bulk_stage(sm_all, blob + (pl.cost_cls ? pl.off_ccls : pl.off_cost), pl.stage_bytes, &mbar,
+                   sm_all + pl.rows_off, blob + pl.off_wtab, pl.rows_bytes);
+    // tier 1 with rows_sm: the consumer-row tables [wtab, crow, chdr, cent] were staged too
+    const char* sr = (MODE == 1 && pl.rows_sm) ? (const char*)sm_all + pl.rows_off - pl.off_wtab : sb;
+    const uint32_t* wtab = (const uint32_t*)(sr + pl.off_wtab);   // [WM][4]: consumer rows, input rows
+    const uint2* crow = (const uint2*)(sr + pl.off_crow);
+    const uint32_t* chdr = (const uint32_t*)(sr + pl.off_chdr);
     const uint32_t* csize = (const uint32_t*)(sb + pl.off_csize);   // size units of each header, row order
-    const uint16_t* cent = (const uint16_t*)(sb + pl.off_cent);
+    const uint16_t* cent = (const uint16_t*)(sr + pl.off_cent);
     const uint2* frow = (const uint2*)(sb + pl.off_frow);
     const uint32_t* fhdr = (const uint32_t*)(sb + pl.off_fhdr);
     const uint16_t* fent = (const uint16_t*)(sb + pl.off_fent);
@@ -390,7 +401,7 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     const double2* rtab = (const double2*)(sb + pl.off_rtab);       // [R] (cost(t_r), swap transfer time)
     const double* cost_s = (MODE != 0 && pl.cost_sm) ? (const double*)sm_all : (const double*)(sb + pl.off_cost);
     // tier 2 with cost classes: cost(v) = class value [class index of v], both staged
-    const bool ccls = MODE == 3 && pl.cost_sm && pl.cost_cls;
+    const bool ccls = (MODE == 1 || MODE == 3) && pl.cost_sm && pl.cost_cls;
     const uint8_t* ccls_idx = (const uint8_t*)(sm_all + pl.ccls_idx_off);
     const uint2* ninfo = (const uint2*)(sb + pl.off_ninfo);
     const uint16_t* lul = (const uint16_t*)(sb + pl.off_lul);
@@ -501,6 +512,9 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 } else {
                     const double* woff = lwoff[c];
                     const int ne = h.nev[c];
+#ifdef MAGIS_ABL_WALK
+                    if (true) { lat = ctot; } else   // ablation (timing only): no latency walk
+#endif
                     if (ne <= cap) {
                         const size_t b0 = (size_t)(slot * P + c) * cap;
                         unsigned long long* key = evk_s + b0;
@@ -1022,7 +1036,11 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     }
                 }
             }
+#ifdef MAGIS_ABL_COST
+            if (false) {                     // ablation (timing only): no swap cost loop / events
+#else
             if (mysw) {
+#endif
                 // swapping candidate: compute-cost prefix (two partial sums
                 // halve the dependent fp64 chain) and the chunk's event steps in
                 // step order; an inactive clone (pos 0) costs nothing

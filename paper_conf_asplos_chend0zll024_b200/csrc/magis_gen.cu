@@ -132,6 +132,7 @@ gen_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32_
         int32_t* perm = perms + kk * (int64_t)NT;
         uint8_t* dec = decs + kk * (int64_t)(R ? R : 1);
         const uint32_t fam = (uint32_t)(rnd(seed, k, S_FAM, 0) % 100u);
+        if (R == 0) dec[0] = 0;                          // the row's pad byte (no decisions)
         for (int32_t r = 0; r < R; r++) {
             const uint32_t x = (uint32_t)(rnd(seed, k, S_DEC, (uint64_t)r) % 10000u);
             const int32_t tr = g.elig[r];
@@ -263,6 +264,7 @@ gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32
         int32_t* perm = perms + kk * (int64_t)NT;
         uint8_t* dec = decs + kk * (int64_t)(R ? R : 1);
         const uint32_t fam = (uint32_t)(mix64(hk[S_FAM]) % 100u);
+        if (R == 0) dec[0] = 0;                          // the row's pad byte (no decisions)
         for (int32_t r = 0; r < R; r++) {
             const uint32_t x = (uint32_t)(mix64(hk[S_DEC] ^ (uint64_t)r) % 10000u);
             const int32_t tr = g.elig[r];

@@ -549,6 +549,20 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
                             std::fprintf(stderr,
                                          "[magis] plan tier=%d teams=%d P=%d L=%d S=%d smem=%u static=%u occ=%d err=%d\n",
                                          tier, T, P, pl.L, pl.S, pl.smem_total, pl.static_bytes, occ, (int)oe);
+                        if (std::getenv("MAGIS_DEBUG") && std::atoi(std::getenv("MAGIS_DEBUG")) > 1)
+                            std::fprintf(stderr,
+                                         "[magis]   tables: wtab %u crow %u chdr %u csize %u cent %u (rows_sm %d) frow %u fhdr %u fent %u "
+                                         "size %u cost %u rtab %u ninfo %u lul %u urow %u ubs %u utr %u rn %u | state: pos %u "
+                                         "last %u af %u dec %u end %u evm %u sdec %u ev %u (cap %d) stage %u\n",
+                                         pl.off_crow - pl.off_wtab, pl.off_chdr - pl.off_crow, pl.off_cent - pl.off_chdr,
+                                         pl.off_frow - pl.off_csize, pl.off_csize - pl.off_cent, pl.rows_sm, pl.off_fhdr - pl.off_frow,
+                                         pl.off_fent - pl.off_fhdr, pl.off_size - pl.off_fent, pl.off_cost - pl.off_size,
+                                         pl.off_rtab - pl.off_cost, pl.off_ninfo - pl.off_rtab, pl.off_lul - pl.off_ninfo,
+                                         pl.off_urow - pl.off_lul, pl.off_ubs - pl.off_urow, pl.off_utr - pl.off_ubs,
+                                         pl.off_rn - pl.off_utr, pl.off_nvar - pl.off_rn, pl.off_last - pl.off_pos,
+                                         pl.off_af - pl.off_last, pl.off_dec - pl.off_af, pl.off_end - pl.off_dec,
+                                         pl.off_evm - pl.off_end, pl.off_sdec - pl.off_evm, pl.off_ev - pl.off_sdec,
+                                         pl.smem_total - pl.off_ev, pl.evcap, pl.stage_bytes);
                         if (oe != cudaSuccess || occ < 1) { cudaGetLastError(); continue; }
                         const int a = P * T * occ, b = bestP * bestT * bestOcc;
                         if (a > b || (a == b && (T < bestT || (T == bestT && occ > bestOcc)))) {

@@ -104,6 +104,8 @@ struct Plan2 {
     uint32_t off_ccls;       // image offset of [class values f64 (a16) | class index u8 [NTX]]
     uint32_t ccls_idx_off;   // offset of the class index inside that region
     uint32_t stage_bytes;    // bytes staged into shared memory on tiers 1 / 2 (cost table or classes)
+    int32_t rows_sm;         // tier 1: [wtab, crow, chdr, cent] also staged, at shared offset rows_off
+    uint32_t rows_off, rows_bytes;
     uint32_t image_bytes;    // whole device image (static_bytes staged on tier 0, then the class tables)
     uint32_t off_pos, off_last, off_af, off_dec, off_end;
     uint32_t off_evm;        // [P][NW] swap-event step marks (bit per step)

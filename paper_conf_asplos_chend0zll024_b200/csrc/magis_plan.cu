@@ -210,8 +210,9 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     p.off_wtab = (uint32_t)o;  o = a16(o + wtab.size() * 4);
     p.off_crow = (uint32_t)o;  o = a16(o + cr.row.size() * 4);
     p.off_chdr = (uint32_t)o;  o = a16(o + cr.hdr.size() * 4);
-    p.off_csize = (uint32_t)o; o = a16(o + cr.hdr.size() * 4);   // size units of each header, row order
     p.off_cent = (uint32_t)o;  o = a16(o + cr.ent.size() * 2);
+    // [wtab, crow, chdr, cent] contiguous: the row tables tier 1 may stage
+    p.off_csize = (uint32_t)o; o = a16(o + cr.hdr.size() * 4);   // size units of each header, row order
     p.off_frow = (uint32_t)o;  o = a16(o + fr.row.size() * 4);
     p.off_fhdr = (uint32_t)o;  o = a16(o + fr.hdr.size() * 4);
     p.off_fent = (uint32_t)o;  o = a16(o + fr.ent.size() * 2);
@@ -237,10 +238,10 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     std::vector<double> cvals(cost_u.begin(), cost_u.end());
     std::sort(cvals.begin(), cvals.end());
     cvals.erase(std::unique(cvals.begin(), cvals.end()), cvals.end());
-    p.cost_cls = (delta_slots && cvals.size() <= 256) ? 1 : 0;   // tier 1: +2.6% time (A/B), not used
+    const bool have_cls = cvals.size() <= 256;
     p.off_ccls = (uint32_t)o;
     p.ccls_idx_off = (uint32_t)a16(cvals.size() * 8);
-    if (p.cost_cls) o = a16(o + p.ccls_idx_off + (size_t)NTX);
+    if (have_cls) o = a16(o + p.ccls_idx_off + (size_t)NTX);
     p.image_bytes = (uint32_t)o;
     // graph tables in shared memory (staged) or read from the global image
     // (L1/L2; the row reads stay coalesced); per-step slots in shared memory or
@@ -254,10 +255,30 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     const size_t static_end = o;
     // tables read from the global image: the cost table (the swap scan's
     // random gather) is still staged into shared memory when it fits with
-    // at least 32 event slots per candidate
-    for (int csm = gmem_static ? 1 : 0; csm >= 0; csm--) {
+    // at least 32 event slots per candidate.  Tier 1 first tries to stage the
+    // consumer-row tables too ([wtab, crow, chdr, cent]; the row sizes stay in
+    // global memory, loaded a row ahead), with the cost table as u8 classes to
+    // make room: the row pass then gathers from shared memory only (rows_sm).
+    struct Att { int rs, csm; };
+    Att atts[3];
+    int na = 0;
+    const char* nors = std::getenv("MAGIS_NO_ROWSM");
+    if (gmem_static) {
+        if (!delta_slots && !gmem_af && have_cls && !(nors && std::atoi(nors) != 0)) atts[na++] = {1, 1};
+        atts[na++] = {0, 1};
+        atts[na++] = {0, 0};
+    } else {
+        atts[na++] = {0, 0};
+    }
+    bool planned = false;
+    for (int ai = 0; ai < na; ai++) {
+    const int csm = atts[ai].csm;
+    p.rows_sm = atts[ai].rs;
+    p.cost_cls = (have_cls && (delta_slots || p.rows_sm)) ? 1 : 0;   // tier 1 without rows_sm: f64 (classes +2.6%, A/B)
     p.stage_bytes = (uint32_t)(p.cost_cls ? a16(p.ccls_idx_off + (size_t)NTX) : a16((size_t)NTX * 8));
-    o = gmem_static ? (csm ? (size_t)p.stage_bytes : 0) : static_end;
+    p.rows_off = p.stage_bytes;
+    p.rows_bytes = p.rows_sm ? (uint32_t)(p.off_csize - p.off_wtab) : 0u;
+    o = gmem_static ? (csm ? (size_t)p.stage_bytes + p.rows_bytes : 0) : static_end;
     p.cost_sm = csm;
     p.state_base = (uint32_t)o;
     // pos: NTX slots + one trash slot (out-of-range ids of a bad permutation
@@ -287,13 +308,12 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
         if (cap <= (csm ? 32 : 8)) break;
         cap /= 2;
     }
-    if (!fit) {
-        if (csm) continue;
-        return false;
-    }
+    if (!fit) continue;
     p.evcap = cap;
+    planned = true;
     break;
     }
+    if (!planned) return false;
     p.ovf_stride = (uint64_t)((std::max(p.max_events, 1) * 24 + 255) / 256 * 256);
     *pl = p;
     img->assign(p.image_bytes, 0);
@@ -315,7 +335,7 @@ bool plan2_build(const SuperGraphHost& sg, int P, int teams, bool gmem_static, b
     put(p.off_fent, fr.ent.data(), fr.ent.size() * 2);
     put(p.off_size, size_u.data(), size_u.size() * 4);
     put(p.off_cost, cost_u.data(), cost_u.size() * 8);
-    if (p.cost_cls) {
+    if (have_cls) {
         put(p.off_ccls, cvals.data(), cvals.size() * 8);
         std::vector<uint8_t> ci(NTX);
         for (int64_t v = 0; v < NTX; v++)
