@@ -571,15 +571,24 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
     constexpr int LR = LMAX <= kRegL ? LMAX : 1;
     int32_t pr[LR];
     // this thread's chunk of candidate cm of group grp_ (-1 past the end)
+    // the chunk's alignment in its row (warp-uniform: a warp serves one
+    // candidate): 16-byte vectors when the row offset allows, else 8-byte
+    // pairs (n_total even), else scalars; a vector never reads past the row
     auto load_chunk = [&](int64_t grp_) {
         const bool vc = grp_ * P + cm < K;
-        const int32_t* Pp = perm + (grp_ * P + cm) * (int64_t)NT + lo;
+        const int64_t eo = (grp_ * P + cm) * (int64_t)NT + lo;
+        const int32_t* Pp = perm + eo;
+        const bool a16 = vec4 || (eo & 3) == 0, a8 = (eo & 1) == 0;
 #pragma unroll
         for (int j = 0; j < LR; j += 4) {
             int4 v = make_int4(-1, -1, -1, -1);
             if (vc && j < L && lo + j < NT) {
-                if (vec4) {
+                if (vec4 || (a16 && lo + j + 3 < NT)) {
                     v = __ldcs(reinterpret_cast<const int4*>(Pp + j));
+                } else if (a8 && lo + j + 3 < NT) {
+                    const int2 x = __ldcs(reinterpret_cast<const int2*>(Pp + j));
+                    const int2 y = __ldcs(reinterpret_cast<const int2*>(Pp + j + 2));
+                    v = make_int4(x.x, x.y, y.x, y.y);
                 } else {
                     v.x = __ldcs(Pp + j);
                     if (lo + j + 1 < NT) v.y = __ldcs(Pp + j + 1);
@@ -674,13 +683,19 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                 }
             } else {
                 // (default caching: the swap cost loop of phase 5 reads the chunk again)
-                const int32_t* Pp = perm + (grp * P + cm) * (int64_t)NT + lo;
+                const int64_t eo = (grp * P + cm) * (int64_t)NT + lo;
+                const int32_t* Pp = perm + eo;
+                const bool a16 = vec4 || (eo & 3) == 0, a8 = (eo & 1) == 0;
 #pragma unroll
                 for (int j = 0; j < LMAX; j += 4) {
                     if (vc && j < L && lo + j < NT) {
                         int4 v = make_int4(-1, -1, -1, -1);
-                        if (vec4) {
+                        if (vec4 || (a16 && lo + j + 3 < NT)) {
                             v = __ldg(reinterpret_cast<const int4*>(Pp + j));
+                        } else if (a8 && lo + j + 3 < NT) {
+                            const int2 x = __ldg(reinterpret_cast<const int2*>(Pp + j));
+                            const int2 y = __ldg(reinterpret_cast<const int2*>(Pp + j + 2));
+                            v = make_int4(x.x, x.y, y.x, y.y);
                         } else {
                             v.x = __ldg(Pp + j);
                             if (lo + j + 1 < NT) v.y = __ldg(Pp + j + 1);
