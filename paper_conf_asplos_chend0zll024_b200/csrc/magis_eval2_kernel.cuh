@@ -1079,13 +1079,30 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
                     // perm chunk re-read from global: batches of 8 steps with the perm
                     // and cost loads issued ahead of the event stores (which the
                     // compiler cannot move loads across)
-                    const int32_t* pp = perm + (grp * P + cm) * (int64_t)NT + lo;
+                    const int64_t eo = (grp * P + cm) * (int64_t)NT + lo;
+                    const int32_t* pp = perm + eo;
+                    const bool a16 = vec4 || (eo & 3) == 0, a8 = (eo & 1) == 0;
                     for (int jb = 0; jb < LMAX; jb += 8) {
                         if (jb >= nst) break;
                         int32_t vv[8];
                         double cv[8];
+                        if (jb + 8 <= nst && (a16 || a8)) {              // last read, as vectors
+                            if (a16) {
+                                const int4 x = __ldcs(reinterpret_cast<const int4*>(pp + jb));
+                                const int4 y = __ldcs(reinterpret_cast<const int4*>(pp + jb + 4));
+                                vv[0] = x.x; vv[1] = x.y; vv[2] = x.z; vv[3] = x.w;
+                                vv[4] = y.x; vv[5] = y.y; vv[6] = y.z; vv[7] = y.w;
+                            } else {
 #pragma unroll
-                        for (int u = 0; u < 8; u++) vv[u] = jb + u < nst ? __ldcs(pp + jb + u) : 0;   // last read
+                                for (int u = 0; u < 8; u += 2) {
+                                    const int2 x = __ldcs(reinterpret_cast<const int2*>(pp + jb + u));
+                                    vv[u] = x.x; vv[u + 1] = x.y;
+                                }
+                            }
+                        } else {
+#pragma unroll
+                            for (int u = 0; u < 8; u++) vv[u] = jb + u < nst ? __ldcs(pp + jb + u) : 0;   // last read
+                        }
 #pragma unroll
                         for (int u = 0; u < 8; u++)
                             cv[u] = jb + u < nst ? (ccls ? cost_s[ccls_idx[vv[u]]] : cost_s[vv[u]]) : 0.0;
