@@ -18,6 +18,16 @@ for cfg in c2 c5; do
     run racecheck $cfg 512 MAGIS_TEAMS=1 $tv
   done
 done
+# tier 1 with the staged row tables (rows_sm) and the device generator (a1)
+run synccheck c3 512 MAGIS_TIER=1
+run racecheck c3 256 MAGIS_TIER=1
+gen() {  # tool cfg K
+  res=$(timeout 1200 compute-sanitizer --tool $1 python scripts/dbg_gen.py $2 $3 2>&1 | grep -E "mismatches|SUMMARY|Error|error" | tr '\n' ' ')
+  echo "$1 generator $2 K=$3 :: $res" | tee -a $out
+}
+gen memcheck c2 1024
+gen racecheck c2 512
+gen memcheck c4 128
 run memcheck c4 256
 run synccheck c4 256
 run racecheck c4 160
