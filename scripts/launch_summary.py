@@ -5,7 +5,7 @@ import collections
 import csv
 import sys
 
-SETUP = ("gen_kernel", "at::", "widen", "base_kernel")
+SETUP = ("gen_kernel", "gen2_kernel", "at::", "widen", "base_kernel")
 rows = [r for r in csv.reader(open(sys.argv[1])) if len(r) > 5]
 h = rows[0]
 ki, mi, vi, ui = h.index("Kernel Name"), h.index("Metric Name"), h.index("Metric Value"), h.index("Metric Unit")
