@@ -615,10 +615,28 @@ eval2_kernel(DevGraph g, Plan2 pl, const char* __restrict__ blob, int64_t K,
         dq1 = (tid + TM < P * Rd && b + tid + TM < lim) ? (uint32_t)__ldcs(dec + b + tid + TM) : 0u;
     };
     if (dreg && Rd > 0 && ncta > 0) load_dec(cta);
+    // streamed perm (tier 2, chunks longer than the register budget): the perm
+    // rows of the group two ahead are pulled into L2 by the bulk-copy engine
+    // (no registers, no shared memory), so phase 1 reads them from L2 (A/B: C4
+    // -1.9%; with the chunk prefetched into registers it is neutral to +1.2%)
+    constexpr bool kL2Pf = LMAX > kRegL;
+    auto l2_prefetch = [&](int64_t grp_) {
+        const int64_t k0 = grp_ * P, k1 = min(K, k0 + P);
+        if (k0 >= K) return;
+        uint64_t a = (uint64_t)(perm + k0 * (int64_t)NT), e = (uint64_t)(perm + k1 * (int64_t)NT);
+        a = (a + 15) & ~15ull;                       // whole 16-byte units inside the rows
+        e &= ~15ull;
+        for (; a + 16 <= e; a += 32768) {
+            const uint32_t nb = (uint32_t)min((uint64_t)32768, e - a);
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"(nb) : "memory");
+        }
+    };
+    if (kL2Pf && tid == 0 && ncta > 1) l2_prefetch(cta + ncta_all);
     for (int gi = 0; gi < ncta; gi++) {
         const int64_t grp = cta + (int64_t)gi * ncta_all;
         const int slot = gi & 1;
         Ctl& cl = ctl[slot];
+        if (kL2Pf && tid == 0 && gi + 2 < ncta) l2_prefetch(grp + 2 * ncta_all);
         // candidate c of this group exists iff bit c of vmask is set
         const int64_t kleft = K - grp * P;
         const uint32_t vmask = kleft >= P ? ((1u << P) - 1u) : ((1u << (uint32_t)kleft) - 1u);
