@@ -229,6 +229,13 @@ __device__ __forceinline__ uint32_t ent_of(uint64_t hk, uint32_t v) { return ((u
 constexpr int kGenHC = 32;        // heap entries on chip per thread (more spill to the thread's global slice)
 constexpr int kGenHG = 1024;      // spill entries; a larger ready set re-runs the candidate on gen_kernel
 
+// graph tables: read-only path, kept in L1 ahead of the per-thread scratch
+__device__ __forceinline__ uint2 ld_tab(const uint2* p) {
+    uint2 r;
+    asm volatile("ld.global.nc.L1::evict_last.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+    return r;
+}
+
 template <bool BSM>
 __global__ void __launch_bounds__(128)
 gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32_t* __restrict__ perms,
@@ -353,11 +360,11 @@ gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32
             return emitted(o0, lo) & emitted(rc.y & 0xffffu, lo) & emitted(rc.y >> 16, lo);
         };
         auto visit = [&](int32_t u, int32_t m, int32_t hi, int32_t lo) {
-            const uint2 si = __ldg(gt.sinfo + u);
+            const uint2 si = ld_tab(gt.sinfo + u);
             const uint32_t cnt = si.y & 0xffffu, qs = si.y >> 16;
             if (qs != 0xffffu) Q[qs] = (uint16_t)m;
             for (uint32_t e = 0; e < cnt; e++) {
-                const uint2 rc = __ldg(gt.rec + si.x + e);
+                const uint2 rc = ld_tab(gt.rec + si.x + e);
                 const int32_t s = (int32_t)(rc.x & 0xffffu);
                 if (s >= hi || !ready(rc, u, lo)) continue;
                 if (nh >= HC + kGenHG) { over = true; return; }
@@ -473,7 +480,7 @@ gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32
                 while ((int32_t)gnext == i) {
                     const uint32_t o = opt[oi++];
                     const int32_t rr = (int32_t)(o & 0x7fffu);
-                    perm[m++] = ((o >> 15) & 1u) == 0 ? n + 3 * rr + 1 : (dec[rr] == 2 ? n + 3 * rr + 2 : n + 3 * rr);
+                    __stcs(perm + m++, ((o >> 15) & 1u) == 0 ? n + 3 * rr + 1 : (dec[rr] == 2 ? n + 3 * rr + 2 : n + 3 * rr));
                     gnext = oi < nopt ? (opt[oi] >> 16) : 0xffffffffu;
                 }
             };
@@ -485,21 +492,21 @@ gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32
 #pragma unroll
                     for (int j = 0; j < 8; j++) {
                         emit_opts(i0 + j);
-                        perm[m++] = (int32_t)((w4[j >> 1] >> (16 * (j & 1))) & 0xffffu);
+                        __stcs(perm + m++, (int32_t)((w4[j >> 1] >> (16 * (j & 1))) & 0xffffu));
                     }
                 }
-                for (int32_t i = n8; i < n; i++) { emit_opts(i); perm[m++] = bs[i]; }
+                for (int32_t i = n8; i < n; i++) { emit_opts(i); __stcs(perm + m++, (int32_t)bs[i]); }
             } else {
                 for (int32_t i = 0; i < n; i++) {
                     emit_opts(i);
-                    perm[m++] = (i >= lo && i < hi) ? (int32_t)bs[i - lo] : i;
+                    __stcs(perm + m++, (i >= lo && i < hi) ? (int32_t)bs[i - lo] : i);
                 }
             }
             emit_opts(n);
             for (int32_t r = 0; r < R; r++) {
                 const uint8_t d = dec[r];
-                if (d != 1) perm[m++] = n + 3 * r;
-                if (d != 2) { perm[m++] = n + 3 * r + 1; perm[m++] = n + 3 * r + 2; }
+                if (d != 1) __stcs(perm + m++, n + 3 * r);
+                if (d != 2) { __stcs(perm + m++, n + 3 * r + 1); __stcs(perm + m++, n + 3 * r + 2); }
             }
         }
         if ((int32_t)fam >= sp.pct_random + sp.pct_local) {
@@ -545,12 +552,41 @@ GenPlan gen_plan(int device, const DevGraph& g, const GenTables& gt, int64_t K) 
         const size_t smem = (size_t)kGenTB * (p.hc + (p.bsm ? NW : 0)) * 4;
         const void* fn = gen2_select(p.bsm);
         cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        // the attribute persists per kernel: start from the all-shared carveout
+        // (an earlier call on a smaller graph may have lowered it)
+        cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
         int per = 0;
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, kGenTB, smem) != cudaSuccess || per < 1) {
             cudaGetLastError();
             per = 1;
         }
         const int64_t cand = (K + kGenTB - 1) / kGenTB * kGenTB;
+        // the rest of the SM's unified memory stays L1 for the graph tables:
+        // ask for the shared-memory carveout of the blocks one wave needs
+        {
+            const int64_t need = std::min<int64_t>(per, (cand / kGenTB + sms - 1) / sms);
+            const size_t bytes = (size_t)need * (smem + 1024);
+            const int pct = (int)std::min<size_t>(100, (bytes * 100 + 228 * 1024 - 1) / (228 * 1024));
+            // (only when it leaves L1 at least 32 KB: C5's 4 x 57 KB at 99% measured
+            // 9.6 -> 13.1 ms; C2 6.1 -> 5.2, C3 30.8 -> 26.2, C4 199 -> 176 ms)
+            const char* cv = std::getenv("MAGIS_GEN_CARVE");
+            const int want = cv ? std::atoi(cv) : (bytes + 32 * 1024 <= 228 * 1024 ? std::max(pct, 1) : 100);
+            cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, want);
+            int per2 = 0;
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per2, fn, kGenTB, smem) != cudaSuccess) {
+                cudaGetLastError();
+                per2 = 0;
+            }
+            if (per2 >= need) {
+                per = per2;
+            } else {                                   // the rounded carveout holds fewer blocks: all shared
+                cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+                if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per2, fn, kGenTB, smem) == cudaSuccess && per2 >= 1)
+                    per = per2;
+                else
+                    cudaGetLastError();
+            }
+        }
         p.T2 = std::min<int64_t>((int64_t)sms * per * kGenTB, cand);
         const size_t nb = (size_t)1 << gen_lgnb(gt);
         p.w2 = ((size_t)gt.S * 4 + 15) / 16 * 16 + ((nb + 1 + 7) & ~(size_t)7) * 2 + (((size_t)gt.nq + 7) & ~(size_t)7) * 2 +
