@@ -548,7 +548,8 @@ GenPlan gen_plan(int device, const DevGraph& g, const GenTables& gt, int64_t K) 
     if (gt.fast && !(off && std::atoi(off) != 0)) {
         const int32_t NW = (g.n + 31) >> 5;
         p.hc = kGenHC;
-        p.bsm = NW <= 96 ? 1 : 0;
+        const char* bf = std::getenv("MAGIS_GEN_BSM");
+        p.bsm = bf ? (std::atoi(bf) != 0 && NW <= 96) : (NW <= 96 ? 1 : 0);
         const size_t smem = (size_t)kGenTB * (p.hc + (p.bsm ? NW : 0)) * 4;
         const void* fn = gen2_select(p.bsm);
         cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
