@@ -256,6 +256,7 @@ gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32
     uint32_t* gbits = (uint32_t*)(bs + (((size_t)n + 7) & ~(size_t)7));            // [NW] (!BSM)
     uint32_t* opt = gbits + (BSM ? 0 : ((NW + 3) & ~3));                           // [2R]
     uint32_t* hg = opt + ((2 * (R ? R : 1) + 3) & ~3) - HC;                        // heap entry i >= HC at hg[i]
+    uint16_t* wc = (uint16_t*)(hg + HC + kGenHG);                                   // [W] emitted inputs of wide nodes
     auto bw = [&](int32_t w) -> uint32_t& { if constexpr (BSM) return smg[(HC + w) * TB + tid]; else return gbits[w]; };
     auto hat = [&](int32_t i) -> uint32_t& { return i < HC ? hp[i * TB] : hg[i]; };
     // per-stream prefixes mix64(seed + G (stream + 1)), shared by all candidates
@@ -347,8 +348,17 @@ gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32
         };
         // successor record of edge u -> s: every other input of s emitted
         // (inputs below lo count as emitted: the window's prefix)
+        bool wide_ok = false;                            // wide-node counters zeroed (F1 / F3)
         auto ready = [&](uint2 rc, int32_t u, int32_t lo) -> bool {
             const uint32_t o0 = rc.x >> 16;
+            if (o0 == 0xfffeu && wide_ok && (rc.y & 0xffffu) != 0xffffu) {
+                // wide node (C4's 32-input merges): count its emitted inputs
+                // instead of scanning them at every input's emission
+                const uint32_t slot = rc.y & 0xffffu;
+                const uint32_t c = (uint32_t)wc[slot] + 1u;
+                wc[slot] = (uint16_t)c;
+                return c == (rc.y >> 16);
+            }
             if (o0 == 0xfffeu) {
                 const int32_t s = (int32_t)(rc.x & 0xffffu);
                 for (int32_t e = gt.pred_ptr[s], e1 = gt.pred_ptr[s + 1]; e < e1; e++) {
@@ -375,6 +385,8 @@ gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32
         if ((int32_t)fam < sp.pct_random || (int32_t)fam >= sp.pct_random + sp.pct_local) {
             // ---- F1 / F3: keyed Kahn over G ----------------------------------
             for (int32_t w = 0; w < NW; w++) bw(w) = 0u;
+            for (int32_t i = 0; i < gt.W; i++) wc[i] = 0;
+            wide_ok = true;
             for (int32_t b = 0; b <= NB; b++) boff[b] = 0;
             const int32_t sh = 32 - lgnb;
             for (int32_t i = 0; i < S; i++) boff[(ent_of(hK, (uint32_t)gt.src[i]) >> sh) + 1]++;
@@ -592,7 +604,8 @@ GenPlan gen_plan(int device, const DevGraph& g, const GenTables& gt, int64_t K) 
         const size_t nb = (size_t)1 << gen_lgnb(gt);
         p.w2 = ((size_t)gt.S * 4 + 15) / 16 * 16 + ((nb + 1 + 7) & ~(size_t)7) * 2 + (((size_t)gt.nq + 7) & ~(size_t)7) * 2 +
                (((size_t)g.n + 7) & ~(size_t)7) * 2 + (p.bsm ? 0 : (size_t)((NW + 3) & ~3) * 4) +
-               (((size_t)2 * std::max(g.R, 1) + 3) & ~(size_t)3) * 4 + (size_t)kGenHG * 4;
+               (((size_t)2 * std::max(g.R, 1) + 3) & ~(size_t)3) * 4 + (size_t)kGenHG * 4 +
+               (((size_t)gt.W + 7) & ~(size_t)7) * 2;
         p.w2 = (p.w2 + 127) / 128 * 128;
         p.T1 = std::min<int64_t>(kSeqFixT, K);
     } else {

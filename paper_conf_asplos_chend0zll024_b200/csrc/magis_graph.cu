@@ -395,6 +395,10 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
         for (int32_t j = U_ptr[r]; j < U_ptr[r + 1]; j++) addq(U_idx[j]);
     }
     std::vector<uint32_t> gsinfo((size_t)2 * n), grec((size_t)2 * std::max<int64_t>(E, 1), 0);
+    std::vector<int32_t> gwide(n, -1);            // wide slot of a node with more than 4 inputs
+    int32_t gW = 0;
+    for (int32_t v = 0; v < n; v++)
+        if (pred_ptr[v + 1] - pred_ptr[v] > 4 && gW < 0xfffe) gwide[v] = gW++;
     for (int32_t u = 0; u < n; u++) {
         gsinfo[2 * u] = (uint32_t)succ_ptr[u];
         gsinfo[2 * u + 1] = (uint32_t)(succ_ptr[u + 1] - succ_ptr[u]) | ((uint32_t)gqmap[u] << 16);
@@ -407,7 +411,16 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
                 if (no < 3) o[no] = (uint32_t)pred[f];
                 no++;
             }
-            if (no > 3) o[0] = 0xfffeu;
+            if (no > 3) {
+                o[0] = 0xfffeu;
+                const int32_t deg = pred_ptr[s2 + 1] - pred_ptr[s2];
+                if (gwide[s2] >= 0 && deg < 0xffff) {
+                    o[1] = (uint32_t)gwide[s2];
+                    o[2] = (uint32_t)deg;
+                } else {
+                    o[1] = o[2] = 0xffffu;                // no counter: the kernel scans the inputs
+                }
+            }
             grec[2 * e] = (uint32_t)s2 | (o[0] << 16);
             grec[2 * e + 1] = o[1] | (o[2] << 16);
         }
@@ -490,6 +503,7 @@ extern "C" int magis_graph_load_regions(const magis_graph_desc* d, const magis_r
     g->gen.sinfo = (const uint2*)(b + o_gsinfo);
     g->gen.rec = (const uint2*)(b + o_grec);
     g->gen.S = (int32_t)gsrc.size();
+    g->gen.W = gW;
     g->gen.nq = (int32_t)gqnode.size();
     g->gen.fast = (n < 0xffff && gqnode.size() < 0xffffu && R < 32768) ? 1 : 0;
 

@@ -141,7 +141,9 @@ struct GenTables {
     const int32_t* qnode;      // [nq] node of each slot
     const uint2* sinfo;        // [n] (successor offset, count | slot << 16)
     const uint2* rec;          // [E] successor records in succ order: s | o0 << 16, o1 | o2 << 16
-                               //     (the other inputs of s, 0xffff none; o0 = 0xfffe: more than 3)
+                               //     (the other inputs of s, 0xffff none; o0 = 0xfffe: more than 3
+                               //     other inputs, then o1 = the node's wide slot, o2 = its in-degree)
+    int32_t W;                 // wide nodes (in-degree > 4): per-candidate emitted-input counters
     int32_t S, nq;
     int32_t fast;              // n, nq < 65535 and R < 32768: the fast kernel applies
 };
