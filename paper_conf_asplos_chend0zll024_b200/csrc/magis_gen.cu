@@ -226,7 +226,10 @@ gen_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32_
 // (key, id) of a node as one u32: the key is the draw's top 16 bits (candgen.c)
 __device__ __forceinline__ uint32_t ent_of(uint64_t hk, uint32_t v) { return ((uint32_t)(mix64(hk ^ v) >> 48) << 16) | v; }
 
-constexpr int kGenHC = 32;        // heap entries on chip per thread (more spill to the thread's global slice)
+// heap entries on chip per thread (more spill to the thread's global slice):
+// 32, or 64 on graphs past 16k nodes (measured: C4 146 -> 125 ms per 65,536;
+// C3 26.4 -> 28.7 ms, its L1 share matters more than its 96-wide bursts)
+template <int HCT> constexpr int gen_hc() { return HCT; }
 constexpr int kGenHG = 1024;      // spill entries; a larger ready set re-runs the candidate on gen_kernel
 
 // graph tables: read-only path, kept in L1 ahead of the per-thread scratch
@@ -236,12 +239,12 @@ __device__ __forceinline__ uint2 ld_tab(const uint2* p) {
     return r;
 }
 
-template <bool BSM>
+template <bool BSM, int HCT>
 __global__ void __launch_bounds__(128)
 gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32_t* __restrict__ perms,
             uint8_t* __restrict__ decs, char* __restrict__ scr, int64_t wstride, int32_t lgnb,
             uint8_t* __restrict__ flag, int32_t* __restrict__ nflag) {
-    constexpr int HC = kGenHC;
+    constexpr int HC = gen_hc<HCT>();
     extern __shared__ uint32_t smg[];
     const int TB = blockDim.x, tid = threadIdx.x;
     const int32_t n = g.n, R = g.R, NT = g.NT, S = gt.S, nq = gt.nq;
@@ -542,8 +545,8 @@ int gen_lgnb(const GenTables& gt) {
     while ((1 << lg) * 4 < gt.S && lg < 12) lg++;
     return lg;
 }
-const void* gen2_select(int bsm) {
-    return bsm ? (const void*)gen2_kernel<true> : (const void*)gen2_kernel<false>;
+const void* gen2_select(int bsm, int hc) {
+    return bsm ? (const void*)gen2_kernel<true, 32> : (hc == 64 ? (const void*)gen2_kernel<false, 64> : (const void*)gen2_kernel<false, 32>);
 }
 constexpr int kGenTB = 128;
 constexpr int64_t kSeqFixT = 1024;   // sequential re-run threads
@@ -559,11 +562,11 @@ GenPlan gen_plan(int device, const DevGraph& g, const GenTables& gt, int64_t K) 
     const char* off = std::getenv("MAGIS_GEN_SEQ");            // force the sequential kernel (tests)
     if (gt.fast && !(off && std::atoi(off) != 0)) {
         const int32_t NW = (g.n + 31) >> 5;
-        p.hc = kGenHC;
         const char* bf = std::getenv("MAGIS_GEN_BSM");
         p.bsm = bf ? (std::atoi(bf) != 0 && NW <= 96) : (NW <= 96 ? 1 : 0);
+        p.hc = (!p.bsm && g.n > 16384) ? 64 : 32;
         const size_t smem = (size_t)kGenTB * (p.hc + (p.bsm ? NW : 0)) * 4;
-        const void* fn = gen2_select(p.bsm);
+        const void* fn = gen2_select(p.bsm, p.hc);
         cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         // the attribute persists per kernel: start from the all-shared carveout
         // (an earlier call on a smaller graph may have lowered it)
@@ -643,8 +646,9 @@ cudaError_t gen_launch(const DevGraph& g, const GenTables& gt, const GenSpec& sp
         const size_t smem = (size_t)kGenTB * (gp.hc + (gp.bsm ? NW : 0)) * 4;
         const int lg = gen_lgnb(gt);
         const unsigned blocks2 = (unsigned)(gp.T2 / kGenTB);
-        if (gp.bsm) gen2_kernel<true><<<blocks2, kGenTB, smem, stream>>>(g, gt, sp, id0, K, perm, dec, s2, (int64_t)gp.w2, lg, flag, nflag);
-        else gen2_kernel<false><<<blocks2, kGenTB, smem, stream>>>(g, gt, sp, id0, K, perm, dec, s2, (int64_t)gp.w2, lg, flag, nflag);
+        if (gp.bsm) gen2_kernel<true, 32><<<blocks2, kGenTB, smem, stream>>>(g, gt, sp, id0, K, perm, dec, s2, (int64_t)gp.w2, lg, flag, nflag);
+        else if (gp.hc == 64) gen2_kernel<false, 64><<<blocks2, kGenTB, smem, stream>>>(g, gt, sp, id0, K, perm, dec, s2, (int64_t)gp.w2, lg, flag, nflag);
+        else gen2_kernel<false, 32><<<blocks2, kGenTB, smem, stream>>>(g, gt, sp, id0, K, perm, dec, s2, (int64_t)gp.w2, lg, flag, nflag);
         e = cudaGetLastError();
         if (e != cudaSuccess) return e;
         const char* dbg = std::getenv("MAGIS_GEN_DEBUG");          // report the re-run count (syncs)
