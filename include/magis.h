@@ -276,12 +276,15 @@ int magis_eval_schedules_host_delta4(magis_graph* g, int64_t K, const uint8_t* h
  * application + re-ordering (§5.2, Alg. 2; DESIGN.md
  * §5): per eligible tensor a decision (re-mat with probability
  * p_remat/10000 if the tensor has inputs, else swap with p_swap/10000);
- * pct_random % random-priority Kahn orders, pct_local % local moves (a window
- * of <= wmax natural-order steps re-ordered by the same keyed Kahn), the rest
- * a random order with one random transposition (may be invalid); Stores right
- * after their producer, Loads / clones 0..slack steps before the
- * first late user, inactive optional nodes last.
- * d_perm [K x n_total] int32, d_dec [K x max(R,1)] uint8: device memory, caller-owned.
+ * pct_random % random-priority Kahn orders (the ready node of smallest
+ * (16-bit priority, id) first), pct_local % local moves (a window of <= wmax
+ * natural-order steps re-ordered by the same keyed Kahn), the rest a random
+ * order with one random transposition (may be invalid); Stores right after
+ * their producer, Loads / clones 0..slack steps before the first
+ * late user, inactive optional nodes last.  Byte-identical to the C generator
+ * magis_inputs/csrc/candgen.c (the test side).
+ * d_perm [K x n_total] int32, d_dec [K x max(R,1)] uint8 (R = 0: one zero pad
+ * byte per row): device memory, caller-owned.
  * Asynchronous on the stream.  The first call allocates graph-owned scratch.
  * Errors: MAGIS_E_INVAL (K < 0, null pointer, bad spec), MAGIS_E_NOMEM / MAGIS_E_CUDA.
  */
