@@ -376,12 +376,27 @@ gen2_kernel(DevGraph g, GenTables gt, GenSpec sp, uint64_t id0, int64_t K, int32
             const uint2 si = ld_tab(gt.sinfo + u);
             const uint32_t cnt = si.y & 0xffffu, qs = si.y >> 16;
             if (qs != 0xffffu) Q[qs] = (uint16_t)m;
-            for (uint32_t e = 0; e < cnt; e++) {
-                const uint2 rc = ld_tab(gt.rec + si.x + e);
-                const int32_t s = (int32_t)(rc.x & 0xffffu);
-                if (s >= hi || !ready(rc, u, lo)) continue;
-                if (nh >= HC + kGenHG) { over = true; return; }
-                push(ent_of(hK, (uint32_t)s));
+            // successors 4 at a time: the records, then the readiness tests of
+            // all 4 (independent loads), then the pushes (the emitted set does
+            // not change inside one node's visit, and the pop order depends on
+            // the keys only, not on the order of pushes)
+            for (uint32_t e0 = 0; e0 < cnt; e0 += 4) {
+                uint2 rc[4];
+#pragma unroll
+                for (int k = 0; k < 4; k++)
+                    rc[k] = e0 + k < cnt ? ld_tab(gt.rec + si.x + e0 + k) : make_uint2(0xffffu, 0u);
+                bool rd[4];
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    const int32_t s = (int32_t)(rc[k].x & 0xffffu);
+                    rd[k] = e0 + k < cnt && s < hi && ready(rc[k], u, lo);
+                }
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    if (!rd[k]) continue;
+                    if (nh >= HC + kGenHG) { over = true; return; }
+                    push(ent_of(hK, rc[k].x & 0xffffu));
+                }
             }
         };
         int32_t lo = 0, hi = n;
