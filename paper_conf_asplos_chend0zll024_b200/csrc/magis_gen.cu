@@ -578,7 +578,7 @@ GenPlan gen_plan(int device, const DevGraph& g, const GenTables& gt, int64_t K) 
     if (gt.fast && !(off && std::atoi(off) != 0)) {
         const int32_t NW = (g.n + 31) >> 5;
         const char* bf = std::getenv("MAGIS_GEN_BSM");
-        p.bsm = bf ? (std::atoi(bf) != 0 && NW <= 96) : (NW <= 96 ? 1 : 0);
+        p.bsm = bf ? (std::atoi(bf) != 0 && NW <= 384) : (NW <= 96 ? 1 : 0);
         p.hc = (!p.bsm && g.n > 16384) ? 64 : 32;
         const size_t smem = (size_t)kGenTB * (p.hc + (p.bsm ? NW : 0)) * 4;
         const void* fn = gen2_select(p.bsm, p.hc);
