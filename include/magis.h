@@ -285,7 +285,9 @@ int magis_eval_schedules_host_delta4(magis_graph* g, int64_t K, const uint8_t* h
  * magis_inputs/csrc/candgen.c (the test side).
  * d_perm [K x n_total] int32, d_dec [K x max(R,1)] uint8 (R = 0: one zero pad
  * byte per row): device memory, caller-owned.
- * Asynchronous on the stream.  The first call allocates graph-owned scratch.
+ * Asynchronous on the stream.  The first call allocates graph-owned scratch
+ * (grown when a later call needs more), so calls on one graph must not overlap
+ * in time on different streams.
  * Errors: MAGIS_E_INVAL (K < 0, null pointer, bad spec), MAGIS_E_NOMEM / MAGIS_E_CUDA.
  */
 typedef struct magis_gen_spec {
