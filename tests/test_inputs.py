@@ -112,3 +112,48 @@ def test_big_graph_sizes(cfg):
     else:
         assert 16384 < s["n_total"] <= 30000       # multi-CTA-sized graph
         assert s["sum_bytes"] > 2 ** 31
+
+
+def test_random_orders_follow_the_keyed_kahn_recipe():
+    """F1 candidates are the keyed Kahn order of the recipe (candgen.c header,
+    DESIGN §5): at every step the ready node with the smallest (priority, id),
+    priority = the top 16 bits of rnd(seed, k, KEY, v), rnd = three SplitMix64
+    mixes.  Written here from the recipe, independently of candgen.c; the
+    device generator is held byte-identical to candgen.c by the GPU tests."""
+    import heapq
+    M = (1 << 64) - 1
+
+    def mix(x):
+        x = (x + 0x9E3779B97F4A7C15) & M
+        x = ((x ^ (x >> 30)) * 0xBF58476D1CE4E5B9) & M
+        x = ((x ^ (x >> 27)) * 0x94D049BB133111EB) & M
+        return x ^ (x >> 31)
+
+    def rnd(seed, k, stream, i):
+        h = mix((seed + 0x9E3779B97F4A7C15 * (stream + 1)) & M)
+        return mix(mix(h ^ k) ^ i)
+
+    wl = build_workload("c2")
+    n, seed = wl.n, 21
+    spec = CandidateSpec(seed=seed, pct_random=100, pct_local=0, p_remat=0, p_swap=0)
+    P, _ = CandidateGenerator(wl, spec).generate(40, 6)
+    preds = [[] for _ in range(n)]
+    succs = [[] for _ in range(n)]
+    for u, v in set(zip(wl.src.tolist(), wl.dst.tolist())):
+        preds[v].append(u)
+        succs[u].append(v)
+    for i in range(6):
+        k = 40 + i
+        key = [rnd(seed, k, 3, v) >> 48 for v in range(n)]
+        indeg = [len(p) for p in preds]
+        ready = [(key[v], v) for v in range(n) if indeg[v] == 0]
+        heapq.heapify(ready)
+        order = []
+        while ready:
+            _, u = heapq.heappop(ready)
+            order.append(u)
+            for s in succs[u]:
+                indeg[s] -= 1
+                if indeg[s] == 0:
+                    heapq.heappush(ready, (key[s], s))
+        assert P[i, :n].tolist() == order
